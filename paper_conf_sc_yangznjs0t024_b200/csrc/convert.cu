@@ -1,0 +1,507 @@
+// convert.cu -- CSR -> two-level tile format on the GPU (Section III-B),
+// per-nonzero precision criterion (Section II-A), per-tile precision, range floor,
+// the SELL-16 kernel layout with lower-precision value planes ("convert once, reuse"),
+// and the persistent-kernel launch plan (P:130-132 task distribution, balanced on nnz+tiles).
+//
+// One half-warp owns one tile row (16 matrix rows, lane r = row 16*TR + r) and merges its 16
+// sorted rows tile column by tile column, so tiles come out in (row, col) order without a sort.
+// Two passes with the same merge: COUNT (sizes per tile row) -> exclusive scans -> FILL.
+#include <cuda_runtime.h>
+#include <stdio.h>
+
+#include <algorithm>
+#include <vector>
+
+#include "mf_internal.cuh"
+
+namespace mf {
+namespace {
+
+constexpr int CNT_TILES = 0, CNT_ROWS = 1, CNT_WIDTH = 2, CNT_NNZP = 3 /*..6*/, CNT_TILEP = 7 /*..10*/;
+constexpr int NCNT = 11;
+constexpr int THREADS = 256;
+
+__device__ __forceinline__ unsigned hw_mask() { return (threadIdx.x & 16) ? 0xFFFF0000u : 0x0000FFFFu; }
+
+template <class T>
+__device__ __forceinline__ T hw_min(T v, unsigned m) {
+    for (int o = 8; o >= 1; o >>= 1) { T u = __shfl_xor_sync(m, v, o); v = u < v ? u : v; }
+    return v;
+}
+template <class T>
+__device__ __forceinline__ T hw_max(T v, unsigned m) {
+    for (int o = 8; o >= 1; o >>= 1) { T u = __shfl_xor_sync(m, v, o); v = u > v ? u : v; }
+    return v;
+}
+template <class T>
+__device__ __forceinline__ T hw_sum(T v, unsigned m) {
+    for (int o = 8; o >= 1; o >>= 1) v += __shfl_xor_sync(m, v, o);
+    return v;
+}
+// exclusive prefix sum over the 16 lanes of the half-warp
+template <class T>
+__device__ __forceinline__ T hw_excl_scan(T v, unsigned m, int lane16) {
+    T incl = v;
+    for (int o = 1; o < 16; o <<= 1) {
+        T u = __shfl_up_sync(m, incl, o, 16);
+        if (lane16 >= o) incl += u;
+    }
+    return incl - v;
+}
+
+// Per-nonzero class: lowest of {FP8, FP16, FP32} whose single-RNE rounding loses less
+// than loss_tol*|v| (relative reading); v == 0 -> FP8.  No contraction: explicit _rn ops.
+__device__ __forceinline__ int classify(double v, double loss_tol) {
+    if (v == 0.0) return 3;
+    double thr = __dmul_rn(loss_tol, fabs(v));
+    if (fabs(__dsub_rn(v, mfk::e4m3_to_d(mfk::to_e4m3(v)))) < thr) return 3;
+    if (fabs(__dsub_rn(v, mfk::f16_to_d(mfk::to_f16(v)))) < thr) return 2;
+    if (fabs(__dsub_rn(v, (double)mfk::to_f32(v))) < thr) return 1;
+    return 0;
+}
+
+// lowest-precision format whose normal range holds |sv|; zeros are neutral (3)
+__device__ __forceinline__ int range_class(double sv) {
+    double a = fabs(sv);
+    if (a == 0.0) return 3;
+    if (a >= 0x1p-6 && a <= 448.0) return 3;
+    if (a >= 0x1p-14 && a <= 65504.0) return 2;
+    if (a >= 0x1p-126 && a <= 3.4028234663852886e38) return 1;
+    return 0;
+}
+
+__global__ void validate_kernel(int64_t n_rows, int64_t n_cols, int64_t nnz, const int64_t* __restrict__ rowptr,
+                                const int32_t* __restrict__ colidx, const double* __restrict__ vals, int* err) {
+    int64_t stride = (int64_t)gridDim.x * blockDim.x;
+    for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < n_rows; i += stride) {
+        int64_t a = rowptr[i], b = rowptr[i + 1];
+        if ((i == 0 && a != 0) || (i == n_rows - 1 && b != nnz) || b < a || a < 0 || b > nnz) {
+            atomicOr(err, 1);
+            continue;
+        }
+        for (int64_t k = a; k < b; ++k) {
+            int32_t c = colidx[k];
+            if (c < 0 || c >= n_cols) atomicOr(err, 1);
+            else if (k > a && c <= colidx[k - 1]) atomicOr(err, 2);
+            if (!isfinite(vals[k])) atomicOr(err, 4);
+        }
+    }
+}
+
+struct Out {  // FILL-pass destinations (all device)
+    int32_t *TileRowidx, *TileColidx;
+    uint8_t *TilePrec, *Floor;
+    int64_t *TileNnz, *Nonrow, *ValOff, *TileRowPtr;
+    uint8_t *RowIndex, *CsrRowptr, *CsrColidx;
+    double* Val64; float* Val32; uint16_t* Val16; uint8_t* Val8;
+    uint32_t* tile_info; uint16_t* sidx;
+    double* p64; float* p32; __half* p16; uint8_t* p8;
+    const int64_t* off;   // [NCNT][ntr+1] exclusive scans of the counts
+    int64_t ntr;
+};
+
+// The merge of one tile row.  FILL == false: write counts; FILL == true: write the arrays.
+template <bool FILL>
+__global__ void __launch_bounds__(THREADS) tile_row_kernel(int64_t n_rows, int64_t ntr, const int64_t* __restrict__ rowptr,
+                                                           const int32_t* __restrict__ colidx,
+                                                           const double* __restrict__ vals, int classify_on,
+                                                           double loss_tol, int64_t* cnt, int* err, Out o) {
+    const unsigned m = hw_mask();
+    const int lane = threadIdx.x & 15;
+    const int64_t TR = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 4;
+    if (TR >= ntr) return;                       // uniform per half-warp
+    const int64_t row = TR * TS + lane;
+    const bool valid = row < n_rows;
+    const int64_t rstart = valid ? rowptr[row] : 0;
+    const int64_t rend = valid ? rowptr[row + 1] : 0;
+    int64_t ptr = rstart;
+    int cur = ptr < rend ? (colidx[ptr] >> 4) : INT32_MAX;
+    const int64_t width = hw_max<int64_t>(rend - rstart, m);
+
+    int64_t j = 0, nz_run = 0, ri_run = 0;
+    int64_t pnnz[4] = {0, 0, 0, 0}, ptile[4] = {0, 0, 0, 0};
+    int64_t tile0 = 0, row0 = 0, nnz0 = 0, slot0 = 0, voff[4] = {0, 0, 0, 0};
+    if (FILL) {
+        const int64_t S = ntr + 1;
+        tile0 = o.off[CNT_TILES * S + TR];
+        row0 = o.off[CNT_ROWS * S + TR];
+        slot0 = o.off[CNT_WIDTH * S + TR];
+        for (int q = 0; q < 4; ++q) voff[q] = o.off[(CNT_NNZP + q) * S + TR];
+        nnz0 = rowptr[TR * TS];
+        if (lane == 0) o.TileRowPtr[TR] = tile0;
+        if (lane == 0 && TR == ntr - 1) o.TileRowPtr[ntr] = tile0 + o.off[CNT_TILES * S + ntr] - tile0;
+    }
+    while (true) {
+        const int tc = hw_min<int>(cur, m);
+        if (tc == INT32_MAX) break;
+        const bool mine = (cur == tc);
+        int64_t q = ptr;
+        int cls = classify_on ? 3 : 0;
+        if (mine) {
+            while (q < rend && (colidx[q] >> 4) == tc) {
+                if (classify_on) { int c = classify(vals[q], loss_tol); cls = c < cls ? c : cls; }
+                ++q;
+            }
+        }
+        const int cnt_r = (int)(q - ptr);
+        const int best = hw_min<int>(mine ? cls : 3, m);        // TilePrec: highest needed precision
+        int rc = 3;
+        if (mine)
+            for (int64_t k = ptr; k < q; ++k) { int c = range_class(mfk::round_to(vals[k], best)); rc = c < rc ? c : rc; }
+        const int minrc = hw_min<int>(rc, m);
+        const int floor_t = minrc > best ? minrc : best;
+        const int tile_nz = hw_sum<int>(cnt_r, m);
+        const unsigned bal = __ballot_sync(m, mine) >> (threadIdx.x & 16);
+        const int rows_in_tile = __popc(bal);
+        if (FILL) {
+            const int64_t t = tile0 + j;
+            const int csr_off = hw_excl_scan<int>(cnt_r, m, lane);
+            const int ri_loc = __popc(bal & ((1u << lane) - 1u));
+            const int64_t vbase = voff[best] + pnnz[best];
+            if (lane == 0) {
+                o.TileRowidx[t] = (int32_t)TR;
+                o.TileColidx[t] = tc;
+                o.TilePrec[t] = (uint8_t)best;
+                o.Floor[t] = (uint8_t)floor_t;
+                o.TileNnz[t] = nnz0 + nz_run;
+                o.Nonrow[t] = row0 + ri_run;
+                o.ValOff[t] = vbase;
+                o.tile_info[t] = ((uint32_t)tc << 4) | ((uint32_t)floor_t << 2) | (uint32_t)best;
+            }
+            if (mine) {
+                const int64_t ri = row0 + ri_run + ri_loc;
+                o.RowIndex[ri] = (uint8_t)lane;
+                o.CsrRowptr[ri] = (uint8_t)csr_off;
+                for (int64_t k = ptr; k < q; ++k) {
+                    const int a = csr_off + (int)(k - ptr);
+                    const double v = vals[k];
+                    const int lc = colidx[k] & 15;
+                    o.CsrColidx[nnz0 + nz_run + a] = (uint8_t)lc;
+                    const int64_t vp = vbase + a;
+                    double sv;
+                    switch (best) {
+                    case 0: o.Val64[vp] = v; sv = v; break;
+                    case 1: { float f = mfk::to_f32(v); o.Val32[vp] = f; sv = (double)f; } break;
+                    case 2: { __half h = mfk::to_f16(v); o.Val16[vp] = __half_as_ushort(h); sv = mfk::f16_to_d(h); } break;
+                    default: { uint8_t b = mfk::to_e4m3(v); o.Val8[vp] = b; sv = mfk::e4m3_to_d(b); } break;
+                    }
+                    // kernel layout: slot (k - rstart) of this row, value planes RNE_q(stored), q >= TilePrec
+                    const int64_t pos = (slot0 + (k - rstart)) * TS + lane;
+                    o.sidx[pos] = (uint16_t)((j << 4) | lc);
+                    if (best <= 0 && o.p64) o.p64[pos] = sv;
+                    if (best <= 1 && o.p32) o.p32[pos] = mfk::to_f32(sv);
+                    if (best <= 2 && o.p16) o.p16[pos] = mfk::to_f16(sv);
+                    if (o.p8) o.p8[pos] = mfk::to_e4m3(sv);
+                }
+            }
+        }
+        if (mine) { ptr = q; cur = ptr < rend ? (colidx[ptr] >> 4) : INT32_MAX; }
+        ++j;
+        nz_run += tile_nz;
+        ri_run += rows_in_tile;
+        pnnz[best] += tile_nz;
+        ptile[best] += 1;
+    }
+    if (FILL) {
+        if (lane == 0 && TR == ntr - 1) {
+            o.TileNnz[tile0 + j] = nnz0 + nz_run;
+            o.Nonrow[tile0 + j] = row0 + ri_run;
+        }
+    } else if (lane == 0) {
+        cnt[CNT_TILES * ntr + TR] = j;
+        cnt[CNT_ROWS * ntr + TR] = ri_run;
+        cnt[CNT_WIDTH * ntr + TR] = width;
+        for (int q = 0; q < 4; ++q) {
+            cnt[(CNT_NNZP + q) * ntr + TR] = pnnz[q];
+            cnt[(CNT_TILEP + q) * ntr + TR] = ptile[q];
+        }
+        if (j > MAX_TILES_PER_TR) atomicOr(err, 8);
+    }
+}
+
+// ------------------------------------------------------------------ exclusive scan (int64)
+constexpr int SCAN_T = 1024, SCAN_CHUNK = 2 * SCAN_T;
+
+__device__ int64_t block_incl_scan(int64_t v, int64_t* sh) {
+    const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
+    for (int o = 1; o < 32; o <<= 1) { int64_t u = __shfl_up_sync(0xffffffffu, v, o); if (lane >= o) v += u; }
+    if (lane == 31) sh[w] = v;
+    __syncthreads();
+    if (w == 0) {
+        int64_t s = lane < (int)(blockDim.x >> 5) ? sh[lane] : 0;
+        for (int o = 1; o < 32; o <<= 1) { int64_t u = __shfl_up_sync(0xffffffffu, s, o); if (lane >= o) s += u; }
+        sh[lane] = s;
+    }
+    __syncthreads();
+    if (w > 0) v += sh[w - 1];
+    __syncthreads();
+    return v;
+}
+
+__global__ void scan_block_sums(const int64_t* __restrict__ in, int64_t n, int64_t* bsum) {
+    __shared__ int64_t sh[32];
+    int64_t base = (int64_t)blockIdx.x * SCAN_CHUNK;
+    int64_t a = base + 2 * threadIdx.x;
+    int64_t v = (a < n ? in[a] : 0) + (a + 1 < n ? in[a + 1] : 0);
+    v = block_incl_scan(v, sh);
+    if (threadIdx.x == blockDim.x - 1) bsum[blockIdx.x] = v;
+}
+
+__global__ void scan_sums_serial(int64_t* bsum, int64_t nb) {   // one block: exclusive scan in place
+    __shared__ int64_t sh[32];
+    __shared__ int64_t carry;
+    if (threadIdx.x == 0) carry = 0;
+    __syncthreads();
+    for (int64_t c = 0; c < nb; c += blockDim.x) {
+        int64_t i = c + threadIdx.x;
+        int64_t v = i < nb ? bsum[i] : 0;
+        int64_t incl = block_incl_scan(v, sh);
+        int64_t cr = carry;
+        if (i < nb) bsum[i] = cr + incl - v;
+        __syncthreads();
+        if (threadIdx.x == blockDim.x - 1) carry = cr + incl;
+        __syncthreads();
+    }
+}
+
+__global__ void scan_apply(const int64_t* __restrict__ in, int64_t n, const int64_t* __restrict__ bsum, int64_t* out) {
+    __shared__ int64_t sh[32];
+    int64_t base = (int64_t)blockIdx.x * SCAN_CHUNK;
+    int64_t a = base + 2 * threadIdx.x;
+    int64_t x0 = a < n ? in[a] : 0, x1 = a + 1 < n ? in[a + 1] : 0;
+    int64_t incl = block_incl_scan(x0 + x1, sh);
+    int64_t excl = bsum[blockIdx.x] + incl - (x0 + x1);
+    if (a < n) out[a] = excl;
+    if (a + 1 < n) out[a + 1] = excl + x0;
+    if (a + 1 == n - 1 || (a == n - 1)) out[n] = excl + x0 + x1;   // total
+    if (n == 0 && blockIdx.x == 0 && threadIdx.x == 0) out[0] = 0;
+}
+
+// out[0..n] = exclusive scan of in[0..n), out[n] = total
+mf_status scan_excl(const int64_t* in, int64_t n, int64_t* out, int64_t* tmp, cudaStream_t s) {
+    int64_t nb = (n + SCAN_CHUNK - 1) / SCAN_CHUNK;
+    if (n == 0) { MF_CUDA(cudaMemsetAsync(out, 0, sizeof(int64_t), s)); return MF_OK; }
+    scan_block_sums<<<(unsigned)nb, SCAN_T, 0, s>>>(in, n, tmp);
+    scan_sums_serial<<<1, SCAN_T, 0, s>>>(tmp, nb);
+    scan_apply<<<(unsigned)nb, SCAN_T, 0, s>>>(in, n, tmp, out);
+    MF_CUDA(cudaGetLastError());
+    return MF_OK;
+}
+
+// ------------------------------------------------------------------ launch plan
+// cost of a tile row: slice bytes (2 B index + ~2 B value per slot) + vector bytes (48 B per row)
+__global__ void tr_cost_kernel(const int64_t* __restrict__ cnt, int64_t ntr, int64_t n_rows, int64_t* cost) {
+    int64_t TR = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
+    if (TR >= ntr) return;
+    int64_t rows = n_rows - TR * TS < TS ? n_rows - TR * TS : TS;
+    cost[TR] = 4 * TS * cnt[CNT_WIDTH * ntr + TR] + 48 * rows + 1;
+}
+
+// plan_tr[g] = first tile row whose exclusive cost prefix reaches g*total/G
+__global__ void plan_kernel(const int64_t* __restrict__ pre, int64_t ntr, int G, int32_t* plan_tr) {
+    int g = blockIdx.x * blockDim.x + threadIdx.x;
+    if (g > G) return;
+    if (g == 0) { plan_tr[0] = 0; return; }
+    if (g == G) { plan_tr[G] = (int32_t)ntr; return; }
+    int64_t total = pre[ntr];
+    int64_t target = (int64_t)((__int128)total * g / G);
+    int64_t lo = 0, hi = ntr;            // first TR with pre[TR] >= target
+    while (lo < hi) { int64_t mid = (lo + hi) / 2; if (pre[mid] >= target) hi = mid; else lo = mid + 1; }
+    plan_tr[g] = (int32_t)lo;
+}
+
+__device__ int owner_of(const int32_t* plan_tr, int G, int64_t TR) {   // CTA owning tile row TR
+    int lo = 0, hi = G - 1;
+    while (lo < hi) { int mid = (lo + hi + 1) / 2; if (plan_tr[mid] <= TR) lo = mid; else hi = mid - 1; }
+    return lo;
+}
+
+// dependency range: CTAs owning the column segments this CTA's tiles gather (square matrices)
+__global__ void deps_kernel(const int32_t* __restrict__ plan_tr, int G, const int64_t* __restrict__ TileRowPtr,
+                            const int32_t* __restrict__ TileColidx, int64_t n_seg_owned, int32_t* dep_lo, int32_t* dep_hi) {
+    int g = blockIdx.x;
+    __shared__ int smin, smax;
+    if (threadIdx.x == 0) { smin = INT32_MAX; smax = -1; }
+    __syncthreads();
+    int lmin = INT32_MAX, lmax = -1;
+    for (int64_t TR = plan_tr[g] + threadIdx.x; TR < plan_tr[g + 1]; TR += blockDim.x) {
+        int64_t a = TileRowPtr[TR], b = TileRowPtr[TR + 1];
+        if (b > a) { lmin = min(lmin, TileColidx[a]); lmax = max(lmax, TileColidx[b - 1]); }
+    }
+    atomicMin(&smin, lmin);
+    atomicMax(&smax, lmax);
+    __syncthreads();
+    if (threadIdx.x == 0) {
+        int lo = g, hi = g;
+        if (smax >= 0) {
+            // column segments beyond the owned row range (non-square / halo) have no owner CTA
+            int64_t cmin = smin, cmax = smax < n_seg_owned ? smax : n_seg_owned - 1;
+            if (cmin < n_seg_owned) lo = min(lo, owner_of(plan_tr, G, cmin));
+            if (cmax >= 0 && cmin < n_seg_owned) hi = max(hi, owner_of(plan_tr, G, cmax));
+        }
+        dep_lo[g] = lo;
+        dep_hi[g] = hi;
+    }
+}
+
+}  // namespace
+
+void destroy_tiles(TileMatrix* A) {
+    cudaStream_t s = A->owner_stream;
+    void* ptrs[] = {A->TileRowidx, A->TileColidx, A->TilePrec, A->Floor, A->TileNnz, A->Nonrow, A->ValOff,
+                    A->TileRowPtr, A->RowIndex, A->CsrRowptr, A->CsrColidx, A->Val64, A->Val32, A->Val16,
+                    A->Val8, A->tr_slot, A->tile_info, A->sidx, A->plane64, A->plane32, A->plane16,
+                    A->plane8, A->plan_tr, A->dep_lo, A->dep_hi};
+    for (void* p : ptrs) if (p) dev_free(p, s);
+    delete[] A->plan_rows_host;
+    *A = TileMatrix();
+}
+
+mf_status convert_csr(int64_t n_rows, int64_t n_cols, int64_t nnz, const int64_t* rowptr, const int32_t* colidx,
+                      const double* vals, const mf_convert_opts& o, cudaStream_t s, TileMatrix* A) {
+    int sms = 0;
+    MF_TRY(check_device(&sms));
+    A->n_rows = n_rows; A->n_cols = n_cols; A->nnz = nnz; A->owner_stream = s;
+    A->ntr = (n_rows + TS - 1) / TS;
+    const int64_t ntr = A->ntr;
+    cudaEvent_t e0, e1;
+    MF_CUDA(cudaEventCreate(&e0));
+    MF_CUDA(cudaEventCreate(&e1));
+    MF_CUDA(cudaEventRecord(e0, s));
+
+    // 1. validation (before any other device work)
+    int* d_err = nullptr;
+    MF_TRY(alloc(&d_err, 1, s));
+    MF_CUDA(cudaMemsetAsync(d_err, 0, sizeof(int), s));
+    if (n_rows > 0) {
+        int blocks = (int)std::min<int64_t>((n_rows + 255) / 256, 4 * 148 * 8);
+        validate_kernel<<<blocks, 256, 0, s>>>(n_rows, n_cols, nnz, rowptr, colidx, vals, d_err);
+        MF_CUDA(cudaGetLastError());
+    }
+    int h_err = 0;
+    MF_CUDA(cudaMemcpyAsync(&h_err, d_err, sizeof(int), cudaMemcpyDeviceToHost, s));
+    MF_CUDA(cudaStreamSynchronize(s));
+    if (h_err & 1) { dev_free(d_err, s); return fail(MF_ERR_INVALID_ARG, "CSR rowptr/colidx out of range or not monotone"); }
+    if (h_err & 2) { dev_free(d_err, s); return fail(MF_ERR_UNSORTED_CSR, "columns not strictly increasing within a row"); }
+    if (h_err & 4) { dev_free(d_err, s); return fail(MF_ERR_NONFINITE, "non-finite matrix value"); }
+
+    // 2. COUNT pass
+    int64_t *cnt = nullptr, *off = nullptr, *tmp = nullptr;
+    const int64_t S = ntr + 1;
+    MF_TRY(alloc(&cnt, (size_t)NCNT * std::max<int64_t>(ntr, 1), s));
+    MF_TRY(alloc(&off, (size_t)NCNT * S, s));
+    MF_TRY(alloc(&tmp, (size_t)(ntr / SCAN_CHUNK + 2), s));
+    const int tr_per_block = THREADS / 16;
+    const unsigned tblocks = (unsigned)std::max<int64_t>((ntr + tr_per_block - 1) / tr_per_block, 1);
+    Out none{};
+    if (ntr > 0) {
+        tile_row_kernel<false><<<tblocks, THREADS, 0, s>>>(n_rows, ntr, rowptr, colidx, vals, o.classify, o.loss_tol,
+                                                            cnt, d_err, none);
+        MF_CUDA(cudaGetLastError());
+    }
+    for (int c = 0; c < NCNT; ++c) MF_TRY(scan_excl(cnt + c * ntr, ntr, off + c * S, tmp, s));
+    std::vector<int64_t> tot(NCNT);
+    for (int c = 0; c < NCNT; ++c)
+        MF_CUDA(cudaMemcpyAsync(&tot[c], off + c * S + ntr, sizeof(int64_t), cudaMemcpyDeviceToHost, s));
+    MF_CUDA(cudaMemcpyAsync(&h_err, d_err, sizeof(int), cudaMemcpyDeviceToHost, s));
+    MF_CUDA(cudaStreamSynchronize(s));
+    if (h_err & 8) {
+        dev_free(d_err, s); dev_free(cnt, s); dev_free(off, s); dev_free(tmp, s);
+        return fail(MF_ERR_UNSUPPORTED, "a tile row holds more than 4096 tiles");
+    }
+    A->tilenum = tot[CNT_TILES];
+    A->rownum = tot[CNT_ROWS];
+    A->slots = tot[CNT_WIDTH];
+    for (int q = 0; q < 4; ++q) { A->nval[q] = tot[CNT_NNZP + q]; A->tiles_per_prec[q] = tot[CNT_TILEP + q]; }
+
+    // 3. allocate
+    const int64_t nt = A->tilenum, nslot = A->slots * TS;
+    MF_TRY(alloc(&A->TileRowidx, nt, s)); MF_TRY(alloc(&A->TileColidx, nt, s));
+    MF_TRY(alloc(&A->TilePrec, nt, s)); MF_TRY(alloc(&A->Floor, nt, s));
+    MF_TRY(alloc(&A->TileNnz, nt + 1, s)); MF_TRY(alloc(&A->Nonrow, nt + 1, s));
+    MF_TRY(alloc(&A->ValOff, nt, s)); MF_TRY(alloc(&A->TileRowPtr, ntr + 1, s));
+    MF_TRY(alloc(&A->RowIndex, A->rownum, s)); MF_TRY(alloc(&A->CsrRowptr, A->rownum, s));
+    MF_TRY(alloc(&A->CsrColidx, nnz, s));
+    MF_TRY(alloc(&A->Val64, A->nval[0], s)); MF_TRY(alloc(&A->Val32, A->nval[1], s));
+    MF_TRY(alloc(&A->Val16, A->nval[2], s)); MF_TRY(alloc(&A->Val8, A->nval[3], s));
+    MF_TRY(alloc(&A->tile_info, nt, s));
+    MF_TRY(alloc(&A->sidx, nslot, s));
+    // value planes: plane q exists when some tile can compute at q (TilePrec <= q)
+    bool need[4] = {false, false, false, false};
+    for (int q = 0; q < 4; ++q)
+        for (int p = 0; p <= q; ++p) if (A->tiles_per_prec[p] > 0) need[q] = true;
+    if (need[0]) MF_TRY(alloc(&A->plane64, nslot, s));
+    if (need[1]) MF_TRY(alloc(&A->plane32, nslot, s));
+    if (need[2]) MF_TRY(alloc(&A->plane16, nslot, s));
+    if (need[3]) MF_TRY(alloc(&A->plane8, nslot, s));
+    if (nslot) MF_CUDA(cudaMemsetAsync(A->sidx, 0xFF, nslot * sizeof(uint16_t), s));
+    if (nt == 0) {
+        MF_CUDA(cudaMemsetAsync(A->TileNnz, 0, sizeof(int64_t), s));
+        MF_CUDA(cudaMemsetAsync(A->Nonrow, 0, sizeof(int64_t), s));
+    }
+    MF_TRY(alloc(&A->tr_slot, ntr + 1, s));
+    MF_CUDA(cudaMemcpyAsync(A->tr_slot, off + CNT_WIDTH * S, (ntr + 1) * sizeof(int64_t), cudaMemcpyDeviceToDevice, s));
+
+    // 4. FILL pass
+    Out fo{A->TileRowidx, A->TileColidx, A->TilePrec, A->Floor, A->TileNnz, A->Nonrow, A->ValOff, A->TileRowPtr,
+           A->RowIndex, A->CsrRowptr, A->CsrColidx, A->Val64, A->Val32, A->Val16, A->Val8, A->tile_info, A->sidx,
+           A->plane64, A->plane32, A->plane16, A->plane8, off, ntr};
+    if (ntr > 0) {
+        tile_row_kernel<true><<<tblocks, THREADS, 0, s>>>(n_rows, ntr, rowptr, colidx, vals, o.classify, o.loss_tol,
+                                                           cnt, d_err, fo);
+        MF_CUDA(cudaGetLastError());
+    } else {
+        MF_CUDA(cudaMemsetAsync(A->TileRowPtr, 0, sizeof(int64_t), s));
+    }
+    // max tiles per tile row (host, from the counts)
+    {
+        std::vector<int64_t> hc(ntr);
+        if (ntr) MF_CUDA(cudaMemcpyAsync(hc.data(), cnt + CNT_TILES * ntr, ntr * sizeof(int64_t), cudaMemcpyDeviceToHost, s));
+        MF_CUDA(cudaStreamSynchronize(s));
+        A->max_nt = ntr ? *std::max_element(hc.begin(), hc.end()) : 0;
+    }
+
+    // 5. launch plan
+    int G = o.grid_ctas, B = o.block_threads;
+    if (B <= 0) B = 1024;
+    if (B % 32 || B > 1024 || B < 32) {
+        return fail(MF_ERR_INVALID_ARG, "block_threads must be a multiple of 32 in [32, 1024]");
+    }
+    if (G <= 0) G = (int)std::max<int64_t>(1, std::min<int64_t>(sms, ntr / 64));
+    if (G > sms * 2) G = sms * 2;
+    if (ntr > 0 && G > ntr) G = (int)ntr;
+    if (G < 1) G = 1;
+    A->G = G; A->B = B;
+    int64_t* cost = nullptr;
+    MF_TRY(alloc(&cost, std::max<int64_t>(ntr, 1), s));
+    if (ntr) tr_cost_kernel<<<(unsigned)((ntr + 255) / 256), 256, 0, s>>>(cnt, ntr, n_rows, cost);
+    MF_TRY(scan_excl(cost, ntr, off, tmp, s));    // reuse off[0..ntr]
+    MF_TRY(alloc(&A->plan_tr, G + 1, s));
+    MF_TRY(alloc(&A->dep_lo, G, s));
+    MF_TRY(alloc(&A->dep_hi, G, s));
+    plan_kernel<<<(G + 1 + 127) / 128, 128, 0, s>>>(off, ntr, G, A->plan_tr);
+    deps_kernel<<<G, 256, 0, s>>>(A->plan_tr, G, A->TileRowPtr, A->TileColidx, ntr, A->dep_lo, A->dep_hi);
+    MF_CUDA(cudaGetLastError());
+    std::vector<int32_t> ptr_h(G + 1);
+    MF_CUDA(cudaMemcpyAsync(ptr_h.data(), A->plan_tr, (G + 1) * sizeof(int32_t), cudaMemcpyDeviceToHost, s));
+    MF_CUDA(cudaEventRecord(e1, s));
+    MF_CUDA(cudaStreamSynchronize(s));
+    A->plan_rows_host = new int64_t[G + 1];
+    for (int g = 0; g <= G; ++g) A->plan_rows_host[g] = std::min<int64_t>((int64_t)ptr_h[g] * TS, n_rows);
+    float ms = 0;
+    MF_CUDA(cudaEventElapsedTime(&ms, e0, e1));
+    A->convert_ms = ms;
+    cudaEventDestroy(e0);
+    cudaEventDestroy(e1);
+    dev_free(cost, s); dev_free(cnt, s); dev_free(off, s); dev_free(tmp, s); dev_free(d_err, s);
+
+    // kernels launched: validate, COUNT, 12 scans x 3, FILL, cost, plan, deps
+    A->convert_launches = (n_rows > 0 ? 1 : 0) + (ntr > 0 ? 2 + 1 : 0) + 12 * (ntr > 0 ? 3 : 0) + 2;
+    A->canonical_bytes = nt * (4 + 4 + 1 + 1 + 8 + 8 + 8) + 16 + (ntr + 1) * 8 + A->rownum * 2 + nnz +
+                         A->nval[0] * 8 + A->nval[1] * 4 + A->nval[2] * 2 + A->nval[3];
+    A->kernel_bytes = nslot * 2 + (A->plane64 ? nslot * 8 : 0) + (A->plane32 ? nslot * 4 : 0) +
+                      (A->plane16 ? nslot * 2 : 0) + (A->plane8 ? nslot : 0) + nt * 4 + (ntr + 1) * 8;
+    return MF_OK;
+}
+
+}  // namespace mf

@@ -1,0 +1,142 @@
+// mf_internal.cuh -- internal declarations of libmf (B200 / sm_100a).
+// Nothing here is shared with oracle/; the two sides are independent implementations.
+#pragma once
+
+#include <cuda_runtime.h>
+#include <cuda_fp16.h>
+#include <cuda_fp8.h>
+#include <stdint.h>
+
+#include <string>
+
+#include "mf.h"
+
+namespace mf {
+
+// ------------------------------------------------------------------ errors
+void set_error(const std::string& msg);
+mf_status fail(mf_status s, const std::string& msg);
+
+#define MF_CUDA(call)                                                                   \
+    do {                                                                                \
+        cudaError_t e_ = (call);                                                        \
+        if (e_ != cudaSuccess)                                                          \
+            return ::mf::fail(MF_ERR_CUDA, std::string(#call) + ": " + cudaGetErrorString(e_)); \
+    } while (0)
+
+#define MF_TRY(call)                                                                    \
+    do {                                                                                \
+        mf_status s_ = (call);                                                          \
+        if (s_ != MF_OK) return s_;                                                     \
+    } while (0)
+
+// ------------------------------------------------------------------ memory
+void* dev_alloc(size_t bytes, cudaStream_t s);
+void dev_free(void* p, cudaStream_t s);
+
+template <class T>
+mf_status alloc(T** p, size_t count, cudaStream_t s) {
+    *p = nullptr;
+    if (count == 0) return MF_OK;
+    *p = static_cast<T*>(dev_alloc(count * sizeof(T), s));
+    if (!*p) return fail(MF_ERR_OOM, "device allocation of " + std::to_string(count * sizeof(T)) + " bytes failed");
+    return MF_OK;
+}
+
+mf_status check_device(int* sm_count);
+
+// ------------------------------------------------------------------ the tile matrix handle
+constexpr int TS = 16;               // tile size
+constexpr int MAX_TILES_PER_TR = 4096;   // 12-bit tile index in the kernel-layout slot word
+constexpr uint16_t SLOT_PAD = 0xFFFF;
+
+struct TileMatrix {
+    int64_t n_rows = 0, n_cols = 0, nnz = 0;
+    int64_t tilenum = 0, rownum = 0, ntr = 0;
+    int64_t nval[4] = {0, 0, 0, 0};
+    int64_t tiles_per_prec[4] = {0, 0, 0, 0};
+    int64_t slots = 0;               // slice columns (each 16 slots wide)
+    int64_t max_nt = 0;              // max tiles in one tile row
+    double convert_ms = 0;
+    int64_t convert_launches = 0;
+    // canonical arrays (device)
+    int32_t *TileRowidx = nullptr, *TileColidx = nullptr;
+    uint8_t *TilePrec = nullptr, *Floor = nullptr;
+    int64_t *TileNnz = nullptr, *Nonrow = nullptr, *ValOff = nullptr, *TileRowPtr = nullptr;
+    uint8_t *RowIndex = nullptr, *CsrRowptr = nullptr, *CsrColidx = nullptr;
+    double* Val64 = nullptr;
+    float* Val32 = nullptr;
+    uint16_t* Val16 = nullptr;
+    uint8_t* Val8 = nullptr;
+    // kernel layout (device): SELL-16 slices, one per tile row, columns in ascending global
+    // column per row; slot word = (tile index in tile row << 4) | local column.
+    int64_t* tr_slot = nullptr;      // [ntr+1] first slice column of each tile row
+    uint32_t* tile_info = nullptr;   // [tilenum] (TileColidx << 4) | (Floor << 2) | TilePrec
+    uint16_t* sidx = nullptr;        // [16*slots]
+    double* plane64 = nullptr;       // [16*slots] value at FP64 (tiles with TilePrec == FP64)
+    float* plane32 = nullptr;        // value rounded to FP32 (tiles with TilePrec <= FP32)
+    __half* plane16 = nullptr;       // ... FP16
+    uint8_t* plane8 = nullptr;       // ... E4M3
+    // launch plan: G CTAs x B threads, CTA g owns tile rows [plan_tr[g], plan_tr[g+1])
+    int32_t G = 0, B = 0;
+    int32_t* plan_tr = nullptr;      // device [G+1]
+    int32_t* dep_lo = nullptr;       // device [G] first CTA whose rows this CTA's tiles gather
+    int32_t* dep_hi = nullptr;       // device [G]
+    int64_t* plan_rows_host = nullptr;  // host [G+1]
+    // distributed (row block of a larger matrix); row_begin == 0 and halo empty on 1 GPU
+    mf_comm* comm = nullptr;
+    int64_t row_begin = 0, n_global = 0;
+    // byte bookkeeping
+    int64_t canonical_bytes = 0, kernel_bytes = 0;
+    cudaStream_t owner_stream = nullptr;
+};
+
+mf_status convert_csr(int64_t n_rows, int64_t n_cols, int64_t nnz, const int64_t* rowptr, const int32_t* colidx,
+                      const double* vals, const mf_convert_opts& o, cudaStream_t s, TileMatrix* A);
+void destroy_tiles(TileMatrix* A);
+
+mf_status run_spmv(const TileMatrix& A, const double* x, double* y, const uint8_t* level, int range_guard,
+                   int64_t* counts_host, cudaStream_t s);
+mf_status run_levels(const double* v, int64_t n, const double* th, uint8_t* level, cudaStream_t s);
+mf_status run_dot(const TileMatrix& A, const double* u, const double* v, double* out_host, cudaStream_t s);
+mf_status run_solve(const TileMatrix& A, bool bicg, const double* b, double* x, const mf_solve_opts& o,
+                    mf_solve_info* info, cudaStream_t s);
+
+}  // namespace mf
+
+struct mf_tile_matrix {
+    mf::TileMatrix m;
+};
+
+// ------------------------------------------------------------------ device helpers
+namespace mfk {
+
+// binary64 -> binary32 with round-to-odd: RZ, then OR the sticky bit into the last place.
+// Rounding this to a format with at least 2 fewer significand bits (FP16, E4M3) with RNE
+// equals a single RNE from the binary64 value.
+__device__ __forceinline__ float d2f_rto(double v) {
+    float f = __double2float_rz(v);
+    if ((double)f != v) f = __int_as_float(__float_as_int(f) | 1);
+    return f;
+}
+__device__ __forceinline__ float to_f32(double v) { return __double2float_rn(v); }
+__device__ __forceinline__ __half to_f16(double v) { return __float2half_rn(d2f_rto(v)); }
+__device__ __forceinline__ uint8_t to_e4m3(double v) {
+    return (uint8_t)__nv_cvt_float_to_fp8(d2f_rto(v), __NV_SATFINITE, __NV_E4M3);
+}
+__device__ __forceinline__ double f16_to_d(__half h) { return (double)__half2float(h); }
+__device__ __forceinline__ double e4m3_to_d(uint8_t b) {
+    __half_raw hr = __nv_cvt_fp8_to_halfraw((__nv_fp8_storage_t)b, __NV_E4M3);
+    return (double)__half2float(__half(hr));
+}
+// value rounded to precision q (0..3) as binary64
+__device__ __forceinline__ double round_to(double v, int q) {
+    switch (q) {
+    case 0: return v;
+    case 1: return (double)to_f32(v);
+    case 2: return f16_to_d(to_f16(v));
+    default: return e4m3_to_d(to_e4m3(v));
+    }
+}
+
+}  // namespace mfk

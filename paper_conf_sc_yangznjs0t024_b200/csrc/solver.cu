@@ -1,0 +1,740 @@
+// solver.cu -- the single-kernel CG and BiCGSTAB of Mille-feuille on sm_100a
+// (Section III-C, Alg. 3; mixed precision Section III-D).
+//
+// One cooperative persistent launch runs the whole solve.  CTA g owns the contiguous tile
+// rows [plan_tr[g], plan_tr[g+1]) (the task distribution of P:130-132, balanced on nnz and
+// tiles) and does every vector operation for its rows.  The paper's dependency
+// counters d_s / d_d / d_a become:
+//   * a monotone-epoch grid barrier (one atomic per CTA, acquire-spin) at each dot product,
+//     carrying the per-CTA partial sums in fixed slots -> deterministic reductions;
+//   * per-CTA "p ready" epoch flags: before an SpMV a CTA waits only for the CTAs owning the
+//     column segments it gathers (the generalisation of d_s), not for the whole grid.
+// The SpMV output mu (and theta) stays in shared memory of the owner CTA across the barrier
+// (spilled to HBM only for rows beyond the smem capacity).  The convergent-element retrieval
+// (Alg. 4) is fused into whoever writes the SpMV input: the level of a 16-element segment is
+// the min over the half-warp that produced it.
+#include <cooperative_groups.h>
+#include <cuda_runtime.h>
+
+#include <algorithm>
+#include <cmath>
+#include <vector>
+
+#include "kernels.cuh"
+#include "mf_internal.cuh"
+
+namespace mf {
+namespace {
+
+using mfk::Counts;
+using mfk::Mat;
+using mfk::Thresh;
+
+constexpr int NSLOT = 4;    // doubles reduced per barrier (max)
+
+struct SolveArgs {
+    Mat A;
+    int32_t G;
+    const int32_t* __restrict__ plan_tr;
+    const int32_t* __restrict__ dep_lo;
+    const int32_t* __restrict__ dep_hi;
+    int64_t n;
+    const double* __restrict__ b;
+    double* x;
+    double* r;
+    double* p;
+    double* mu_g;      // spill of mu beyond mu_cap rows per CTA [n]
+    uint8_t* lev_p;
+    double* rh;        // BiCGSTAB r0*
+    double* s;
+    double* th_g;      // spill of theta
+    uint8_t* lev_s;
+    double* slots;     // [2][NSLOT][G]
+    unsigned* bar;     // grid barrier counter
+    unsigned* flags;   // [G] ready epochs
+    int* abort_flag;
+    unsigned long long* bar_ns;   // [G] time spent spinning
+    double* hist;
+    int64_t hist_cap;
+    unsigned long long* lcounts;  // [lc_cap][10]: tiles[5], nnz[5] per SpMV
+    int64_t lc_cap;
+    double* out;       // [8]: iterations, converged, relres, status
+    double tol, switch_eps;
+    int switch_abs, range_guard;
+    int64_t max_iter;
+    int mu_cap;
+    unsigned long long timeout_ns;
+};
+
+__device__ __forceinline__ unsigned ld_acquire(const unsigned* p) {
+    unsigned v;
+    asm volatile("ld.acquire.gpu.global.u32 %0, [%1];" : "=r"(v) : "l"(p) : "memory");
+    return v;
+}
+__device__ __forceinline__ void st_release(unsigned* p, unsigned v) {
+    asm volatile("st.release.gpu.global.u32 [%0], %1;" ::"l"(p), "r"(v) : "memory");
+}
+__device__ __forceinline__ unsigned long long gtimer() {
+    unsigned long long t;
+    asm volatile("mov.u64 %0, %globaltimer;" : "=l"(t));
+    return t;
+}
+
+struct Ctx {
+    unsigned bar_target = 0;
+    int parity = 0;
+    int spmv = 0;
+};
+
+// ---- synchronisation
+__device__ bool grid_barrier(const SolveArgs& a, Ctx& c) {
+    __shared__ int s_abort;
+    c.bar_target += (unsigned)a.G;
+    __syncthreads();
+    if (threadIdx.x == 0) {
+        const unsigned long long t0 = gtimer();
+        __threadfence();
+        atomicAdd(a.bar, 1u);
+        int ab = 0;
+        while (ld_acquire(a.bar) < c.bar_target) {
+            if (*(volatile int*)a.abort_flag) { ab = 1; break; }
+            if (gtimer() - t0 > a.timeout_ns) { atomicExch(a.abort_flag, 1); ab = 1; break; }
+        }
+        __threadfence();
+        a.bar_ns[blockIdx.x] += gtimer() - t0;
+        s_abort = ab;
+    }
+    __syncthreads();
+    return s_abort == 0;
+}
+
+__device__ void publish(const SolveArgs& a, unsigned epoch) {
+    __syncthreads();
+    if (threadIdx.x == 0) {
+        __threadfence();
+        st_release(&a.flags[blockIdx.x], epoch);
+    }
+}
+
+__device__ bool wait_deps(const SolveArgs& a, unsigned epoch) {
+    __shared__ int s_abort;
+    const int lo = a.dep_lo[blockIdx.x], hi = a.dep_hi[blockIdx.x];
+    if (threadIdx.x == 0) s_abort = 0;
+    __syncthreads();
+    const unsigned long long t0 = gtimer();
+    for (int h = lo + (int)threadIdx.x; h <= hi; h += blockDim.x) {
+        while (ld_acquire(&a.flags[h]) < epoch) {
+            if (*(volatile int*)a.abort_flag) { s_abort = 1; break; }
+            if (gtimer() - t0 > a.timeout_ns) { atomicExch(a.abort_flag, 1); s_abort = 1; break; }
+        }
+    }
+    __threadfence();
+    __syncthreads();
+    if (threadIdx.x == 0) a.bar_ns[blockIdx.x] += gtimer() - t0;
+    return s_abort == 0;
+}
+
+// K doubles: thread fma chains -> warp butterfly -> tree32 over warps -> slot -> barrier ->
+// tree32 over CTAs.  Every thread returns the grid totals.
+template <int K>
+__device__ bool grid_reduce(double (&v)[K], const SolveArgs& a, Ctx& c, double* red) {
+    const int w = threadIdx.x >> 5, l = threadIdx.x & 31, W = blockDim.x >> 5;
+#pragma unroll
+    for (int k = 0; k < K; ++k) {
+        const double wt = mfk::butterfly32(v[k]);
+        if (l == 0) red[k * 32 + w] = wt;
+    }
+    __syncthreads();
+    if (w == 0) {
+#pragma unroll
+        for (int k = 0; k < K; ++k) {
+            const double ct = mfk::tree32(red + k * 32, W);
+            if (l == 0) a.slots[((size_t)c.parity * NSLOT + k) * a.G + blockIdx.x] = ct;
+        }
+    }
+    const bool ok = grid_barrier(a, c);
+    if (w == 0) {
+#pragma unroll
+        for (int k = 0; k < K; ++k) {
+            const double gt = mfk::tree32(a.slots + ((size_t)c.parity * NSLOT + k) * a.G, a.G);
+            if (l == 0) red[128 + k] = gt;
+        }
+    }
+    __syncthreads();
+#pragma unroll
+    for (int k = 0; k < K; ++k) v[k] = red[128 + k];
+    __syncthreads();
+    c.parity ^= 1;
+    return ok;
+}
+
+template <bool COUNT>
+__device__ void flush_counts(const SolveArgs& a, Ctx& c, Counts& cnt, int* ired) {
+    if (!COUNT) return;
+    if (threadIdx.x < 10) ired[threadIdx.x] = 0;
+    __syncthreads();
+#pragma unroll
+    for (int q = 0; q < 5; ++q) {
+        int tv = cnt.tiles(q), nv = cnt.nnz(q);
+        for (int o = 16; o >= 1; o >>= 1) { tv += __shfl_xor_sync(0xffffffffu, tv, o); nv += __shfl_xor_sync(0xffffffffu, nv, o); }
+        if ((threadIdx.x & 31) == 0) { atomicAdd(&ired[q], tv); atomicAdd(&ired[5 + q], nv); }
+    }
+    __syncthreads();
+    if (threadIdx.x < 10 && c.spmv < a.lc_cap && ired[threadIdx.x])
+        atomicAdd(&a.lcounts[(size_t)c.spmv * 10 + threadIdx.x], (unsigned long long)ired[threadIdx.x]);
+    cnt.zero();
+    c.spmv++;
+}
+
+__device__ __forceinline__ Thresh make_thresh(const SolveArgs& a, double v0norm) {
+    const double tau = a.switch_abs ? a.switch_eps : __ddiv_rn(__dmul_rn(a.switch_eps, v0norm), sqrt((double)a.n));
+    return Thresh{__dmul_rn(tau, 1e-3), __dmul_rn(tau, 1e-2), __dmul_rn(tau, 1e-1), tau};
+}
+
+struct Smem {
+    double* mu;      // [mu_cap]
+    double* th;      // [mu_cap] (BiCGSTAB)
+    double* red;     // [4*32 + 8]
+    uint32_t* stage; // [H][STAGE]
+    int* ired;       // [16]
+};
+
+__device__ Smem carve(const SolveArgs& a, int nvec) {
+    extern __shared__ __align__(16) unsigned char smem_raw[];
+    Smem s;
+    double* d = reinterpret_cast<double*>(smem_raw);
+    s.mu = d;
+    s.th = d + a.mu_cap;
+    s.red = d + (size_t)nvec * a.mu_cap;
+    s.ired = reinterpret_cast<int*>(s.red + 4 * 32 + 8);
+    s.stage = reinterpret_cast<uint32_t*>(s.ired + 16);
+    return s;
+}
+
+// -------------------------------------------------------------------------- CG (Alg. 1 / Alg. 3)
+template <bool DYN, bool COUNT>
+__global__ void __launch_bounds__(1024, 1) cg_persistent(SolveArgs a) {
+    Smem sm = carve(a, 1);
+    Ctx c;
+    Counts cnt;
+    cnt.zero();
+    const int t = threadIdx.x, B = blockDim.x, H = B >> 4, h = t >> 4, lane = t & 15;
+    const unsigned m = mfk::hw_mask();
+    uint32_t* stage = sm.stage + h * mfk::STAGE;
+    const int64_t tr0 = a.plan_tr[blockIdx.x], tr1 = a.plan_tr[blockIdx.x + 1];
+    const int64_t R0 = tr0 * 16, Rend = min(tr1 * 16, a.n);
+    const int64_t n = a.n;
+    auto mu_at = [&](int64_t li) -> double& { return li < a.mu_cap ? sm.mu[li] : a.mu_g[R0 + li]; };
+
+    // init: r = b - A~ x0 at TilePrec; p = r; partial (b,b), (r,r)
+    double v2[2] = {0.0, 0.0};
+    for (int64_t TR = tr0 + h; TR < tr1; TR += H) {
+        const double ax = mfk::spmv_tile_row<false, false>(a.A, TR, lane, a.x, nullptr, 0, stage, m, nullptr);
+        const int64_t i = TR * 16 + lane;
+        if (i < n) {
+            const double bi = a.b[i], ri = __dsub_rn(bi, ax);
+            a.r[i] = ri;
+            a.p[i] = ri;
+            v2[0] = __fma_rn(bi, bi, v2[0]);
+            v2[1] = __fma_rn(ri, ri, v2[1]);
+        }
+    }
+    bool ok = grid_reduce<2>(v2, a, c, sm.red);
+    const double nb = sqrt(v2[0]);
+    double rho = v2[1];
+    int64_t j = 0;
+    int converged = 0, status = ok ? MF_OK : MF_ERR_DEADLOCK;
+    if (ok && nb == 0.0) {
+        for (int64_t i = R0 + t; i < Rend; i += B) a.x[i] = 0.0;
+        converged = 1;
+        if (blockIdx.x == 0 && t == 0 && a.hist_cap > 0) a.hist[0] = 0.0;
+    } else if (ok) {
+        const Thresh th = make_thresh(a, sqrt(rho));
+        if (DYN) {
+            for (int64_t TR = tr0 + h; TR < tr1; TR += H) {
+                const int64_t i = TR * 16 + lane;
+                const int lv = mfk::hw_min_i(i < n ? mfk::level_of(a.p[i], th) : 4, m);
+                if (lane == 0) a.lev_p[TR] = (uint8_t)lv;
+            }
+        }
+        publish(a, 1);
+        for (;; ++j) {
+            const double relres = __ddiv_rn(sqrt(rho), nb);
+            if (blockIdx.x == 0 && t == 0) { if (j < a.hist_cap) a.hist[j] = relres; a.out[2] = relres; }
+            if (relres < a.tol) { converged = 1; break; }
+            if (j == a.max_iter) break;
+            if (!wait_deps(a, (unsigned)(j + 1))) { status = MF_ERR_DEADLOCK; break; }
+            // step A: mu = A~_j p_j (own tile rows) with the fused partial (mu, p)
+            double sg[1] = {0.0};
+            for (int64_t TR = tr0 + h; TR < tr1; TR += H) {
+                const double mv = mfk::spmv_tile_row<DYN, COUNT>(a.A, TR, lane, a.p, a.lev_p, a.range_guard, stage, m, &cnt);
+                const int64_t i = TR * 16 + lane;
+                if (i < n) {
+                    mu_at(i - R0) = mv;
+                    sg[0] = __fma_rn(mv, a.p[i], sg[0]);
+                }
+            }
+            flush_counts<COUNT>(a, c, cnt, sm.ired);
+            // step B: sigma = (mu, p) over the grid -> alpha
+            if (!grid_reduce<1>(sg, a, c, sm.red)) { status = MF_ERR_DEADLOCK; break; }
+            const double sigma = sg[0];
+            if (!(sigma > 0.0) || !isfinite(sigma)) { status = MF_ERR_BREAKDOWN; break; }
+            const double alpha = __ddiv_rn(rho, sigma);
+            // step C: x += alpha p, r -= alpha mu, partial (r, r)
+            double rr[1] = {0.0};
+            for (int64_t li = t; R0 + li < Rend; li += B) {
+                const int64_t i = R0 + li;
+                a.x[i] = __fma_rn(alpha, a.p[i], a.x[i]);
+                const double ri = __fma_rn(-alpha, mu_at(li), a.r[i]);
+                a.r[i] = ri;
+                rr[0] = __fma_rn(ri, ri, rr[0]);
+            }
+            if (!grid_reduce<1>(rr, a, c, sm.red)) { status = MF_ERR_DEADLOCK; break; }
+            const double beta = __ddiv_rn(rr[0], rho);
+            rho = rr[0];
+            // step D: p = r + beta p (own rows) and the levels of its segments (Alg. 4)
+            for (int64_t TR = tr0 + h; TR < tr1; TR += H) {
+                const int64_t i = TR * 16 + lane;
+                double pn = 0.0;
+                if (i < n) { pn = __fma_rn(beta, a.p[i], a.r[i]); a.p[i] = pn; }
+                if (DYN) {
+                    const int lv = mfk::hw_min_i(i < n ? mfk::level_of(pn, th) : 4, m);
+                    if (lane == 0) a.lev_p[TR] = (uint8_t)lv;
+                }
+            }
+            publish(a, (unsigned)(j + 2));
+        }
+    }
+    if (blockIdx.x == 0 && t == 0) {
+        a.out[0] = (double)j;
+        a.out[1] = converged;
+        a.out[3] = status;
+    }
+    if (status == MF_ERR_DEADLOCK && t == 0) atomicExch(a.abort_flag, 1);
+}
+
+// -------------------------------------------------------------------------- BiCGSTAB (Alg. 2)
+template <bool DYN, bool COUNT>
+__global__ void __launch_bounds__(1024, 1) bicgstab_persistent(SolveArgs a) {
+    Smem sm = carve(a, 2);
+    Ctx c;
+    Counts cnt;
+    cnt.zero();
+    const int t = threadIdx.x, B = blockDim.x, H = B >> 4, h = t >> 4, lane = t & 15;
+    const unsigned m = mfk::hw_mask();
+    uint32_t* stage = sm.stage + h * mfk::STAGE;
+    const int64_t tr0 = a.plan_tr[blockIdx.x], tr1 = a.plan_tr[blockIdx.x + 1];
+    const int64_t R0 = tr0 * 16, Rend = min(tr1 * 16, a.n);
+    const int64_t n = a.n;
+    auto mu_at = [&](int64_t li) -> double& { return li < a.mu_cap ? sm.mu[li] : a.mu_g[R0 + li]; };
+    auto th_at = [&](int64_t li) -> double& { return li < a.mu_cap ? sm.th[li] : a.th_g[R0 + li]; };
+
+    // init: r = b - A~ x0; r0* = r; p = r; partial (b,b), (r,r), (r,r0*)
+    double v3[3] = {0.0, 0.0, 0.0};
+    for (int64_t TR = tr0 + h; TR < tr1; TR += H) {
+        const double ax = mfk::spmv_tile_row<false, false>(a.A, TR, lane, a.x, nullptr, 0, stage, m, nullptr);
+        const int64_t i = TR * 16 + lane;
+        if (i < n) {
+            const double bi = a.b[i], ri = __dsub_rn(bi, ax);
+            a.r[i] = ri; a.rh[i] = ri; a.p[i] = ri;
+            v3[0] = __fma_rn(bi, bi, v3[0]);
+            v3[1] = __fma_rn(ri, ri, v3[1]);
+            v3[2] = __fma_rn(ri, ri, v3[2]);
+        }
+    }
+    bool ok = grid_reduce<3>(v3, a, c, sm.red);
+    const double nb = sqrt(v3[0]);
+    double rr = v3[1], rho = v3[2];
+    int64_t j = 0;
+    int converged = 0, status = ok ? MF_OK : MF_ERR_DEADLOCK;
+    unsigned epoch = 0;
+    if (ok && nb == 0.0) {
+        for (int64_t i = R0 + t; i < Rend; i += B) a.x[i] = 0.0;
+        converged = 1;
+        if (blockIdx.x == 0 && t == 0 && a.hist_cap > 0) a.hist[0] = 0.0;
+    } else if (ok) {
+        const Thresh th = make_thresh(a, sqrt(rr));
+        if (DYN) {
+            for (int64_t TR = tr0 + h; TR < tr1; TR += H) {
+                const int64_t i = TR * 16 + lane;
+                const int lv = mfk::hw_min_i(i < n ? mfk::level_of(a.p[i], th) : 4, m);
+                if (lane == 0) a.lev_p[TR] = (uint8_t)lv;
+            }
+        }
+        publish(a, ++epoch);
+        for (;; ++j) {
+            const double relres = __ddiv_rn(sqrt(rr), nb);
+            if (blockIdx.x == 0 && t == 0) { if (j < a.hist_cap) a.hist[j] = relres; a.out[2] = relres; }
+            if (relres < a.tol) { converged = 1; break; }
+            if (j == a.max_iter) break;
+            if (!wait_deps(a, epoch)) { status = MF_ERR_DEADLOCK; break; }
+            // mu = A~ p ; partial (mu, r0*)
+            double eta[1] = {0.0};
+            for (int64_t TR = tr0 + h; TR < tr1; TR += H) {
+                const double mv = mfk::spmv_tile_row<DYN, COUNT>(a.A, TR, lane, a.p, a.lev_p, a.range_guard, stage, m, &cnt);
+                const int64_t i = TR * 16 + lane;
+                if (i < n) { mu_at(i - R0) = mv; eta[0] = __fma_rn(mv, a.rh[i], eta[0]); }
+            }
+            flush_counts<COUNT>(a, c, cnt, sm.ired);
+            if (!grid_reduce<1>(eta, a, c, sm.red)) { status = MF_ERR_DEADLOCK; break; }
+            if (eta[0] == 0.0 || !isfinite(eta[0])) { status = MF_ERR_BREAKDOWN; break; }
+            const double alpha = __ddiv_rn(rho, eta[0]);
+            // s = r - alpha mu (own rows) + levels of s
+            for (int64_t TR = tr0 + h; TR < tr1; TR += H) {
+                const int64_t i = TR * 16 + lane;
+                double si = 0.0;
+                if (i < n) { si = __fma_rn(-alpha, mu_at(i - R0), a.r[i]); a.s[i] = si; }
+                if (DYN) {
+                    const int lv = mfk::hw_min_i(i < n ? mfk::level_of(si, th) : 4, m);
+                    if (lane == 0) a.lev_s[TR] = (uint8_t)lv;
+                }
+            }
+            publish(a, ++epoch);
+            if (!wait_deps(a, epoch)) { status = MF_ERR_DEADLOCK; break; }
+            // theta = A~ s ; partial (theta, theta), (theta, s)
+            double tt[2] = {0.0, 0.0};
+            for (int64_t TR = tr0 + h; TR < tr1; TR += H) {
+                const double tv = mfk::spmv_tile_row<DYN, COUNT>(a.A, TR, lane, a.s, a.lev_s, a.range_guard, stage, m, &cnt);
+                const int64_t i = TR * 16 + lane;
+                if (i < n) {
+                    th_at(i - R0) = tv;
+                    tt[0] = __fma_rn(tv, tv, tt[0]);
+                    tt[1] = __fma_rn(tv, a.s[i], tt[1]);
+                }
+            }
+            flush_counts<COUNT>(a, c, cnt, sm.ired);
+            if (!grid_reduce<2>(tt, a, c, sm.red)) { status = MF_ERR_DEADLOCK; break; }
+            if (tt[0] == 0.0) {
+                // theta == 0: take the half step x += alpha p, r = s, and stop (reading R14)
+                double r2[1] = {0.0};
+                for (int64_t li = t; R0 + li < Rend; li += B) {
+                    const int64_t i = R0 + li;
+                    a.x[i] = __fma_rn(alpha, a.p[i], a.x[i]);
+                    const double si = a.s[i];
+                    a.r[i] = si;
+                    r2[0] = __fma_rn(si, si, r2[0]);
+                }
+                if (!grid_reduce<1>(r2, a, c, sm.red)) { status = MF_ERR_DEADLOCK; break; }
+                ++j;
+                const double rl = __ddiv_rn(sqrt(r2[0]), nb);
+                if (blockIdx.x == 0 && t == 0) { if (j < a.hist_cap) a.hist[j] = rl; a.out[2] = rl; }
+                if (rl < a.tol) converged = 1; else status = MF_ERR_BREAKDOWN;
+                break;
+            }
+            const double omega = __ddiv_rn(tt[1], tt[0]);
+            if (omega == 0.0 || !isfinite(omega)) { status = MF_ERR_BREAKDOWN; break; }
+            // x += alpha p + omega s ; r = s - omega theta ; partial (r, r0*), (r, r)
+            double rv[2] = {0.0, 0.0};
+            for (int64_t li = t; R0 + li < Rend; li += B) {
+                const int64_t i = R0 + li;
+                const double si = a.s[i];
+                a.x[i] = __fma_rn(omega, si, __fma_rn(alpha, a.p[i], a.x[i]));
+                const double ri = __fma_rn(-omega, th_at(li), si);
+                a.r[i] = ri;
+                rv[0] = __fma_rn(ri, a.rh[i], rv[0]);
+                rv[1] = __fma_rn(ri, ri, rv[1]);
+            }
+            if (!grid_reduce<2>(rv, a, c, sm.red)) { status = MF_ERR_DEADLOCK; break; }
+            rr = rv[1];
+            if (rv[0] == 0.0 || !isfinite(rv[0])) {
+                ++j;
+                const double rl = __ddiv_rn(sqrt(rr), nb);
+                if (blockIdx.x == 0 && t == 0) { if (j < a.hist_cap) a.hist[j] = rl; a.out[2] = rl; }
+                if (rl < a.tol) converged = 1; else status = MF_ERR_BREAKDOWN;
+                break;
+            }
+            const double beta = __dmul_rn(__ddiv_rn(rv[0], rho), __ddiv_rn(alpha, omega));
+            rho = rv[0];
+            // p = r + beta (p - omega mu) (own rows) + levels of p
+            for (int64_t TR = tr0 + h; TR < tr1; TR += H) {
+                const int64_t i = TR * 16 + lane;
+                double pn = 0.0;
+                if (i < n) { pn = __fma_rn(beta, __fma_rn(-omega, mu_at(i - R0), a.p[i]), a.r[i]); a.p[i] = pn; }
+                if (DYN) {
+                    const int lv = mfk::hw_min_i(i < n ? mfk::level_of(pn, th) : 4, m);
+                    if (lane == 0) a.lev_p[TR] = (uint8_t)lv;
+                }
+            }
+            publish(a, ++epoch);
+        }
+    }
+    if (blockIdx.x == 0 && t == 0) {
+        a.out[0] = (double)j;
+        a.out[1] = converged;
+        a.out[3] = status;
+    }
+    if (status == MF_ERR_DEADLOCK && t == 0) atomicExch(a.abort_flag, 1);
+}
+
+// -------------------------------------------------------------------------- standalone kernels
+template <bool DYN, bool COUNT>
+__global__ void __launch_bounds__(256) spmv_kernel(Mat A, const double* __restrict__ x, double* __restrict__ y,
+                                                   const uint8_t* __restrict__ level, int range_guard,
+                                                   unsigned long long* counts) {
+    __shared__ uint32_t stage_all[256 / 16 * mfk::STAGE];
+    __shared__ int ired[10];
+    const int h = threadIdx.x >> 4, lane = threadIdx.x & 15;
+    const unsigned m = mfk::hw_mask();
+    Counts cnt;
+    cnt.zero();
+    if (COUNT && threadIdx.x < 10) ired[threadIdx.x] = 0;
+    const int64_t H = (int64_t)gridDim.x * (blockDim.x >> 4);
+    for (int64_t TR = (int64_t)blockIdx.x * (blockDim.x >> 4) + h; TR < A.ntr; TR += H) {
+        const double v = mfk::spmv_tile_row<DYN, COUNT>(A, TR, lane, x, level, range_guard,
+                                                        stage_all + h * mfk::STAGE, m, &cnt);
+        const int64_t i = TR * 16 + lane;
+        if (i < A.n_rows) y[i] = v;
+    }
+    if (COUNT) {
+        __syncthreads();
+#pragma unroll
+        for (int q = 0; q < 5; ++q) {
+            if (cnt.tiles(q)) atomicAdd(&ired[q], cnt.tiles(q));
+            if (cnt.nnz(q)) atomicAdd(&ired[5 + q], cnt.nnz(q));
+        }
+        __syncthreads();
+        if (threadIdx.x < 10 && ired[threadIdx.x]) atomicAdd(&counts[threadIdx.x], (unsigned long long)ired[threadIdx.x]);
+    }
+}
+
+__global__ void levels_kernel(const double* __restrict__ v, int64_t n, Thresh th, uint8_t* level) {
+    const unsigned m = mfk::hw_mask();
+    const int lane = threadIdx.x & 15;
+    const int64_t nseg = (n + 15) / 16;
+    const int64_t H = (int64_t)gridDim.x * (blockDim.x >> 4);
+    for (int64_t J = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 4; J < nseg; J += H) {
+        const int64_t i = J * 16 + lane;
+        const int lv = mfk::hw_min_i(i < n ? mfk::level_of(v[i], th) : 4, m);
+        if (lane == 0) level[J] = (uint8_t)lv;
+    }
+}
+
+// dot with the plan's tree: block g = CTA g of the plan, B threads
+__global__ void dot_partial_kernel(const int32_t* __restrict__ plan_tr, int64_t n, const double* __restrict__ u,
+                                   const double* __restrict__ v, double* slots) {
+    __shared__ double red[32];
+    const int64_t R0 = (int64_t)plan_tr[blockIdx.x] * 16, Rend = min((int64_t)plan_tr[blockIdx.x + 1] * 16, n);
+    double acc = 0.0;
+    for (int64_t i = R0 + threadIdx.x; i < Rend; i += blockDim.x) acc = __fma_rn(u[i], v[i], acc);
+    const double wt = mfk::butterfly32(acc);
+    if ((threadIdx.x & 31) == 0) red[threadIdx.x >> 5] = wt;
+    __syncthreads();
+    if (threadIdx.x < 32) {
+        const double ct = mfk::tree32(red, blockDim.x >> 5);
+        if (threadIdx.x == 0) slots[blockIdx.x] = ct;
+    }
+}
+__global__ void dot_final_kernel(const double* __restrict__ slots, int G, double* out) {
+    const double gt = mfk::tree32(slots, G);
+    if (threadIdx.x == 0) *out = gt;
+}
+
+Mat mat_view(const TileMatrix& A) {
+    return Mat{A.n_rows, A.n_cols, A.ntr, A.tr_slot, A.TileRowPtr, A.tile_info, A.sidx,
+               A.plane64, A.plane32, A.plane16, A.plane8};
+}
+
+}  // namespace
+
+// ------------------------------------------------------------------------------- host side
+mf_status run_spmv(const TileMatrix& A, const double* x, double* y, const uint8_t* level, int range_guard,
+                   int64_t* counts_host, cudaStream_t s) {
+    if (A.ntr == 0) return MF_OK;
+    Mat M = mat_view(A);
+    int blocks = (int)std::min<int64_t>((A.ntr + 15) / 16, 148 * 16);
+    unsigned long long* dcnt = nullptr;
+    if (counts_host) {
+        MF_TRY(alloc(&dcnt, 10, s));
+        MF_CUDA(cudaMemsetAsync(dcnt, 0, 10 * sizeof(unsigned long long), s));
+    }
+    if (level) {
+        if (counts_host) spmv_kernel<true, true><<<blocks, 256, 0, s>>>(M, x, y, level, range_guard, dcnt);
+        else spmv_kernel<true, false><<<blocks, 256, 0, s>>>(M, x, y, level, range_guard, dcnt);
+    } else {
+        if (counts_host) spmv_kernel<false, true><<<blocks, 256, 0, s>>>(M, x, y, level, range_guard, dcnt);
+        else spmv_kernel<false, false><<<blocks, 256, 0, s>>>(M, x, y, level, range_guard, dcnt);
+    }
+    MF_CUDA(cudaGetLastError());
+    if (counts_host) {
+        unsigned long long h[10];
+        MF_CUDA(cudaMemcpyAsync(h, dcnt, sizeof(h), cudaMemcpyDeviceToHost, s));
+        MF_CUDA(cudaStreamSynchronize(s));
+        for (int q = 0; q < 5; ++q) counts_host[q] = (int64_t)h[q];
+        dev_free(dcnt, s);
+    }
+    return MF_OK;
+}
+
+mf_status run_levels(const double* v, int64_t n, const double* th, uint8_t* level, cudaStream_t s) {
+    if (n == 0) return MF_OK;
+    Thresh t{th[0], th[1], th[2], th[3]};
+    int64_t nseg = (n + 15) / 16;
+    int blocks = (int)std::min<int64_t>((nseg + 15) / 16, 148 * 16);
+    levels_kernel<<<blocks, 256, 0, s>>>(v, n, t, level);
+    MF_CUDA(cudaGetLastError());
+    return MF_OK;
+}
+
+mf_status run_dot(const TileMatrix& A, const double* u, const double* v, double* out_host, cudaStream_t s) {
+    double* slots = nullptr;
+    MF_TRY(alloc(&slots, A.G + 1, s));
+    dot_partial_kernel<<<A.G, A.B, 0, s>>>(A.plan_tr, A.n_rows, u, v, slots);
+    dot_final_kernel<<<1, 32, 0, s>>>(slots, A.G, slots + A.G);
+    MF_CUDA(cudaGetLastError());
+    MF_CUDA(cudaMemcpyAsync(out_host, slots + A.G, sizeof(double), cudaMemcpyDeviceToHost, s));
+    MF_CUDA(cudaStreamSynchronize(s));
+    dev_free(slots, s);
+    return MF_OK;
+}
+
+// byte model per SpMV: values at e_t + 0.5 B/nnz + 1 B per non-empty
+// tile row + 8 B per tile, non-bypassed tiles only (index bytes of bypassed tiles excluded)
+static double spmv_model_bytes(const TileMatrix& A, const unsigned long long* c10) {
+    static const double vb[4] = {8, 4, 2, 1};
+    double bytes = 0;
+    double tiles_nb = 0, nnz_nb = 0;
+    for (int q = 0; q < 4; ++q) { bytes += vb[q] * (double)c10[5 + q]; tiles_nb += (double)c10[q]; nnz_nb += (double)c10[5 + q]; }
+    const double tiles_all = tiles_nb + (double)c10[4];
+    const double rows_frac = tiles_all > 0 ? tiles_nb / tiles_all : 0;
+    return bytes + 0.5 * nnz_nb + (double)A.rownum * rows_frac + 8.0 * tiles_nb;
+}
+
+mf_status run_solve(const TileMatrix& A, bool bicg, const double* b, double* x, const mf_solve_opts& o,
+                    mf_solve_info* info, cudaStream_t s) {
+    if (A.n_rows != A.n_cols) return fail(MF_ERR_INVALID_ARG, "solve needs a square matrix");
+    if (o.sticky) return fail(MF_ERR_NOT_IMPLEMENTED, "sticky (in-place) downgrade is not implemented on the GPU path");
+    if (o.M) return fail(MF_ERR_NOT_IMPLEMENTED, "preconditioned solves go through mf_precond (see precond.cu)");
+    int dev = 0, sms = 0, smem_optin = 0;
+    MF_CUDA(cudaGetDevice(&dev));
+    MF_CUDA(cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev));
+    MF_CUDA(cudaDeviceGetAttribute(&smem_optin, cudaDevAttrMaxSharedMemoryPerBlockOptin, dev));
+    const int64_t n = A.n_rows;
+    const int G = A.G, B = A.B, H = B / 16;
+    const bool dyn = o.mode == MF_MODE_DYNAMIC_MIXED;
+    const int nvec = bicg ? 2 : 1;
+    // per-SpMV level statistics (tile_level_counts, exact dynamic byte model) cost ALU in the
+    // SpMV loop: collected only on request
+    const bool count = o.tile_level_counts != nullptr || o.collect_stats;
+    int64_t max_rows = 0;
+    for (int g = 0; g < G; ++g) max_rows = std::max(max_rows, A.plan_rows_host[g + 1] - A.plan_rows_host[g]);
+    const size_t fixed = (4 * 32 + 8) * sizeof(double) + 16 * sizeof(int) + (size_t)H * mfk::STAGE * sizeof(uint32_t);
+    int64_t cap = ((int64_t)smem_optin - (int64_t)fixed - 64) / (8 * nvec);
+    cap = std::max<int64_t>(0, std::min(cap, max_rows));
+    const size_t smem = fixed + (size_t)cap * 8 * nvec;
+
+    // workspace
+    double *r = nullptr, *p = nullptr, *mu_g = nullptr, *rh = nullptr, *sv = nullptr, *th_g = nullptr;
+    double *slots = nullptr, *hist = nullptr, *out = nullptr;
+    uint8_t *lev_p = nullptr, *lev_s = nullptr;
+    unsigned* sync = nullptr;
+    unsigned long long *lcounts = nullptr, *bar_ns = nullptr;
+    const bool spill = cap < max_rows;
+    const int64_t hist_cap = o.max_iter + 2;
+    const int64_t lc_cap = (bicg ? 2 : 1) * (o.max_iter + 1);
+    MF_TRY(alloc(&r, n, s));
+    MF_TRY(alloc(&p, n, s));
+    if (spill) MF_TRY(alloc(&mu_g, n, s));
+    MF_TRY(alloc(&lev_p, A.ntr + 1, s));
+    if (bicg) {
+        MF_TRY(alloc(&rh, n, s));
+        MF_TRY(alloc(&sv, n, s));
+        MF_TRY(alloc(&lev_s, A.ntr + 1, s));
+        if (spill) MF_TRY(alloc(&th_g, n, s));
+    }
+    MF_TRY(alloc(&slots, (size_t)2 * NSLOT * G, s));
+    MF_TRY(alloc(&hist, hist_cap, s));
+    MF_TRY(alloc(&out, 8, s));
+    MF_TRY(alloc(&sync, (size_t)G + 2, s));
+    MF_TRY(alloc(&bar_ns, G, s));
+    if (count) MF_TRY(alloc(&lcounts, (size_t)lc_cap * 10, s));
+    MF_CUDA(cudaMemsetAsync(sync, 0, (G + 2) * sizeof(unsigned), s));
+    MF_CUDA(cudaMemsetAsync(bar_ns, 0, G * sizeof(unsigned long long), s));
+    MF_CUDA(cudaMemsetAsync(out, 0, 8 * sizeof(double), s));
+    if (count) MF_CUDA(cudaMemsetAsync(lcounts, 0, (size_t)lc_cap * 10 * sizeof(unsigned long long), s));
+
+    SolveArgs a{};
+    a.A = mat_view(A);
+    a.G = G; a.plan_tr = A.plan_tr; a.dep_lo = A.dep_lo; a.dep_hi = A.dep_hi;
+    a.n = n; a.b = b; a.x = x; a.r = r; a.p = p; a.mu_g = mu_g; a.lev_p = lev_p;
+    a.rh = rh; a.s = sv; a.th_g = th_g; a.lev_s = lev_s;
+    a.slots = slots; a.bar = sync; a.abort_flag = reinterpret_cast<int*>(sync + 1); a.flags = sync + 2;
+    a.bar_ns = bar_ns; a.hist = hist; a.hist_cap = hist_cap; a.lcounts = lcounts; a.lc_cap = count ? lc_cap : 0;
+    a.out = out; a.tol = o.tol; a.switch_eps = o.switch_eps < 0 ? o.tol : o.switch_eps;
+    a.switch_abs = o.switch_absolute; a.range_guard = o.range_guard; a.max_iter = o.max_iter;
+    a.mu_cap = (int)cap; a.timeout_ns = 60ull * 1000000000ull;
+
+    void* kfn;
+    if (bicg) kfn = dyn ? (count ? (void*)bicgstab_persistent<true, true> : (void*)bicgstab_persistent<true, false>)
+                        : (count ? (void*)bicgstab_persistent<false, true> : (void*)bicgstab_persistent<false, false>);
+    else kfn = dyn ? (count ? (void*)cg_persistent<true, true> : (void*)cg_persistent<true, false>)
+                   : (count ? (void*)cg_persistent<false, true> : (void*)cg_persistent<false, false>);
+    MF_CUDA(cudaFuncSetAttribute(kfn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
+    int per_sm = 0;
+    MF_CUDA(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, kfn, B, smem));
+    if (per_sm * sms < G) return fail(MF_ERR_INVALID_ARG, "plan G exceeds co-resident CTAs for this launch");
+
+    cudaEvent_t e0, e1;
+    MF_CUDA(cudaEventCreate(&e0));
+    MF_CUDA(cudaEventCreate(&e1));
+    void* args[] = {&a};
+    MF_CUDA(cudaEventRecord(e0, s));
+    MF_CUDA(cudaLaunchCooperativeKernel(kfn, dim3(G), dim3(B), args, smem, s));
+    MF_CUDA(cudaEventRecord(e1, s));
+    double hout[8];
+    MF_CUDA(cudaMemcpyAsync(hout, out, sizeof(hout), cudaMemcpyDeviceToHost, s));
+    MF_CUDA(cudaStreamSynchronize(s));
+    float ms = 0;
+    MF_CUDA(cudaEventElapsedTime(&ms, e0, e1));
+    cudaEventDestroy(e0);
+    cudaEventDestroy(e1);
+    const int64_t iters = (int64_t)hout[0];
+    info->iterations = iters;
+    info->converged = (int)hout[1];
+    info->rel_residual = hout[2];
+    info->status = (mf_status)(int)hout[3];
+    info->kernel_ms = ms;
+    info->launches = 1;
+    const int64_t nspmv = (bicg ? 2 : 1) * iters;
+    info->n_spmv = nspmv;
+    if (o.residual_history && o.history_cap > 0) {
+        const int64_t k = std::min<int64_t>(o.history_cap, std::min<int64_t>(iters + 1, hist_cap));
+        MF_CUDA(cudaMemcpyAsync(o.residual_history, hist, k * sizeof(double), cudaMemcpyDeviceToHost, s));
+    }
+    std::vector<unsigned long long> lc;
+    if (count) {
+        const int64_t k = std::min<int64_t>(lc_cap, nspmv + 2);
+        lc.resize((size_t)k * 10);
+        MF_CUDA(cudaMemcpyAsync(lc.data(), lcounts, lc.size() * sizeof(unsigned long long), cudaMemcpyDeviceToHost, s));
+    }
+    MF_CUDA(cudaStreamSynchronize(s));
+    double model = 0;
+    if (!count) {   // every tile at TilePrec, nothing bypassed (static / FP64 modes)
+        unsigned long long c10[10] = {0, 0, 0, 0, 0, 0, 0, 0, 0, 0};
+        for (int q = 0; q < 4; ++q) { c10[q] = (unsigned long long)A.tiles_per_prec[q]; c10[5 + q] = (unsigned long long)A.nval[q]; }
+        model = dyn ? 0.0 : spmv_model_bytes(A, c10) * (double)nspmv;
+    } else {
+        const int64_t k = (int64_t)lc.size() / 10;
+        for (int64_t q = 0; q < k; ++q) {
+            unsigned long long tot = 0;
+            for (int e = 0; e < 5; ++e) tot += lc[q * 10 + e];
+            if (tot == 0) continue;
+            model += spmv_model_bytes(A, &lc[q * 10]);
+            if (o.tile_level_counts && q < o.level_counts_cap)
+                for (int e = 0; e < 5; ++e) o.tile_level_counts[q * 5 + e] = (int64_t)lc[q * 10 + e];
+        }
+    }
+    // vectors: CG 48n per iteration (read p,x,r; write x,r,p); BiCGSTAB 72n (read p,x,r,r0*,s;
+    // write s,x,r,p); + 16n per SpMV output that cannot stay on chip (capacity rule)
+    const double vec = bicg ? 72.0 : 48.0;
+    const double spill_b = spill ? (bicg ? 32.0 : 16.0) : 0.0;
+    info->model_bytes = model + (vec + spill_b) * (double)n * (double)iters;
+    mf_status st = info->status;
+    dev_free(r, s); dev_free(p, s); dev_free(mu_g, s); dev_free(lev_p, s); dev_free(rh, s); dev_free(sv, s);
+    dev_free(lev_s, s); dev_free(th_g, s); dev_free(slots, s); dev_free(hist, s); dev_free(out, s);
+    dev_free(sync, s); dev_free(bar_ns, s); dev_free(lcounts, s);
+    if (st == MF_ERR_BREAKDOWN) return fail(st, "numerical breakdown");
+    if (st == MF_ERR_DEADLOCK) return fail(st, "grid-barrier watchdog expired");
+    return st;
+}
+
+}  // namespace mf

@@ -1,0 +1,274 @@
+"""GPU parity: libmf (C-ABI, sm_100a kernels) against the oracle, element by element.
+
+Gates (BASELINE.json north_star):
+  * tile conversion and indexing bit-exact           -> every canonical array byte-identical
+  * all-FP64 mode residual histories to 1e-12 rel.    -> asserted bit-identical (kernel-order)
+  * mixed solves: stopping residual, ||x-x_o||/||x_o|| <= 1e-6, iterations within 10 %
+                                                      -> asserted bit-identical x / history
+The oracle runs in kernel-order mode with the launch plan the library exports (PlanRows).
+"""
+import numpy as np
+import pytest
+
+import workloads as W
+
+pytestmark = pytest.mark.gpu
+
+torch = pytest.importorskip("torch")
+
+
+@pytest.fixture(scope="module")
+def mf():
+    if not torch.cuda.is_available():
+        pytest.skip("no CUDA device")
+    import paper_conf_sc_yangznjs0t024_b200 as m
+    m.build()
+    m.lib()
+    return m
+
+
+CANON = ("TileRowidx", "TileColidx", "TilePrec", "Floor", "TileNnz", "Nonrow", "ValOff", "TileRowPtr",
+         "RowIndex", "CsrRowptr", "CsrColidx", "Val64", "Val32", "Val16", "Val8")
+
+
+def oracle_tiles(orc, A, classify=True):
+    return orc.Tiles(A.n_rows, A.n_cols, A.rowptr, A.colidx, A.vals, classify=classify)
+
+
+def assert_canonical_equal(g, o):
+    for k in CANON:
+        a, b = g[k], o[k]
+        assert a.dtype == b.dtype and a.shape == b.shape, (k, a.shape, b.shape)
+        assert np.array_equal(a.view(np.uint8), b.view(np.uint8)), k
+
+
+def dev(x):
+    return torch.from_numpy(np.ascontiguousarray(x)).cuda()
+
+
+# ------------------------------------------------------------------------------ conversion
+CONVERT_CASES = [
+    ("rand-mixed-0", lambda: W.random_csr(257, 257, 0.05, 0, "mixed")),
+    ("rand-mixed-1", lambda: W.random_csr(100, 333, 0.08, 1, "mixed")),
+    ("rand-f64", lambda: W.random_csr(513, 513, 0.02, 2, "f64")),
+    ("rand-int", lambda: W.random_csr(45, 45, 0.3, 3, "int")),
+    ("C1", lambda: W.make("C1")),
+    ("C2-32", lambda: W.make("C2", 32)),
+    ("C3-64", lambda: W.make("C3", 64)),
+    ("C4spd-14", lambda: W.make("C4spd", 1 << 14)),
+    ("C4ind-12", lambda: W.make("C4ind", 1 << 12)),
+    ("poisson2d-33", lambda: W.poisson2d(33)),
+]
+
+
+@pytest.mark.parametrize("name,make", CONVERT_CASES, ids=[c[0] for c in CONVERT_CASES])
+@pytest.mark.parametrize("classify", [True, False])
+def test_convert_bit_exact(mf, orc, name, make, classify):
+    A = make()
+    g = mf.TileMatrix.from_host_csr(A, classify=classify).export()
+    assert_canonical_equal(g, oracle_tiles(orc, A, classify).arrays())
+
+
+def test_convert_value_edge_cases(mf, orc):
+    """Every closed-form classification vector, tiny / huge magnitudes (range floor), zeros."""
+    import json
+    import os
+    g = json.load(open(os.path.join(os.path.dirname(__file__), "golden", "classify_vectors.json")))
+    vals = [float(eval(e)) for e, _, _ in g["vectors"]]
+    vals += [1e-3, 3e-5, 7e4, 1e6, 1e30, 1e300, -2.0 ** -130, 5e-324, 0.0, 448.0, 464.0, 465.0, 65519.0]
+    vals = np.array(vals)
+    n = 64
+    rng = np.random.default_rng(0)
+    rows = np.sort(rng.integers(0, n, vals.size * 4))
+    cols = rng.integers(0, n, rows.size)
+    key = np.unique(rows * n + cols)
+    rows, cols = key // n, key % n
+    v = vals[rng.integers(0, vals.size, rows.size)]
+    rp = np.zeros(n + 1, np.int64)
+    np.cumsum(np.bincount(rows, minlength=n), out=rp[1:])
+    A = W.CSR(n, n, rp, cols.astype(np.int32), v)
+    gexp = mf.TileMatrix.from_host_csr(A).export()
+    assert_canonical_equal(gexp, oracle_tiles(orc, A).arrays())
+    # one value per tile: each tile's class equals the oracle's per-value class
+    for val in vals:
+        B = W.CSR(16, 16, np.array([0] + [1] * 16, np.int64), np.array([3], np.int32), np.array([val]))
+        assert_canonical_equal(mf.TileMatrix.from_host_csr(B).export(), oracle_tiles(orc, B).arrays())
+
+
+def test_convert_invalid_inputs(mf):
+    def conv(rp, ci, va, n=2):
+        return mf.TileMatrix(n, n, dev(np.array(rp, np.int64)), dev(np.array(ci, np.int32)),
+                             dev(np.array(va, np.float64)))
+    with pytest.raises(mf.MFError) as e:
+        conv([0, 2, 3], [1, 0, 1], [1, 1, 1])
+    assert e.value.status == 2
+    with pytest.raises(mf.MFError) as e:
+        conv([0, 2, 3], [0, 1, 1], [1, np.inf, 1])
+    assert e.value.status == 3
+    with pytest.raises(mf.MFError) as e:
+        conv([0, 2, 3], [0, 2, 1], [1, 1, 1])
+    assert e.value.status == 1
+    with pytest.raises(mf.MFError) as e:
+        conv([0, 3, 2], [0, 1, 1], [1, 1, 1])
+    assert e.value.status == 1
+    # empty matrix is fine
+    E = mf.TileMatrix(5, 5, dev(np.zeros(6, np.int64)), dev(np.zeros(0, np.int32)), dev(np.zeros(0)))
+    assert E.info()["tilenum"] == 0
+
+
+@pytest.mark.slow
+@pytest.mark.parametrize("name", ["C2", "C3"])
+def test_convert_full_size_bit_exact(mf, orc, name):
+    A = W.make(name)
+    assert_canonical_equal(mf.TileMatrix.from_host_csr(A).export(), oracle_tiles(orc, A).arrays())
+
+
+# ------------------------------------------------------------------------------ SpMV / levels / dot
+@pytest.mark.parametrize("name,make", CONVERT_CASES[:8], ids=[c[0] for c in CONVERT_CASES[:8]])
+@pytest.mark.parametrize("range_guard", [True, False])
+def test_spmv_bit_exact_with_levels(mf, orc, name, make, range_guard):
+    A = make()
+    T = oracle_tiles(orc, A)
+    G = mf.TileMatrix.from_host_csr(A)
+    rng = np.random.default_rng(7)
+    x = rng.standard_normal(A.n_cols) * np.exp2(rng.integers(-30, 5, A.n_cols))
+    for trial in range(3):
+        level = rng.integers(0, 5, (A.n_cols + 15) // 16).astype(np.uint8) if trial else None
+        yo, co = T.spmv(x, level, range_guard=range_guard)
+        yg, cg = G.spmv(dev(x), None if level is None else dev(level), range_guard=range_guard, counts=True)
+        assert np.array_equal(yg.cpu().numpy(), yo), trial
+        assert np.array_equal(cg, co)
+
+
+def test_levels_bit_exact(mf, orc):
+    rng = np.random.default_rng(3)
+    tau = 1.7e-9
+    th = np.array([tau * 1e-3, tau * 1e-2, tau * 1e-1, tau])
+    for n in (1, 15, 16, 17, 1000, 4099):
+        v = rng.standard_normal(n) * tau * np.exp2(rng.integers(-14, 3, n))
+        v[rng.random(n) < 0.1] = 0.0
+        v[::97] = th[rng.integers(0, 4)]     # exactly at a threshold
+        if n > 20:
+            v[5] = np.nan
+        assert np.array_equal(mf.levels(dev(v), th).cpu().numpy(), orc.levels(v, 16, th))
+
+
+@pytest.mark.parametrize("G,B", [(1, 1024), (3, 256), (8, 512), (37, 128)])
+def test_dot_tree_bit_exact(mf, orc, G, B):
+    A = W.poisson2d(70)      # n = 4900: ragged last tile row
+    T = mf.TileMatrix.from_host_csr(A, grid_ctas=G, block_threads=B)
+    g, b, R = T.plan()
+    assert (g, b) == (G, B) and R[0] == 0 and R[-1] == A.n_rows
+    rng = np.random.default_rng(G)
+    u, v = rng.standard_normal(A.n_rows), rng.standard_normal(A.n_rows)
+    assert T.dot(dev(u), dev(v)) == orc.dot(u, v, orc.Plan(G, B, R))
+
+
+# ------------------------------------------------------------------------------ solves
+def run_pair(mf, orc, A, solver, mode, classify=True, G=0, B=0, max_iter=1000, x0=None, b=None, **kw):
+    b = W.rhs_ones(A) if b is None else b
+    Gm = mf.TileMatrix.from_host_csr(A, classify=classify, grid_ctas=G, block_threads=B)
+    g, bb, R = Gm.plan()
+    plan = orc.Plan(g, bb, R)
+    T = oracle_tiles(orc, A, classify)
+    ofn = orc.cg if solver == "cg" else orc.bicgstab
+    gfn = mf.cg_solve if solver == "cg" else mf.bicgstab_solve
+    ro = ofn(T, b, x0=x0, mode=mode, plan=plan, max_iter=max_iter, **kw)
+    rg = gfn(Gm, dev(b), x0=None if x0 is None else dev(x0), mode=mode, max_iter=max_iter, level_counts=True,
+             raise_on_breakdown=False, **kw)
+    return ro, rg, Gm
+
+
+SOLVE_CASES = [
+    # name, matrix, solver, mode, classify, G, B
+    ("C1-fp64", lambda: W.make("C1"), "cg", 0, False, 0, 0),
+    ("C1-dyn-G1", lambda: W.make("C1"), "cg", 2, True, 1, 1024),
+    ("C1-dyn-G4", lambda: W.make("C1"), "cg", 2, True, 4, 256),
+    ("C2-32-dyn", lambda: W.make("C2", 32), "cg", 2, True, 8, 512),
+    ("C2-32-static", lambda: W.make("C2", 32), "cg", 1, True, 16, 1024),
+    ("C2-32-dyn-148", lambda: W.make("C2", 32), "cg", 2, True, 148, 128),
+    ("C3-64-dyn", lambda: W.make("C3", 64), "bicgstab", 2, True, 8, 512),
+    ("C3-64-fp64", lambda: W.make("C3", 64), "bicgstab", 0, False, 5, 256),
+    ("C4spd-dyn", lambda: W.make("C4spd", 1 << 13), "cg", 2, True, 12, 256),
+    ("C4ind-dyn", lambda: W.make("C4ind", 1 << 12), "bicgstab", 2, True, 6, 256),
+    ("ragged-dyn", lambda: W.poisson2d(33), "cg", 2, True, 3, 64),
+    ("ragged-bicg", lambda: W.convdiff2d(35), "bicgstab", 2, True, 4, 128),
+]
+
+
+@pytest.mark.parametrize("name,make,solver,mode,classify,G,B", SOLVE_CASES, ids=[c[0] for c in SOLVE_CASES])
+def test_solve_kernel_order_parity(mf, orc, name, make, solver, mode, classify, G, B):
+    A = make()
+    ro, rg, _ = run_pair(mf, orc, A, solver, mode, classify, G, B, max_iter=3000)
+    assert rg.status == ro["status"] == 0
+    assert rg.converged and ro["converged"]
+    assert rg.iterations == ro["iterations"]
+    ho, hg = ro["history"], rg.history
+    assert np.max(np.abs(hg - ho) / ho) <= 1e-12           # gate; expected exactly 0
+    assert np.array_equal(hg, ho)
+    xo, xg = ro["x"], rg.x.cpu().numpy()
+    assert np.linalg.norm(xg - xo) / np.linalg.norm(xo) <= 1e-6
+    assert np.array_equal(xg, xo)
+    if mode == 2:
+        assert np.array_equal(rg.level_counts, ro["level_counts"])
+
+
+def test_solve_edge_cases(mf, orc):
+    A = W.poisson2d(20)
+    # b == 0 -> x = 0, converged at iteration 0
+    ro, rg, _ = run_pair(mf, orc, A, "cg", 2, b=np.zeros(A.n_rows), x0=np.ones(A.n_rows))
+    assert rg.converged and rg.iterations == 0 and torch.all(rg.x == 0)
+    # max_iter reached: not an error
+    ro, rg, _ = run_pair(mf, orc, A, "cg", 2, max_iter=5)
+    assert rg.status == 0 and not rg.converged and rg.iterations == 5 and np.array_equal(rg.history, ro["history"])
+    # nonzero x0
+    x0 = np.random.default_rng(1).standard_normal(A.n_rows)
+    ro, rg, _ = run_pair(mf, orc, A, "cg", 2, x0=x0, G=3, B=128)
+    assert np.array_equal(rg.x.cpu().numpy(), ro["x"]) and rg.iterations == ro["iterations"]
+    ro, rg, _ = run_pair(mf, orc, W.convdiff2d(20), "bicgstab", 2, x0=x0, G=2, B=64)
+    assert np.array_equal(rg.x.cpu().numpy(), ro["x"]) and rg.iterations == ro["iterations"]
+    # breakdown on an indefinite matrix
+    D = W.CSR(32, 32, np.arange(33, dtype=np.int64), np.arange(32, dtype=np.int32),
+              np.where(np.arange(32) % 2 == 0, 1.0, -1.0))
+    ro, rg, _ = run_pair(mf, orc, D, "cg", 0, classify=False)
+    assert ro["status"] == 7 and rg.status == 7
+
+
+def test_torch_allocator_path(mf, orc):
+    import gc
+    mf.use_torch_allocator()
+    try:
+        A = W.make("C2", 16)
+        ro, rg, Gm = run_pair(mf, orc, A, "cg", 2, G=4, B=256)
+        assert np.array_equal(rg.x.cpu().numpy(), ro["x"])
+        Gm.close()
+        del Gm
+        gc.collect()
+    finally:
+        mf.lib().mf_set_allocator(mf._ALLOC_CB(0), mf._FREE_CB(0), None)
+
+
+@pytest.mark.slow
+def test_full_size_C2_parity(mf, orc):
+    """BASELINE configs[1] at full size, in the bench's launch configuration (auto plan)."""
+    A = W.make("C2")
+    ro, rg, Gm = run_pair(mf, orc, A, "cg", 2)
+    assert rg.converged and rg.iterations == ro["iterations"]
+    assert np.array_equal(rg.history, ro["history"])
+    assert np.array_equal(rg.x.cpu().numpy(), ro["x"])
+    b = W.rhs_ones(A)
+    assert orc.true_relres(A.rowptr, A.colidx, A.vals, b, rg.x.cpu().numpy()) < 1e-9
+
+
+@pytest.mark.slow
+def test_full_size_C3_prefix_and_convergence(mf, orc):
+    """C3 at full size: bit-identical first 25 iterations vs the oracle; the full GPU solve
+    reaches 1e-10 and its true residual is checked by the oracle."""
+    A = W.make("C3")
+    ro, rg, Gm = run_pair(mf, orc, A, "bicgstab", 2, max_iter=25, tol=0.0)
+    assert np.array_equal(rg.history, ro["history"]) and np.array_equal(rg.x.cpu().numpy(), ro["x"])
+    b = W.rhs_ones(A)
+    full = mf.bicgstab_solve(Gm, dev(b), max_iter=20000)
+    assert full.converged
+    tr = orc.true_relres(A.rowptr, A.colidx, A.vals, b, full.x.cpu().numpy())
+    assert tr < 1e-9
