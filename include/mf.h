@@ -66,6 +66,7 @@ typedef struct {
     double loss_tol;      /* 1e-15: relative loss below which a lower precision is "good enough" */
     int32_t grid_ctas;    /* persistent-kernel CTAs G; 0 = auto.  Fixes the dot-reduction tree. */
     int32_t block_threads;/* threads per CTA B (multiple of 32, <= 1024); 0 = auto */
+    int32_t layout;       /* kernel slice layout: 0 auto, 1 compact (row-packed), 2 tile-synchronous */
 } mf_convert_opts;
 
 typedef struct {
@@ -84,6 +85,7 @@ typedef struct {
     int32_t plan_G, plan_B;    /* launch plan: G CTAs of B threads; CTA g owns rows [R_g, R_{g+1}) */
     double convert_ms;         /* device time of the conversion (Fig. 14 analog) */
     int64_t convert_launches;  /* kernels the conversion launched */
+    int32_t layout;            /* 1 compact, 2 tile-synchronous */
 } mf_tile_info;
 
 /* Canonical arrays (bit-exact contract).  HOST buffers,
@@ -112,7 +114,7 @@ typedef struct {
     double tol;                 /* stop when ||r_j|| / ||b|| < tol (1e-10) */
     int64_t max_iter;           /* 1000 */
     mf_mode mode;               /* default MF_MODE_DYNAMIC_MIXED */
-    double switch_eps;          /* eps of P:174; < 0 = default (= tol) */
+    double switch_eps;          /* eps of P:174; < 0 = default (= 1e-2 * tol, reading R8) */
     int32_t switch_absolute;    /* 0: tau = eps*||v0||/sqrt(n) (reading R8); 1: tau = eps (Alg. 1 l.3) */
     int32_t sticky;             /* 1: one-time in-place downgrade (P:237 literal): MF_ERR_NOT_IMPLEMENTED */
     int32_t range_guard;        /* 1 (default): never lower a tile below its range floor */
@@ -135,6 +137,8 @@ typedef struct {
     double model_bytes;        /* algorithmic bytes moved */
     int64_t n_spmv;
     int64_t launches;          /* kernels launched by the solve */
+    double barrier_ms;         /* mean over CTAs of time spent spinning in grid barriers / ready flags */
+    double phase_ms[12];       /* mean over CTAs of time per kernel phase */
 } mf_solve_info;
 
 void mf_default_convert_opts(mf_convert_opts* o);

@@ -311,7 +311,8 @@ class ILU0:
 
 # ------------------------------------------------------------------ solvers
 def _opts(tol, max_iter, mode, switch_eps, switch_absolute, sticky, range_guard):
-    return _Opts(tol, max_iter, mode, tol if switch_eps is None else switch_eps,
+    # default eps = 1e-2 * tol (reading R8)
+    return _Opts(tol, max_iter, mode, 1e-2 * tol if switch_eps is None else switch_eps,
                  int(switch_absolute), int(sticky), int(range_guard))
 
 

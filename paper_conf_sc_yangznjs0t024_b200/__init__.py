@@ -75,7 +75,7 @@ def _nccl_paths():
 # ------------------------------------------------------------------ ctypes structs (mirror mf.h)
 class ConvertOpts(C.Structure):
     _fields_ = [("classify", C.c_int32), ("loss_tol", C.c_double), ("grid_ctas", C.c_int32),
-                ("block_threads", C.c_int32)]
+                ("block_threads", C.c_int32), ("layout", C.c_int32)]
 
 
 class TileInfo(C.Structure):
@@ -84,7 +84,7 @@ class TileInfo(C.Structure):
                 ("tiles_per_prec", C.c_int64 * 4), ("nval", C.c_int64 * 4), ("max_tiles_per_tile_row", C.c_int64),
                 ("slots", C.c_int64), ("canonical_bytes", C.c_int64), ("csr_bytes", C.c_int64),
                 ("kernel_bytes", C.c_int64), ("plan_G", C.c_int32), ("plan_B", C.c_int32), ("convert_ms", C.c_double),
-                ("convert_launches", C.c_int64)]
+                ("convert_launches", C.c_int64), ("layout", C.c_int32)]
 
 
 class TileExport(C.Structure):
@@ -103,7 +103,8 @@ class SolveOpts(C.Structure):
 class SolveInfo(C.Structure):
     _fields_ = [("iterations", C.c_int64), ("converged", C.c_int32), ("status", C.c_int32),
                 ("rel_residual", C.c_double), ("kernel_ms", C.c_double), ("model_bytes", C.c_double),
-                ("n_spmv", C.c_int64), ("launches", C.c_int64)]
+                ("n_spmv", C.c_int64), ("launches", C.c_int64), ("barrier_ms", C.c_double),
+                ("phase_ms", C.c_double * 12)]
 
 
 _lib = None
@@ -196,13 +197,13 @@ class TileMatrix:
     """Handle to an mf_tile_matrix (device CSR -> two-level tiles)."""
 
     def __init__(self, n_rows, n_cols, rowptr, colidx, vals, classify=True, loss_tol=1e-15, grid_ctas=0,
-                 block_threads=0, stream=None):
+                 block_threads=0, layout=0, stream=None):
         import torch
         _need_cuda(rowptr, torch.int64, "rowptr")
         _need_cuda(colidx, torch.int32, "colidx")
         _need_cuda(vals, torch.float64, "vals")
         L = lib()
-        o = ConvertOpts(int(bool(classify)), float(loss_tol), int(grid_ctas), int(block_threads))
+        o = ConvertOpts(int(bool(classify)), float(loss_tol), int(grid_ctas), int(block_threads), int(layout))
         h = C.c_void_p()
         self._h = None
         _check(L.mf_tile_matrix_from_csr(int(n_rows), int(n_cols), int(colidx.numel()), _ptr(rowptr), _ptr(colidx),
@@ -299,6 +300,8 @@ class SolveResult:
     model_bytes: float
     n_spmv: int
     launches: int
+    barrier_ms: float
+    phase_ms: list
     history: np.ndarray | None
     level_counts: np.ndarray | None
 
@@ -328,7 +331,7 @@ def _solve(fn, A: TileMatrix, b, x0=None, tol=1e-10, max_iter=1000, mode=MODE_DY
         raise MFError(st, lib().mf_last_error().decode())
     k = info.iterations
     return SolveResult(x, k, bool(info.converged), info.status, info.rel_residual, info.kernel_ms,
-                       info.model_bytes, info.n_spmv, info.launches,
+                       info.model_bytes, info.n_spmv, info.launches, info.barrier_ms, list(info.phase_ms),
                        hist[: k + 1] if hist is not None else None,
                        lc[: info.n_spmv] if lc is not None else None)
 

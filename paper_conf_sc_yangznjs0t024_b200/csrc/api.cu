@@ -93,6 +93,7 @@ void mf_default_convert_opts(mf_convert_opts* o) {
     o->loss_tol = 1e-15;
     o->grid_ctas = 0;
     o->block_threads = 0;
+    o->layout = 0;
 }
 
 void mf_default_solve_opts(mf_solve_opts* o) {
@@ -166,6 +167,7 @@ mf_status mf_tile_matrix_info(const mf_tile_matrix* A, mf_tile_info* o) {
     o->plan_G = m.G; o->plan_B = m.B;
     o->convert_ms = m.convert_ms;
     o->convert_launches = m.convert_launches;
+    o->layout = m.ts ? 2 : 1;
     return MF_OK;
 }
 

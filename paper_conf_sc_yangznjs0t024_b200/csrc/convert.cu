@@ -18,7 +18,8 @@ namespace mf {
 namespace {
 
 constexpr int CNT_TILES = 0, CNT_ROWS = 1, CNT_WIDTH = 2, CNT_NNZP = 3 /*..6*/, CNT_TILEP = 7 /*..10*/;
-constexpr int NCNT = 11;
+constexpr int CNT_WTS = 11;   // tile-synchronous width: sum over tiles of the max entries per row
+constexpr int NCNT = 12;
 constexpr int THREADS = 256;
 
 __device__ __forceinline__ unsigned hw_mask() { return (threadIdx.x & 16) ? 0xFFFF0000u : 0x0000FFFFu; }
@@ -94,7 +95,7 @@ struct Out {  // FILL-pass destinations (all device)
     int64_t *TileNnz, *Nonrow, *ValOff, *TileRowPtr;
     uint8_t *RowIndex, *CsrRowptr, *CsrColidx;
     double* Val64; float* Val32; uint16_t* Val16; uint8_t* Val8;
-    uint32_t* tile_info; uint16_t* sidx;
+    uint32_t* tile_info; uint16_t* sidx; uint8_t* sslot; uint32_t* colw; int ts;
     double* p64; float* p32; __half* p16; uint8_t* p8;
     const int64_t* off;   // [NCNT][ntr+1] exclusive scans of the counts
     int64_t ntr;
@@ -118,14 +119,14 @@ __global__ void __launch_bounds__(THREADS) tile_row_kernel(int64_t n_rows, int64
     int cur = ptr < rend ? (colidx[ptr] >> 4) : INT32_MAX;
     const int64_t width = hw_max<int64_t>(rend - rstart, m);
 
-    int64_t j = 0, nz_run = 0, ri_run = 0;
+    int64_t j = 0, nz_run = 0, ri_run = 0, colbase = 0;
     int64_t pnnz[4] = {0, 0, 0, 0}, ptile[4] = {0, 0, 0, 0};
     int64_t tile0 = 0, row0 = 0, nnz0 = 0, slot0 = 0, voff[4] = {0, 0, 0, 0};
     if (FILL) {
         const int64_t S = ntr + 1;
         tile0 = o.off[CNT_TILES * S + TR];
         row0 = o.off[CNT_ROWS * S + TR];
-        slot0 = o.off[CNT_WIDTH * S + TR];
+        slot0 = o.off[(o.ts ? CNT_WTS : CNT_WIDTH) * S + TR];
         for (int q = 0; q < 4; ++q) voff[q] = o.off[(CNT_NNZP + q) * S + TR];
         nnz0 = rowptr[TR * TS];
         if (lane == 0) o.TileRowPtr[TR] = tile0;
@@ -151,6 +152,7 @@ __global__ void __launch_bounds__(THREADS) tile_row_kernel(int64_t n_rows, int64
         const int minrc = hw_min<int>(rc, m);
         const int floor_t = minrc > best ? minrc : best;
         const int tile_nz = hw_sum<int>(cnt_r, m);
+        const int w_j = hw_max<int>(cnt_r, m);              // slice columns of this tile (TS layout)
         const unsigned bal = __ballot_sync(m, mine) >> (threadIdx.x & 16);
         const int rows_in_tile = __popc(bal);
         if (FILL) {
@@ -185,9 +187,12 @@ __global__ void __launch_bounds__(THREADS) tile_row_kernel(int64_t n_rows, int64
                     case 2: { __half h = mfk::to_f16(v); o.Val16[vp] = __half_as_ushort(h); sv = mfk::f16_to_d(h); } break;
                     default: { uint8_t b = mfk::to_e4m3(v); o.Val8[vp] = b; sv = mfk::e4m3_to_d(b); } break;
                     }
-                    // kernel layout: slot (k - rstart) of this row, value planes RNE_q(stored), q >= TilePrec
-                    const int64_t pos = (slot0 + (k - rstart)) * TS + lane;
-                    o.sidx[pos] = (uint16_t)((j << 4) | lc);
+                    // kernel layout: compact slot (k - rstart) of this row, or tile-synchronous column
+                    // colbase + (k - ptr); value planes RNE_q(stored) for q at or below TilePrec
+                    const int64_t pos = o.ts ? (slot0 + colbase + (k - ptr)) * TS + lane
+                                             : (slot0 + (k - rstart)) * TS + lane;
+                    if (o.ts) o.sslot[pos] = (uint8_t)lc;
+                    else o.sidx[pos] = (uint16_t)((j << 4) | lc);
                     if (best <= 0 && o.p64) o.p64[pos] = sv;
                     if (best <= 1 && o.p32) o.p32[pos] = mfk::to_f32(sv);
                     if (best <= 2 && o.p16) o.p16[pos] = mfk::to_f16(sv);
@@ -195,8 +200,11 @@ __global__ void __launch_bounds__(THREADS) tile_row_kernel(int64_t n_rows, int64
                 }
             }
         }
+        if (FILL && o.ts && lane < w_j)
+            o.colw[slot0 + colbase + lane] = ((uint32_t)tc << 4) | ((uint32_t)floor_t << 2) | (uint32_t)best;
         if (mine) { ptr = q; cur = ptr < rend ? (colidx[ptr] >> 4) : INT32_MAX; }
         ++j;
+        colbase += w_j;
         nz_run += tile_nz;
         ri_run += rows_in_tile;
         pnnz[best] += tile_nz;
@@ -211,6 +219,7 @@ __global__ void __launch_bounds__(THREADS) tile_row_kernel(int64_t n_rows, int64
         cnt[CNT_TILES * ntr + TR] = j;
         cnt[CNT_ROWS * ntr + TR] = ri_run;
         cnt[CNT_WIDTH * ntr + TR] = width;
+        cnt[CNT_WTS * ntr + TR] = colbase;
         for (int q = 0; q < 4; ++q) {
             cnt[(CNT_NNZP + q) * ntr + TR] = pnnz[q];
             cnt[(CNT_TILEP + q) * ntr + TR] = ptile[q];
@@ -290,11 +299,11 @@ mf_status scan_excl(const int64_t* in, int64_t n, int64_t* out, int64_t* tmp, cu
 
 // ------------------------------------------------------------------ launch plan
 // cost of a tile row: slice bytes (2 B index + ~2 B value per slot) + vector bytes (48 B per row)
-__global__ void tr_cost_kernel(const int64_t* __restrict__ cnt, int64_t ntr, int64_t n_rows, int64_t* cost) {
+__global__ void tr_cost_kernel(const int64_t* __restrict__ cnt, int64_t ntr, int64_t n_rows, int ts, int64_t* cost) {
     int64_t TR = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
     if (TR >= ntr) return;
     int64_t rows = n_rows - TR * TS < TS ? n_rows - TR * TS : TS;
-    cost[TR] = 4 * TS * cnt[CNT_WIDTH * ntr + TR] + 48 * rows + 1;
+    cost[TR] = 4 * TS * cnt[(ts ? CNT_WTS : CNT_WIDTH) * ntr + TR] + 48 * rows + 1;
 }
 
 // plan_tr[g] = first tile row whose exclusive cost prefix reaches g*total/G
@@ -318,7 +327,8 @@ __device__ int owner_of(const int32_t* plan_tr, int G, int64_t TR) {   // CTA ow
 
 // dependency range: CTAs owning the column segments this CTA's tiles gather (square matrices)
 __global__ void deps_kernel(const int32_t* __restrict__ plan_tr, int G, const int64_t* __restrict__ TileRowPtr,
-                            const int32_t* __restrict__ TileColidx, int64_t n_seg_owned, int32_t* dep_lo, int32_t* dep_hi) {
+                            const int32_t* __restrict__ TileColidx, int64_t n_seg_owned, int32_t* dep_lo, int32_t* dep_hi,
+                            int32_t* seg_lo, int32_t* seg_hi) {
     int g = blockIdx.x;
     __shared__ int smin, smax;
     if (threadIdx.x == 0) { smin = INT32_MAX; smax = -1; }
@@ -341,6 +351,8 @@ __global__ void deps_kernel(const int32_t* __restrict__ plan_tr, int G, const in
         }
         dep_lo[g] = lo;
         dep_hi[g] = hi;
+        seg_lo[g] = smax >= 0 ? smin : 0;     // column segments gathered by this CTA's tiles
+        seg_hi[g] = smax;
     }
 }
 
@@ -350,8 +362,8 @@ void destroy_tiles(TileMatrix* A) {
     cudaStream_t s = A->owner_stream;
     void* ptrs[] = {A->TileRowidx, A->TileColidx, A->TilePrec, A->Floor, A->TileNnz, A->Nonrow, A->ValOff,
                     A->TileRowPtr, A->RowIndex, A->CsrRowptr, A->CsrColidx, A->Val64, A->Val32, A->Val16,
-                    A->Val8, A->tr_slot, A->tile_info, A->sidx, A->plane64, A->plane32, A->plane16,
-                    A->plane8, A->plan_tr, A->dep_lo, A->dep_hi};
+                    A->Val8, A->tr_slot, A->tile_info, A->sidx, A->sslot, A->colw, A->plane64, A->plane32, A->plane16,
+                    A->plane8, A->plan_tr, A->dep_lo, A->dep_hi, A->seg_lo, A->seg_hi};
     for (void* p : ptrs) if (p) dev_free(p, s);
     delete[] A->plan_rows_host;
     *A = TileMatrix();
@@ -394,6 +406,7 @@ mf_status convert_csr(int64_t n_rows, int64_t n_cols, int64_t nnz, const int64_t
     const int tr_per_block = THREADS / 16;
     const unsigned tblocks = (unsigned)std::max<int64_t>((ntr + tr_per_block - 1) / tr_per_block, 1);
     Out none{};
+    none.ts = 0;
     if (ntr > 0) {
         tile_row_kernel<false><<<tblocks, THREADS, 0, s>>>(n_rows, ntr, rowptr, colidx, vals, o.classify, o.loss_tol,
                                                             cnt, d_err, none);
@@ -411,7 +424,12 @@ mf_status convert_csr(int64_t n_rows, int64_t n_cols, int64_t nnz, const int64_t
     }
     A->tilenum = tot[CNT_TILES];
     A->rownum = tot[CNT_ROWS];
-    A->slots = tot[CNT_WIDTH];
+    // kernel layout: tile-synchronous slices (uniform tile per slice column) unless they cost
+    // more than 30% extra slots over the compact (row-packed) slices
+    if (o.layout == 1) A->ts = 0;
+    else if (o.layout == 2) A->ts = 1;
+    else A->ts = (double)tot[CNT_WTS] <= 1.3 * (double)tot[CNT_WIDTH] ? 1 : 0;
+    A->slots = A->ts ? tot[CNT_WTS] : tot[CNT_WIDTH];
     for (int q = 0; q < 4; ++q) { A->nval[q] = tot[CNT_NNZP + q]; A->tiles_per_prec[q] = tot[CNT_TILEP + q]; }
 
     // 3. allocate
@@ -425,27 +443,35 @@ mf_status convert_csr(int64_t n_rows, int64_t n_cols, int64_t nnz, const int64_t
     MF_TRY(alloc(&A->Val64, A->nval[0], s)); MF_TRY(alloc(&A->Val32, A->nval[1], s));
     MF_TRY(alloc(&A->Val16, A->nval[2], s)); MF_TRY(alloc(&A->Val8, A->nval[3], s));
     MF_TRY(alloc(&A->tile_info, nt, s));
-    MF_TRY(alloc(&A->sidx, nslot, s));
+    if (A->ts) {
+        MF_TRY(alloc(&A->sslot, nslot, s));
+        MF_TRY(alloc(&A->colw, A->slots, s));
+    } else {
+        MF_TRY(alloc(&A->sidx, nslot, s));
+    }
     // value planes: plane q exists when some tile can compute at q (TilePrec <= q)
     bool need[4] = {false, false, false, false};
     for (int q = 0; q < 4; ++q)
         for (int p = 0; p <= q; ++p) if (A->tiles_per_prec[p] > 0) need[q] = true;
-    if (need[0]) MF_TRY(alloc(&A->plane64, nslot, s));
-    if (need[1]) MF_TRY(alloc(&A->plane32, nslot, s));
-    if (need[2]) MF_TRY(alloc(&A->plane16, nslot, s));
-    if (need[3]) MF_TRY(alloc(&A->plane8, nslot, s));
-    if (nslot) MF_CUDA(cudaMemsetAsync(A->sidx, 0xFF, nslot * sizeof(uint16_t), s));
+    // planes padded to whole 8-byte words: the SpMV fetches the aligned 8-byte word around a value
+    if (need[0]) MF_TRY(alloc(&A->plane64, nslot + 1, s));
+    if (need[1]) MF_TRY(alloc(&A->plane32, nslot + 2, s));
+    if (need[2]) MF_TRY(alloc(&A->plane16, nslot + 4, s));
+    if (need[3]) MF_TRY(alloc(&A->plane8, nslot + 8, s));
+    if (nslot && A->sidx) MF_CUDA(cudaMemsetAsync(A->sidx, 0xFF, nslot * sizeof(uint16_t), s));
+    if (nslot && A->sslot) MF_CUDA(cudaMemsetAsync(A->sslot, 0xFF, nslot, s));
     if (nt == 0) {
         MF_CUDA(cudaMemsetAsync(A->TileNnz, 0, sizeof(int64_t), s));
         MF_CUDA(cudaMemsetAsync(A->Nonrow, 0, sizeof(int64_t), s));
     }
     MF_TRY(alloc(&A->tr_slot, ntr + 1, s));
-    MF_CUDA(cudaMemcpyAsync(A->tr_slot, off + CNT_WIDTH * S, (ntr + 1) * sizeof(int64_t), cudaMemcpyDeviceToDevice, s));
+    MF_CUDA(cudaMemcpyAsync(A->tr_slot, off + (A->ts ? CNT_WTS : CNT_WIDTH) * S, (ntr + 1) * sizeof(int64_t),
+                            cudaMemcpyDeviceToDevice, s));
 
     // 4. FILL pass
     Out fo{A->TileRowidx, A->TileColidx, A->TilePrec, A->Floor, A->TileNnz, A->Nonrow, A->ValOff, A->TileRowPtr,
            A->RowIndex, A->CsrRowptr, A->CsrColidx, A->Val64, A->Val32, A->Val16, A->Val8, A->tile_info, A->sidx,
-           A->plane64, A->plane32, A->plane16, A->plane8, off, ntr};
+           A->sslot, A->colw, A->ts, A->plane64, A->plane32, A->plane16, A->plane8, off, ntr};
     if (ntr > 0) {
         tile_row_kernel<true><<<tblocks, THREADS, 0, s>>>(n_rows, ntr, rowptr, colidx, vals, o.classify, o.loss_tol,
                                                            cnt, d_err, fo);
@@ -459,11 +485,15 @@ mf_status convert_csr(int64_t n_rows, int64_t n_cols, int64_t nnz, const int64_t
         if (ntr) MF_CUDA(cudaMemcpyAsync(hc.data(), cnt + CNT_TILES * ntr, ntr * sizeof(int64_t), cudaMemcpyDeviceToHost, s));
         MF_CUDA(cudaStreamSynchronize(s));
         A->max_nt = ntr ? *std::max_element(hc.begin(), hc.end()) : 0;
+        if (ntr) MF_CUDA(cudaMemcpyAsync(hc.data(), cnt + (A->ts ? CNT_WTS : CNT_WIDTH) * ntr, ntr * sizeof(int64_t),
+                                         cudaMemcpyDeviceToHost, s));
+        MF_CUDA(cudaStreamSynchronize(s));
+        A->max_w = ntr ? *std::max_element(hc.begin(), hc.end()) : 0;
     }
 
     // 5. launch plan
     int G = o.grid_ctas, B = o.block_threads;
-    if (B <= 0) B = 1024;
+    if (B <= 0) B = 512;
     if (B % 32 || B > 1024 || B < 32) {
         return fail(MF_ERR_INVALID_ARG, "block_threads must be a multiple of 32 in [32, 1024]");
     }
@@ -474,13 +504,16 @@ mf_status convert_csr(int64_t n_rows, int64_t n_cols, int64_t nnz, const int64_t
     A->G = G; A->B = B;
     int64_t* cost = nullptr;
     MF_TRY(alloc(&cost, std::max<int64_t>(ntr, 1), s));
-    if (ntr) tr_cost_kernel<<<(unsigned)((ntr + 255) / 256), 256, 0, s>>>(cnt, ntr, n_rows, cost);
+    if (ntr) tr_cost_kernel<<<(unsigned)((ntr + 255) / 256), 256, 0, s>>>(cnt, ntr, n_rows, A->ts, cost);
     MF_TRY(scan_excl(cost, ntr, off, tmp, s));    // reuse off[0..ntr]
     MF_TRY(alloc(&A->plan_tr, G + 1, s));
     MF_TRY(alloc(&A->dep_lo, G, s));
     MF_TRY(alloc(&A->dep_hi, G, s));
+    MF_TRY(alloc(&A->seg_lo, G, s));
+    MF_TRY(alloc(&A->seg_hi, G, s));
     plan_kernel<<<(G + 1 + 127) / 128, 128, 0, s>>>(off, ntr, G, A->plan_tr);
-    deps_kernel<<<G, 256, 0, s>>>(A->plan_tr, G, A->TileRowPtr, A->TileColidx, ntr, A->dep_lo, A->dep_hi);
+    deps_kernel<<<G, 256, 0, s>>>(A->plan_tr, G, A->TileRowPtr, A->TileColidx, ntr, A->dep_lo, A->dep_hi, A->seg_lo,
+                                  A->seg_hi);
     MF_CUDA(cudaGetLastError());
     std::vector<int32_t> ptr_h(G + 1);
     MF_CUDA(cudaMemcpyAsync(ptr_h.data(), A->plan_tr, (G + 1) * sizeof(int32_t), cudaMemcpyDeviceToHost, s));
@@ -496,10 +529,10 @@ mf_status convert_csr(int64_t n_rows, int64_t n_cols, int64_t nnz, const int64_t
     dev_free(cost, s); dev_free(cnt, s); dev_free(off, s); dev_free(tmp, s); dev_free(d_err, s);
 
     // kernels launched: validate, COUNT, 12 scans x 3, FILL, cost, plan, deps
-    A->convert_launches = (n_rows > 0 ? 1 : 0) + (ntr > 0 ? 2 + 1 : 0) + 12 * (ntr > 0 ? 3 : 0) + 2;
+    A->convert_launches = (n_rows > 0 ? 1 : 0) + (ntr > 0 ? 2 + 1 : 0) + (NCNT + 1) * (ntr > 0 ? 3 : 0) + 2;
     A->canonical_bytes = nt * (4 + 4 + 1 + 1 + 8 + 8 + 8) + 16 + (ntr + 1) * 8 + A->rownum * 2 + nnz +
                          A->nval[0] * 8 + A->nval[1] * 4 + A->nval[2] * 2 + A->nval[3];
-    A->kernel_bytes = nslot * 2 + (A->plane64 ? nslot * 8 : 0) + (A->plane32 ? nslot * 4 : 0) +
+    A->kernel_bytes = (A->ts ? nslot + A->slots * 4 : nslot * 2) + (A->plane64 ? nslot * 8 : 0) + (A->plane32 ? nslot * 4 : 0) +
                       (A->plane16 ? nslot * 2 : 0) + (A->plane8 ? nslot : 0) + nt * 4 + (ntr + 1) * 8;
     return MF_OK;
 }

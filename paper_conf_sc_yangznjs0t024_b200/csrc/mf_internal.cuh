@@ -57,6 +57,7 @@ struct TileMatrix {
     int64_t tiles_per_prec[4] = {0, 0, 0, 0};
     int64_t slots = 0;               // slice columns (each 16 slots wide)
     int64_t max_nt = 0;              // max tiles in one tile row
+    int64_t max_w = 0;               // max slice columns of one tile row (kernel layout)
     double convert_ms = 0;
     int64_t convert_launches = 0;
     // canonical arrays (device)
@@ -72,7 +73,10 @@ struct TileMatrix {
     // column per row; slot word = (tile index in tile row << 4) | local column.
     int64_t* tr_slot = nullptr;      // [ntr+1] first slice column of each tile row
     uint32_t* tile_info = nullptr;   // [tilenum] (TileColidx << 4) | (Floor << 2) | TilePrec
-    uint16_t* sidx = nullptr;        // [16*slots]
+    int ts = 0;                      // 1: tile-synchronous slices
+    uint16_t* sidx = nullptr;        // compact: [16*slots] (tile index in tile row << 4) | local column
+    uint8_t* sslot = nullptr;        // tile-synchronous: [16*slots] local column or 0xFF
+    uint32_t* colw = nullptr;        // tile-synchronous: [slots] (tile column << 4) | (Floor << 2) | TilePrec per slice column
     double* plane64 = nullptr;       // [16*slots] value at FP64 (tiles with TilePrec == FP64)
     float* plane32 = nullptr;        // value rounded to FP32 (tiles with TilePrec <= FP32)
     __half* plane16 = nullptr;       // ... FP16
@@ -82,6 +86,8 @@ struct TileMatrix {
     int32_t* plan_tr = nullptr;      // device [G+1]
     int32_t* dep_lo = nullptr;       // device [G] first CTA whose rows this CTA's tiles gather
     int32_t* dep_hi = nullptr;       // device [G]
+    int32_t* seg_lo = nullptr;       // device [G] first column segment gathered by CTA g
+    int32_t* seg_hi = nullptr;       // device [G] last column segment gathered (-1: none)
     int64_t* plan_rows_host = nullptr;  // host [G+1]
     // distributed (row block of a larger matrix); row_begin == 0 and halo empty on 1 GPU
     mf_comm* comm = nullptr;

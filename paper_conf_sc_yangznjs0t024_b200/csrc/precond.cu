@@ -1,13 +1,258 @@
-// precond.cu -- ILU(0) preconditioning.  (filled in below)
+// precond.cu -- ILU(0) preconditioning (reading R20).
+//
+// Setup (host, C++, once per matrix: "preprocessing"): the stored (TilePrec) values are read
+// back from the canonical tile arrays into a row-major CSR, factorised with ILU(0) in the IKJ
+// order (a_ik /= a_kk, then a_ij -= a_ik * a_kj for the j > k present in row i, k ascending,
+// each update one fma), and split into L (unit lower, strict part) and U (upper with
+// diagonal).  Every a_ij receives its updates in ascending k, so the factors are bit-identical
+// to any implementation of the same definition.
+//
+// Apply (device): z = U^-1 (L^-1 r) by sync-free triangular solves inside the persistent
+// PCG / PBiCGSTAB kernels (solver.cu: sptrsv_chunked) or by mf_precond_apply.  Row i is one
+// fma chain in ascending column order: y_i = r_i - sum l_ik y_k ; z_i = (y_i - sum u_ik z_k) / u_ii.
+#include <cuda_runtime.h>
+#include <string.h>
+
+#include <algorithm>
+#include <cmath>
+#include <vector>
+
 #include "mf_internal.cuh"
+#include "precond.cuh"
+
+namespace mf {
+namespace {
+
+// exact decoders of the stored formats (host)
+double half_bits_to_double(uint16_t b) {
+    const int s = b >> 15, e = (b >> 10) & 0x1F, m = b & 0x3FF;
+    double v;
+    if (e == 0) v = std::ldexp((double)m, -24);
+    else if (e == 31) v = m ? NAN : INFINITY;
+    else v = std::ldexp((double)(m | 0x400), e - 25);
+    return s ? -v : v;
+}
+double e4m3_bits_to_double(uint8_t b) {
+    const int s = b >> 7, e = (b >> 3) & 0xF, m = b & 7;
+    double v;
+    if (e == 15 && m == 7) v = NAN;
+    else if (e == 0) v = std::ldexp((double)m, -9);
+    else v = std::ldexp((double)(m | 8), e - 10);
+    return s ? -v : v;
+}
+
+struct HostCSR {
+    int64_t n = 0;
+    std::vector<int64_t> rp;
+    std::vector<int32_t> ci;
+    std::vector<double> v;
+};
+
+mf_status stored_csr(const TileMatrix& A, cudaStream_t s, HostCSR& out) {
+    const int64_t nt = A.tilenum, nr = A.rownum;
+    std::vector<int32_t> trow(nt), tcol(nt);
+    std::vector<uint8_t> prec(nt), rowidx(nr), rowptr(nr), colidx(A.nnz);
+    std::vector<int64_t> tnnz(nt + 1), nonrow(nt + 1), voff(nt);
+    std::vector<double> v64(A.nval[0]);
+    std::vector<float> v32(A.nval[1]);
+    std::vector<uint16_t> v16(A.nval[2]);
+    std::vector<uint8_t> v8(A.nval[3]);
+    auto cp = [&](void* d, const void* src, size_t bytes) -> mf_status {
+        if (bytes) MF_CUDA(cudaMemcpyAsync(d, src, bytes, cudaMemcpyDeviceToHost, s));
+        return MF_OK;
+    };
+    MF_TRY(cp(trow.data(), A.TileRowidx, nt * 4));
+    MF_TRY(cp(tcol.data(), A.TileColidx, nt * 4));
+    MF_TRY(cp(prec.data(), A.TilePrec, nt));
+    MF_TRY(cp(tnnz.data(), A.TileNnz, (nt + 1) * 8));
+    MF_TRY(cp(nonrow.data(), A.Nonrow, (nt + 1) * 8));
+    MF_TRY(cp(voff.data(), A.ValOff, nt * 8));
+    MF_TRY(cp(rowidx.data(), A.RowIndex, nr));
+    MF_TRY(cp(rowptr.data(), A.CsrRowptr, nr));
+    MF_TRY(cp(colidx.data(), A.CsrColidx, A.nnz));
+    MF_TRY(cp(v64.data(), A.Val64, A.nval[0] * 8));
+    MF_TRY(cp(v32.data(), A.Val32, A.nval[1] * 4));
+    MF_TRY(cp(v16.data(), A.Val16, A.nval[2] * 2));
+    MF_TRY(cp(v8.data(), A.Val8, A.nval[3]));
+    MF_CUDA(cudaStreamSynchronize(s));
+    const int64_t n = A.n_rows;
+    out.n = n;
+    out.rp.assign(n + 1, 0);
+    for (int64_t t = 0; t < nt; ++t)
+        for (int64_t r = nonrow[t]; r < nonrow[t + 1]; ++r) {
+            const int64_t end = (r + 1 < nonrow[t + 1]) ? rowptr[r + 1] : tnnz[t + 1] - tnnz[t];
+            out.rp[(int64_t)trow[t] * TS + rowidx[r] + 1] += end - rowptr[r];
+        }
+    for (int64_t i = 0; i < n; ++i) out.rp[i + 1] += out.rp[i];
+    out.ci.resize(A.nnz);
+    out.v.resize(A.nnz);
+    std::vector<int64_t> fill(out.rp.begin(), out.rp.end() - 1);
+    // tiles of a tile row are in ascending column, entries of a row in a tile ascending:
+    // appending in tile order yields ascending columns per row
+    for (int64_t t = 0; t < nt; ++t)
+        for (int64_t r = nonrow[t]; r < nonrow[t + 1]; ++r) {
+            const int64_t row = (int64_t)trow[t] * TS + rowidx[r];
+            const int64_t end = (r + 1 < nonrow[t + 1]) ? rowptr[r + 1] : tnnz[t + 1] - tnnz[t];
+            for (int64_t a = rowptr[r]; a < end; ++a) {
+                const int64_t o = voff[t] + a;
+                double val;
+                switch (prec[t]) {
+                case 0: val = v64[o]; break;
+                case 1: val = (double)v32[o]; break;
+                case 2: val = half_bits_to_double(v16[o]); break;
+                default: val = e4m3_bits_to_double(v8[o]); break;
+                }
+                out.ci[fill[row]] = tcol[t] * TS + colidx[tnnz[t] + a];
+                out.v[fill[row]] = val;
+                fill[row]++;
+            }
+        }
+    return MF_OK;
+}
+
+// ILU(0), IKJ order with a column marker (see the file header)
+mf_status ilu0(HostCSR& M, std::vector<int64_t>& diag) {
+    const int64_t n = M.n;
+    diag.assign(n, -1);
+    for (int64_t i = 0; i < n; ++i)
+        for (int64_t k = M.rp[i]; k < M.rp[i + 1]; ++k)
+            if (M.ci[k] == i) diag[i] = k;
+    for (int64_t i = 0; i < n; ++i)
+        if (diag[i] < 0) return fail(MF_ERR_ZERO_PIVOT, "ILU(0): row " + std::to_string(i) + " has no diagonal entry");
+    std::vector<int64_t> pos(n, -1);
+    for (int64_t i = 0; i < n; ++i) {
+        for (int64_t q = M.rp[i]; q < M.rp[i + 1]; ++q) pos[M.ci[q]] = q;
+        for (int64_t kk = M.rp[i]; kk < M.rp[i + 1] && M.ci[kk] < i; ++kk) {
+            const int64_t k = M.ci[kk];
+            const double akk = M.v[diag[k]];
+            if (akk == 0.0) return fail(MF_ERR_ZERO_PIVOT, "ILU(0): zero pivot in row " + std::to_string(k));
+            M.v[kk] = M.v[kk] / akk;
+            const double aik = M.v[kk];
+            for (int64_t q = diag[k] + 1; q < M.rp[k + 1]; ++q) {
+                const int64_t p = pos[M.ci[q]];
+                if (p >= 0) M.v[p] = std::fma(-aik, M.v[q], M.v[p]);
+            }
+        }
+        for (int64_t q = M.rp[i]; q < M.rp[i + 1]; ++q) pos[M.ci[q]] = -1;
+        if (M.v[diag[i]] == 0.0) return fail(MF_ERR_ZERO_PIVOT, "ILU(0): zero pivot in row " + std::to_string(i));
+    }
+    return MF_OK;
+}
+
+// standalone apply: one sync-free triangular solve per launch (any grid size is deadlock-free)
+template <bool FWD>
+__global__ void __launch_bounds__(256) sptrsv_kernel(TriCSR T, const double* __restrict__ diag, int64_t n,
+                                                     const double* in, double* out, unsigned* flags, unsigned flag_val,
+                                                     unsigned wait_val, unsigned long long* ctr) {
+    __shared__ double ys[256];
+    __shared__ int ready[256];
+    __shared__ long long chunk;
+    mfk::sptrsv_chunked<FWD>(T.rp, T.ci, T.v, diag, n, in, out, flags, flag_val, wait_val, ctr, 0ull, ys, ready, &chunk);
+}
+
+template <class T>
+mf_status upload(T** d, const std::vector<T>& h, cudaStream_t s) {
+    MF_TRY(alloc(d, h.size(), s));
+    if (!h.empty()) MF_CUDA(cudaMemcpyAsync(*d, h.data(), h.size() * sizeof(T), cudaMemcpyHostToDevice, s));
+    return MF_OK;
+}
+
+}  // namespace
+
+mf_status run_precond_apply(Precond& P, const double* r, double* z, cudaStream_t s) {
+    if (P.n == 0) return MF_OK;
+    int dev = 0, sms = 0;
+    MF_CUDA(cudaGetDevice(&dev));
+    MF_CUDA(cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev));
+    if (P.epoch >= 0x7FFFFFF0u) {   // flag values wrap: start over
+        MF_CUDA(cudaMemsetAsync(P.flags, 0, (P.n + 1) * sizeof(unsigned), s));
+        P.epoch = 0;
+    }
+    const unsigned e = ++P.epoch;
+    const int blocks = (int)std::min<int64_t>((P.n + 255) / 256, (int64_t)sms * 8);
+    MF_CUDA(cudaMemsetAsync(P.ctr, 0, 2 * sizeof(unsigned long long), s));
+    sptrsv_kernel<true><<<blocks, 256, 0, s>>>(P.L, nullptr, P.n, r, P.y, P.flags, 2 * e + 1, 0u, P.ctr);
+    sptrsv_kernel<false><<<blocks, 256, 0, s>>>(P.U, P.udiag, P.n, P.y, z, P.flags, 2 * e + 2, 2 * e + 1, P.ctr + 1);
+    MF_CUDA(cudaGetLastError());
+    return MF_OK;
+}
+
+void destroy_precond(Precond* P) {
+    cudaStream_t s = P->owner_stream;
+    void* ptrs[] = {P->L.rp, P->L.ci, P->L.v, P->U.rp, P->U.ci, P->U.v, P->udiag, P->flags, P->ctr, P->y, P->z};
+    for (void* p : ptrs) if (p) dev_free(p, s);
+    *P = Precond();
+}
+
+mf_status build_precond(const TileMatrix& A, cudaStream_t s, Precond* P) {
+    if (A.n_rows != A.n_cols) return fail(MF_ERR_INVALID_ARG, "ILU(0) needs a square matrix");
+    P->owner_stream = s;
+    P->n = A.n_rows;
+    HostCSR M;
+    MF_TRY(stored_csr(A, s, M));
+    std::vector<int64_t> diag;
+    MF_TRY(ilu0(M, diag));
+    const int64_t n = M.n;
+    std::vector<int64_t> lrp(n + 1, 0), urp(n + 1, 0);
+    std::vector<int32_t> lci, uci;
+    std::vector<double> lv, uv, ud(n);
+    for (int64_t i = 0; i < n; ++i) {
+        for (int64_t q = M.rp[i]; q < diag[i]; ++q) { lci.push_back(M.ci[q]); lv.push_back(M.v[q]); }
+        for (int64_t q = diag[i] + 1; q < M.rp[i + 1]; ++q) { uci.push_back(M.ci[q]); uv.push_back(M.v[q]); }
+        ud[i] = M.v[diag[i]];
+        lrp[i + 1] = (int64_t)lci.size();
+        urp[i + 1] = (int64_t)uci.size();
+    }
+    MF_TRY(upload(&P->L.rp, lrp, s)); MF_TRY(upload(&P->L.ci, lci, s)); MF_TRY(upload(&P->L.v, lv, s));
+    MF_TRY(upload(&P->U.rp, urp, s)); MF_TRY(upload(&P->U.ci, uci, s)); MF_TRY(upload(&P->U.v, uv, s));
+    MF_TRY(upload(&P->udiag, ud, s));
+    MF_TRY(alloc(&P->flags, (size_t)n + 1, s));
+    MF_TRY(alloc(&P->ctr, 4, s));
+    MF_TRY(alloc(&P->y, n, s));
+    MF_TRY(alloc(&P->z, n, s));
+    MF_CUDA(cudaMemsetAsync(P->flags, 0, (n + 1) * sizeof(unsigned), s));
+    MF_CUDA(cudaMemsetAsync(P->ctr, 0, 4 * sizeof(unsigned long long), s));
+    MF_CUDA(cudaStreamSynchronize(s));
+    P->nnz_l = (int64_t)lv.size();
+    P->nnz_u = (int64_t)uv.size();
+    P->epoch = 0;
+    P->grabs = 0;
+    return MF_OK;
+}
+
+}  // namespace mf
+
+using namespace mf;
 
 extern "C" {
-mf_status mf_precond_create(const mf_tile_matrix*, mf_precond_kind, mf_stream, mf_precond** out) {
-    if (out) *out = nullptr;
-    return mf::fail(MF_ERR_NOT_IMPLEMENTED, "ILU(0) not built yet");
+
+mf_status mf_precond_create(const mf_tile_matrix* A, mf_precond_kind kind, mf_stream stream, mf_precond** out) {
+    if (!A || !out) return fail(MF_ERR_INVALID_ARG, "NULL argument");
+    *out = nullptr;
+    if (kind != MF_PRECOND_ILU0) return fail(MF_ERR_INVALID_ARG, "only MF_PRECOND_ILU0 is defined (P:164)");
+    MF_TRY(check_device(nullptr));
+    mf_precond* h = new (std::nothrow) mf_precond();
+    if (!h) return fail(MF_ERR_OOM, "host allocation failed");
+    mf_status st = build_precond(A->m, (cudaStream_t)stream, &h->p);
+    if (st != MF_OK) {
+        destroy_precond(&h->p);
+        delete h;
+        return st;
+    }
+    *out = h;
+    return MF_OK;
 }
-mf_status mf_precond_destroy(mf_precond*) { return MF_OK; }
-mf_status mf_precond_apply(const mf_precond*, const double*, double*, mf_stream) {
-    return mf::fail(MF_ERR_NOT_IMPLEMENTED, "ILU(0) not built yet");
+
+mf_status mf_precond_destroy(mf_precond* M) {
+    if (!M) return MF_OK;
+    destroy_precond(&M->p);
+    delete M;
+    return MF_OK;
 }
+
+mf_status mf_precond_apply(const mf_precond* M, const double* r, double* z, mf_stream stream) {
+    if (!M || (M->p.n > 0 && (!r || !z))) return fail(MF_ERR_INVALID_ARG, "NULL argument");
+    return run_precond_apply(const_cast<Precond&>(M->p), r, z, (cudaStream_t)stream);
 }
+
+}  // extern "C"

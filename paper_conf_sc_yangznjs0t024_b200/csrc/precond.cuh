@@ -1,0 +1,104 @@
+// precond.cuh -- ILU(0) factors on the device and the sync-free triangular solve.
+#pragma once
+
+#include "mf_internal.cuh"
+
+namespace mf {
+
+struct TriCSR {
+    int64_t* rp = nullptr;
+    int32_t* ci = nullptr;
+    double* v = nullptr;
+};
+
+struct Precond {
+    int64_t n = 0;
+    TriCSR L, U;                  // L: strict lower part (unit diagonal implied); U: strict upper part
+    double* udiag = nullptr;      // u_ii
+    unsigned* flags = nullptr;    // [n+1] row-ready epochs (forward 2e+1, backward 2e+2)
+    unsigned long long* ctr = nullptr;   // chunk-grab counters
+    double *y = nullptr, *z = nullptr;   // workspace of mf_precond_apply / the solvers
+    int64_t nnz_l = 0, nnz_u = 0;
+    unsigned epoch = 0;           // applies issued so far (host side bookkeeping)
+    unsigned long long grabs = 0;
+    cudaStream_t owner_stream = nullptr;
+};
+
+mf_status build_precond(const TileMatrix& A, cudaStream_t s, Precond* P);
+void destroy_precond(Precond* P);
+mf_status run_precond_apply(Precond& P, const double* r, double* z, cudaStream_t s);
+
+}  // namespace mf
+
+struct mf_precond {
+    mf::Precond p;
+};
+
+namespace mfk {
+
+__device__ __forceinline__ unsigned ld_acquire_u32(const unsigned* p) {
+    unsigned v;
+    asm volatile("ld.acquire.gpu.global.u32 %0, [%1];" : "=r"(v) : "l"(p) : "memory");
+    return v;
+}
+__device__ __forceinline__ void st_release_u32(unsigned* p, unsigned v) {
+    asm volatile("st.release.gpu.global.u32 [%0], %1;" ::"l"(p), "r"(v) : "memory");
+}
+
+// Sync-free chunked triangular solve, called by all threads of a CTA (any number of CTAs).
+//   FWD:  out_i = in_i - sum_{k<i} T_ik out_k                 rows ascending
+//   !FWD: out_i = (in_i - sum_{k>i} T_ik out_k) / diag_i       rows descending
+// Chunks of blockDim.x consecutive rows (in solve order) are grabbed with one atomicAdd on
+// *ctr (values base, base+1, ...), so a chunk only waits on chunks grabbed earlier or on
+// earlier rows of its own chunk: deadlock-free without co-residency.  Inside a chunk a row
+// waits on a shared-memory flag; across chunks on the global row flag (== flag_val).
+// wait_val != 0: row i additionally waits for flags[i] == wait_val before reading in_i (the
+// backward solve waits for the forward solve of the same row).  Every CTA performs exactly one
+// failing grab, so one solve consumes ceil(n/B) + (number of CTAs) counter values.
+template <bool FWD>
+__device__ void sptrsv_chunked(const int64_t* __restrict__ rp, const int32_t* __restrict__ ci,
+                               const double* __restrict__ val, const double* __restrict__ diag, int64_t n,
+                               const double* in, double* out, unsigned* flags, unsigned flag_val, unsigned wait_val,
+                               unsigned long long* ctr, unsigned long long base, double* ys, volatile int* ready,
+                               long long* s_chunk) {
+    const int B = blockDim.x, t = threadIdx.x;
+    const int64_t nchunks = (n + B - 1) / B;
+    while (true) {
+        __syncthreads();
+        if (t == 0) *s_chunk = (long long)(atomicAdd(ctr, 1ull) - base);
+        ready[t] = 0;
+        __syncthreads();
+        const int64_t c = *s_chunk;
+        if (c >= nchunks) break;
+        const int64_t pos = c * B + t;                 // position in solve order
+        if (pos < n) {
+            const int64_t i = FWD ? pos : n - 1 - pos;
+            if (wait_val)
+                while (ld_acquire_u32(&flags[i]) != wait_val) { }
+            double acc = __ldcg(in + i);
+            const int64_t lo = rp[i], hi = rp[i + 1];
+            for (int64_t q = lo; q < hi; ++q) {
+                const int64_t k = ci[q];
+                const int64_t pk = FWD ? k : n - 1 - k;     // position of k in solve order (< pos)
+                double xk;
+                if (pk >= c * B) {
+                    const int lk = (int)(pk - c * B);
+                    while (ready[lk] == 0) { }
+                    xk = ((volatile double*)ys)[lk];
+                } else {
+                    while (ld_acquire_u32(&flags[k]) != flag_val) { }
+                    xk = __ldcg(out + k);
+                }
+                acc = __fma_rn(-val[q], xk, acc);
+            }
+            if (!FWD) acc = __ddiv_rn(acc, diag[i]);
+            ys[t] = acc;
+            out[i] = acc;
+            __threadfence();
+            ready[t] = 1;
+            st_release_u32(&flags[i], flag_val);
+        }
+    }
+}
+
+}  // namespace mfk

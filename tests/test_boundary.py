@@ -52,7 +52,7 @@ def test_status_strings_and_defaults(mf):
     assert (o.tol, o.max_iter, o.mode, o.switch_eps, o.range_guard, o.sticky) == (1e-10, 1000, 2, -1.0, 1, 0)
     c = mf.ConvertOpts()
     L.mf_default_convert_opts(C.byref(c))
-    assert (c.classify, c.loss_tol, c.grid_ctas, c.block_threads) == (1, 1e-15, 0, 0)
+    assert (c.classify, c.loss_tol, c.grid_ctas, c.block_threads, c.layout) == (1, 1e-15, 0, 0, 0)
     assert L.mf_abi_version() == 1
 
 
@@ -62,7 +62,7 @@ def test_struct_sizes_match_header(mf, tmp_path):
     prog.write_text('#include <stdio.h>\n#include <stddef.h>\n#include "mf.h"\nint main(){'
                     'printf("%zu %zu %zu %zu %zu\\n", sizeof(mf_convert_opts), sizeof(mf_tile_info),'
                     'sizeof(mf_tile_export), sizeof(mf_solve_opts), sizeof(mf_solve_info));'
-                    'printf("%zu %zu\\n", offsetof(mf_solve_opts, collect_stats), offsetof(mf_tile_info, convert_launches));'
+                    'printf("%zu %zu\\n", offsetof(mf_solve_opts, collect_stats), offsetof(mf_tile_info, layout));'
                     'return 0;}')
     exe = tmp_path / "sz"
     assert os.system(f"gcc -I{ROOT}/include -o {exe} {prog}") == 0
@@ -70,7 +70,7 @@ def test_struct_sizes_match_header(mf, tmp_path):
     assert [int(s) for s in sizes[:5]] == [C.sizeof(mf.ConvertOpts), C.sizeof(mf.TileInfo), C.sizeof(mf.TileExport),
                                           C.sizeof(mf.SolveOpts), C.sizeof(mf.SolveInfo)]
     assert int(sizes[5]) == mf.SolveOpts.collect_stats.offset
-    assert int(sizes[6]) == mf.TileInfo.convert_launches.offset
+    assert int(sizes[6]) == mf.TileInfo.layout.offset
 
 
 def test_compute_calls_fail_loudly_without_gpu(mf):

@@ -126,10 +126,12 @@ def test_convert_full_size_bit_exact(mf, orc, name):
 # ------------------------------------------------------------------------------ SpMV / levels / dot
 @pytest.mark.parametrize("name,make", CONVERT_CASES[:8], ids=[c[0] for c in CONVERT_CASES[:8]])
 @pytest.mark.parametrize("range_guard", [True, False])
-def test_spmv_bit_exact_with_levels(mf, orc, name, make, range_guard):
+@pytest.mark.parametrize("layout", [1, 2])
+def test_spmv_bit_exact_with_levels(mf, orc, name, make, range_guard, layout):
     A = make()
     T = oracle_tiles(orc, A)
-    G = mf.TileMatrix.from_host_csr(A)
+    G = mf.TileMatrix.from_host_csr(A, layout=layout)
+    assert G.info()["layout"] == layout
     rng = np.random.default_rng(7)
     x = rng.standard_normal(A.n_cols) * np.exp2(rng.integers(-30, 5, A.n_cols))
     for trial in range(3):
@@ -165,9 +167,9 @@ def test_dot_tree_bit_exact(mf, orc, G, B):
 
 
 # ------------------------------------------------------------------------------ solves
-def run_pair(mf, orc, A, solver, mode, classify=True, G=0, B=0, max_iter=1000, x0=None, b=None, **kw):
+def run_pair(mf, orc, A, solver, mode, classify=True, G=0, B=0, max_iter=1000, x0=None, b=None, layout=0, **kw):
     b = W.rhs_ones(A) if b is None else b
-    Gm = mf.TileMatrix.from_host_csr(A, classify=classify, grid_ctas=G, block_threads=B)
+    Gm = mf.TileMatrix.from_host_csr(A, classify=classify, grid_ctas=G, block_threads=B, layout=layout)
     g, bb, R = Gm.plan()
     plan = orc.Plan(g, bb, R)
     T = oracle_tiles(orc, A, classify)
@@ -180,7 +182,7 @@ def run_pair(mf, orc, A, solver, mode, classify=True, G=0, B=0, max_iter=1000, x
 
 
 SOLVE_CASES = [
-    # name, matrix, solver, mode, classify, G, B
+    # name, matrix, solver, mode, classify, G, B  (layout: auto, plus the forced variants below)
     ("C1-fp64", lambda: W.make("C1"), "cg", 0, False, 0, 0),
     ("C1-dyn-G1", lambda: W.make("C1"), "cg", 2, True, 1, 1024),
     ("C1-dyn-G4", lambda: W.make("C1"), "cg", 2, True, 4, 256),
@@ -196,10 +198,11 @@ SOLVE_CASES = [
 ]
 
 
+@pytest.mark.parametrize("layout", [0, 1, 2])
 @pytest.mark.parametrize("name,make,solver,mode,classify,G,B", SOLVE_CASES, ids=[c[0] for c in SOLVE_CASES])
-def test_solve_kernel_order_parity(mf, orc, name, make, solver, mode, classify, G, B):
+def test_solve_kernel_order_parity(mf, orc, name, make, solver, mode, classify, G, B, layout):
     A = make()
-    ro, rg, _ = run_pair(mf, orc, A, solver, mode, classify, G, B, max_iter=3000)
+    ro, rg, _ = run_pair(mf, orc, A, solver, mode, classify, G, B, max_iter=3000, layout=layout)
     assert rg.status == ro["status"] == 0
     assert rg.converged and ro["converged"]
     assert rg.iterations == ro["iterations"]
@@ -272,3 +275,66 @@ def test_full_size_C3_prefix_and_convergence(mf, orc):
     assert full.converged
     tr = orc.true_relres(A.rowptr, A.colidx, A.vals, b, full.x.cpu().numpy())
     assert tr < 1e-9
+
+
+# ------------------------------------------------------------------------------ ILU(0)
+@pytest.mark.parametrize("name,make", [("C4spd-12", lambda: W.make("C4spd", 1 << 12)),
+                                       ("C4ind-12", lambda: W.make("C4ind", 1 << 12)),
+                                       ("C2-16", lambda: W.make("C2", 16)),
+                                       ("C3-40", lambda: W.make("C3", 40))])
+def test_ilu0_apply_bit_exact(mf, orc, name, make):
+    """ILU(0) of the stored values (reading R20): z = U^-1 L^-1 r bit-identical to the oracle."""
+    A = make()
+    T = oracle_tiles(orc, A)
+    rp, ci, sv = T.stored_csr()
+    M = orc.ILU0(rp, ci, sv)
+    G = mf.TileMatrix.from_host_csr(A)
+    P = mf.Precond(G)
+    rng = np.random.default_rng(5)
+    for _ in range(3):
+        r = rng.standard_normal(A.n_rows)
+        assert np.array_equal(P.apply(dev(r)).cpu().numpy(), M.apply(r))
+
+
+def test_ilu0_zero_pivot_reported(mf):
+    A = W.CSR(2, 2, np.array([0, 2, 4], np.int64), np.array([0, 1, 0, 1], np.int32), np.array([0.0, 1, 1, 2]))
+    G = mf.TileMatrix.from_host_csr(A)
+    with pytest.raises(mf.MFError) as e:
+        mf.Precond(G)
+    assert e.value.status == 8
+
+
+PRE_CASES = [
+    ("C4spd-12-dyn", lambda: W.make("C4spd", 1 << 12), "cg", 2, 6, 256),
+    ("C4spd-13-static", lambda: W.make("C4spd", 1 << 13), "cg", 1, 0, 0),
+    ("C4ind-12-dyn", lambda: W.make("C4ind", 1 << 12), "bicgstab", 2, 5, 128),
+    ("C4ind-13-static", lambda: W.make("C4ind", 1 << 13), "bicgstab", 1, 0, 0),
+    ("C2-16-pcg", lambda: W.make("C2", 16), "cg", 2, 4, 512),
+    ("C3-48-pbicg", lambda: W.make("C3", 48), "bicgstab", 2, 3, 256),
+]
+
+
+@pytest.mark.parametrize("name,make,solver,mode,G,B", PRE_CASES, ids=[c[0] for c in PRE_CASES])
+def test_preconditioned_solve_parity(mf, orc, name, make, solver, mode, G, B):
+    """PCG / right-preconditioned PBiCGSTAB with ILU(0) in the persistent kernel:
+    histories, x and level counts bit-identical to the oracle in kernel-order mode."""
+    A = make()
+    b = W.rhs_ones(A)
+    Gm = mf.TileMatrix.from_host_csr(A, grid_ctas=G, block_threads=B)
+    g, bb, R = Gm.plan()
+    T = oracle_tiles(orc, A)
+    rp, ci, sv = T.stored_csr()
+    M = orc.ILU0(rp, ci, sv)
+    P = mf.Precond(Gm)
+    ofn = orc.cg if solver == "cg" else orc.bicgstab
+    gfn = mf.cg_solve if solver == "cg" else mf.bicgstab_solve
+    ro = ofn(T, b, M=M, mode=mode, plan=orc.Plan(g, bb, R), max_iter=500)
+    rg = gfn(Gm, dev(b), M=P, mode=mode, max_iter=500, level_counts=True)
+    assert ro["converged"] and rg.converged and rg.iterations == ro["iterations"]
+    assert np.array_equal(rg.history, ro["history"])
+    assert np.array_equal(rg.x.cpu().numpy(), ro["x"])
+    if mode == 2:
+        assert np.array_equal(rg.level_counts, ro["level_counts"])
+    # second solve on the same preconditioner (flag epochs advance, counters reset)
+    rg2 = gfn(Gm, dev(b), M=P, mode=mode, max_iter=500)
+    assert np.array_equal(rg2.x.cpu().numpy(), ro["x"])
