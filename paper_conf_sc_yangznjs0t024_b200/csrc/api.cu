@@ -27,6 +27,20 @@ void* dev_alloc(size_t bytes, cudaStream_t s) {
         std::lock_guard<std::mutex> lk(g_alloc_mu);
         if (g_alloc) return g_alloc(bytes, (mf_stream)s, g_alloc_ctx);
     }
+    // stream-ordered allocator: keep freed blocks in the device's default pool across
+    // synchronisations (release threshold = max) so repeated conversions / solves reuse them
+    // instead of re-mapping physical memory each time
+    static thread_local int pool_dev = -1;
+    int dev = 0;
+    if (cudaGetDevice(&dev) == cudaSuccess && dev != pool_dev) {
+        cudaMemPool_t pool;
+        if (cudaDeviceGetDefaultMemPool(&pool, dev) == cudaSuccess) {
+            unsigned long long thr = ~0ull;
+            cudaMemPoolSetAttribute(pool, cudaMemPoolAttrReleaseThreshold, &thr);
+        }
+        cudaGetLastError();
+        pool_dev = dev;
+    }
     void* p = nullptr;
     if (cudaMallocAsync(&p, bytes, s) != cudaSuccess) {
         cudaGetLastError();

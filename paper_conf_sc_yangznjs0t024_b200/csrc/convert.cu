@@ -12,6 +12,7 @@
 #include <algorithm>
 #include <vector>
 
+#include "kernels.cuh"
 #include "mf_internal.cuh"
 
 namespace mf {
@@ -19,7 +20,8 @@ namespace {
 
 constexpr int CNT_TILES = 0, CNT_ROWS = 1, CNT_WIDTH = 2, CNT_NNZP = 3 /*..6*/, CNT_TILEP = 7 /*..10*/;
 constexpr int CNT_WTS = 11;   // tile-synchronous width: sum over tiles of the max entries per row
-constexpr int NCNT = 12;
+constexpr int CNT_VB = 12;    // tile-synchronous value bytes: sum over tiles of width * 16 * size(TilePrec)
+constexpr int NCNT = 13;
 constexpr int THREADS = 256;
 
 __device__ __forceinline__ unsigned hw_mask() { return (threadIdx.x & 16) ? 0xFFFF0000u : 0x0000FFFFu; }
@@ -95,7 +97,7 @@ struct Out {  // FILL-pass destinations (all device)
     int64_t *TileNnz, *Nonrow, *ValOff, *TileRowPtr;
     uint8_t *RowIndex, *CsrRowptr, *CsrColidx;
     double* Val64; float* Val32; uint16_t* Val16; uint8_t* Val8;
-    uint32_t* tile_info; uint16_t* sidx; uint8_t* sslot; uint32_t* colw; int ts;
+    uint32_t* tile_info; uint16_t* sidx; uint8_t* sslot; uint2* crec; int ts; uint8_t* vstream;
     double* p64; float* p32; __half* p16; uint8_t* p8;
     const int64_t* off;   // [NCNT][ntr+1] exclusive scans of the counts
     int64_t ntr;
@@ -121,12 +123,13 @@ __global__ void __launch_bounds__(THREADS) tile_row_kernel(int64_t n_rows, int64
 
     int64_t j = 0, nz_run = 0, ri_run = 0, colbase = 0;
     int64_t pnnz[4] = {0, 0, 0, 0}, ptile[4] = {0, 0, 0, 0};
-    int64_t tile0 = 0, row0 = 0, nnz0 = 0, slot0 = 0, voff[4] = {0, 0, 0, 0};
+    int64_t tile0 = 0, row0 = 0, nnz0 = 0, slot0 = 0, voff[4] = {0, 0, 0, 0}, vb0 = 0, vb_run = 0;
     if (FILL) {
         const int64_t S = ntr + 1;
         tile0 = o.off[CNT_TILES * S + TR];
         row0 = o.off[CNT_ROWS * S + TR];
         slot0 = o.off[(o.ts ? CNT_WTS : CNT_WIDTH) * S + TR];
+        vb0 = o.off[CNT_VB * S + TR];
         for (int q = 0; q < 4; ++q) voff[q] = o.off[(CNT_NNZP + q) * S + TR];
         nnz0 = rowptr[TR * TS];
         if (lane == 0) o.TileRowPtr[TR] = tile0;
@@ -191,8 +194,19 @@ __global__ void __launch_bounds__(THREADS) tile_row_kernel(int64_t n_rows, int64
                     // colbase + (k - ptr); value planes RNE_q(stored) for q at or below TilePrec
                     const int64_t pos = o.ts ? (slot0 + colbase + (k - ptr)) * TS + lane
                                              : (slot0 + (k - rstart)) * TS + lane;
-                    if (o.ts) o.sslot[pos] = (uint8_t)lc;
-                    else o.sidx[pos] = (uint16_t)((j << 4) | lc);
+                    if (o.ts) {
+                        o.sslot[pos] = (uint8_t)lc;
+                        // value stream: column (colbase + k - ptr) of the tile row, 16 * size(TilePrec) bytes
+                        const int64_t vb = vb0 + vb_run + ((k - ptr) * 16 + lane) * (8 >> best);
+                        switch (best) {
+                        case 0: *reinterpret_cast<double*>(o.vstream + vb) = sv; break;
+                        case 1: *reinterpret_cast<float*>(o.vstream + vb) = (float)sv; break;
+                        case 2: *reinterpret_cast<__half*>(o.vstream + vb) = mfk::to_f16(sv); break;
+                        default: o.vstream[vb] = mfk::to_e4m3(sv); break;
+                        }
+                    } else {
+                        o.sidx[pos] = (uint16_t)((j << 4) | lc);
+                    }
                     if (best <= 0 && o.p64) o.p64[pos] = sv;
                     if (best <= 1 && o.p32) o.p32[pos] = mfk::to_f32(sv);
                     if (best <= 2 && o.p16) o.p16[pos] = mfk::to_f16(sv);
@@ -200,11 +214,14 @@ __global__ void __launch_bounds__(THREADS) tile_row_kernel(int64_t n_rows, int64
                 }
             }
         }
+        // static column record: word, value offset within the tile row (stage_kernel rebases it)
         if (FILL && o.ts && lane < w_j)
-            o.colw[slot0 + colbase + lane] = ((uint32_t)tc << 4) | ((uint32_t)floor_t << 2) | (uint32_t)best;
+            o.crec[slot0 + colbase + lane] = make_uint2(((uint32_t)tc << 4) | ((uint32_t)floor_t << 2) | (uint32_t)best,
+                                                        (uint32_t)(vb_run + (int64_t)lane * 16 * (8 >> best)));
         if (mine) { ptr = q; cur = ptr < rend ? (colidx[ptr] >> 4) : INT32_MAX; }
         ++j;
         colbase += w_j;
+        vb_run += (int64_t)w_j * 16 * (8 >> best);
         nz_run += tile_nz;
         ri_run += rows_in_tile;
         pnnz[best] += tile_nz;
@@ -220,6 +237,7 @@ __global__ void __launch_bounds__(THREADS) tile_row_kernel(int64_t n_rows, int64
         cnt[CNT_ROWS * ntr + TR] = ri_run;
         cnt[CNT_WIDTH * ntr + TR] = width;
         cnt[CNT_WTS * ntr + TR] = colbase;
+        cnt[CNT_VB * ntr + TR] = vb_run;
         for (int q = 0; q < 4; ++q) {
             cnt[(CNT_NNZP + q) * ntr + TR] = pnnz[q];
             cnt[(CNT_TILEP + q) * ntr + TR] = ptile[q];
@@ -356,14 +374,159 @@ __global__ void deps_kernel(const int32_t* __restrict__ plan_tr, int G, const in
     }
 }
 
+// max over tile rows of the tile-synchronous width and value bytes (stage-capacity check)
+__global__ void max2_kernel(const int64_t* __restrict__ a, const int64_t* __restrict__ b, int64_t n, unsigned long long* out) {
+    unsigned long long ma = 0, mb = 0;
+    for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x) {
+        ma = max(ma, (unsigned long long)a[i]);
+        mb = max(mb, (unsigned long long)b[i]);
+    }
+    for (int o = 16; o >= 1; o >>= 1) {
+        ma = max(ma, __shfl_xor_sync(0xffffffffu, ma, o));
+        mb = max(mb, __shfl_xor_sync(0xffffffffu, mb, o));
+    }
+    if ((threadIdx.x & 31) == 0) { atomicMax(&out[0], ma); atomicMax(&out[1], mb); }
+}
+
+// Stages of the TMA pipeline (kernels.cuh): one warp per CTA of the plan walks its tile rows and
+// cuts them greedily into stages within the caps (tile rows, slice columns, value bytes), each
+// a whole number of H-row groups when one fits, so that every half-warp gets the same number of
+// tile rows per stage.  COUNT pass: stages per CTA; FILL pass: the records.
+template <bool FILL>
+__global__ void stage_kernel(const int32_t* __restrict__ plan_tr, int G, int H, const int64_t* __restrict__ tr_slot,
+                             const int64_t* __restrict__ tr_vb, int32_t* nst, const int32_t* __restrict__ sptr,
+                             mfk::PipeStage* stg) {
+    const int g = blockIdx.x;
+    const int lane = threadIdx.x & 31;
+    if (g >= G) return;
+    const int64_t tr0 = plan_tr[g], tr1 = plan_tr[g + 1];
+    const int64_t base = FILL ? sptr[g] : 0;
+    int64_t S = tr0;
+    int32_t k = 0;
+    while (S < tr1) {
+        const int64_t c0 = tr_slot[S], v0 = tr_vb[S];
+        const int64_t lim = min(S + (int64_t)mfk::PIPE_KCAP, tr1);
+        int64_t emax = S;
+        for (int64_t e0 = S + 1; e0 <= lim; e0 += 32) {
+            const int64_t E = e0 + lane;
+            const bool fit = E <= lim && tr_slot[E] - c0 <= mfk::PIPE_CCAP && tr_vb[E] - v0 <= mfk::PIPE_VCAP;
+            const int nfit = __popc(__ballot_sync(0xffffffffu, fit));     // fits are a prefix (monotone)
+            if (nfit > 0) emax = e0 + nfit - 1;
+            if (nfit < 32) break;
+        }
+        if (emax == S) emax = S + 1;          // oversize tile row: excluded by the host's capacity check
+        const int64_t grp = tr0 + ((emax - tr0) / H) * H;
+        const int64_t E = grp > S ? grp : emax;
+        if (FILL && lane == 0) {
+            mfk::PipeStage st{};
+            st.col0 = c0; st.col1 = tr_slot[E];
+            st.tr0 = (int32_t)S; st.tr1 = (int32_t)E;
+            stg[base + k] = st;
+        }
+        ++k;
+        S = E;
+    }
+    if (!FILL && lane == 0) nst[g] = k;
+}
+
+// Blob of each stage (layout in kernels.cuh): its byte size (from the record), then, after an
+// exclusive scan of the sizes, its contents: headers, column words, local columns, the group
+// permutation and the values grouped by TilePrec.  One block of PIPE_CCAP threads per stage:
+// thread c owns column c of the stage.
+__device__ __forceinline__ void blob_layout(int K, int64_t nc, int64_t nv, int* off_cw, int* off_ss, int* off_dst, int* off_val, int* bytes) {
+    *off_cw = mfk::pipe_r16((K + 1) * 4);
+    *off_ss = *off_cw + mfk::pipe_r16((int)nc * 4);
+    *off_dst = *off_ss + (int)nc * 16;
+    *off_val = *off_dst + mfk::pipe_r16((int)nc * 2);
+    *bytes = *off_val + (int)nv;
+}
+__global__ void blob_size_kernel(const mfk::PipeStage* __restrict__ stg, int64_t n, const int64_t* __restrict__ tr_vb, int64_t* sz) {
+    const int64_t s = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
+    if (s >= n) return;
+    const mfk::PipeStage st = stg[s];
+    int a, b, c, d, bytes;
+    blob_layout(st.tr1 - st.tr0, st.col1 - st.col0, tr_vb[st.tr1] - tr_vb[st.tr0], &a, &b, &c, &d, &bytes);
+    sz[s] = bytes;
+}
+__global__ void __launch_bounds__(mfk::PIPE_CCAP) blob_fill_kernel(mfk::PipeStage* stg, const int64_t* __restrict__ boff,
+                                                                     const int64_t* __restrict__ tr_slot, const int64_t* __restrict__ tr_vb,
+                                                                     const uint2* __restrict__ crec, const uint8_t* __restrict__ sslot,
+                                                                     const uint8_t* __restrict__ vstream, uint8_t* blob) {
+    __shared__ int32_t hdr[mfk::PIPE_KCAP + 1];
+    __shared__ unsigned long long wsum[mfk::PIPE_CCAP / 32];
+    __shared__ int gtot[4];
+    const int64_t sidx = blockIdx.x;
+    mfk::PipeStage st = stg[sidx];
+    const int K = st.tr1 - st.tr0, c = threadIdx.x;
+    const int nc = (int)(st.col1 - st.col0);
+    const int64_t nv = tr_vb[st.tr1] - tr_vb[st.tr0];
+    int off_cw, off_ss, off_dst, off_val, bytes;
+    blob_layout(K, nc, nv, &off_cw, &off_ss, &off_dst, &off_val, &bytes);
+    uint8_t* b = blob + boff[sidx];
+    for (int k = c; k <= K; k += blockDim.x) {
+        hdr[k] = (int32_t)(tr_slot[st.tr0 + k] - st.col0);
+        reinterpret_cast<int32_t*>(b)[k] = hdr[k];
+    }
+    uint2 rc = make_uint2(0u, 0u);
+    int q = 0;
+    if (c < nc) {
+        rc = crec[st.col0 + c];
+        q = (int)(rc.x & 3u);
+        reinterpret_cast<uint32_t*>(b + off_cw)[c] = rc.x;
+        reinterpret_cast<uint4*>(b + off_ss)[c] = reinterpret_cast<const uint4*>(sslot)[st.col0 + c];
+    }
+    // rank of column c within its precision group: block exclusive scan of 4 packed 16-bit counters
+    const unsigned long long one = c < nc ? 1ull << (16 * q) : 0ull;
+    unsigned long long incl = one;
+    const int lane = c & 31, w = c >> 5;
+    for (int o = 1; o < 32; o <<= 1) { const unsigned long long u = __shfl_up_sync(0xffffffffu, incl, o); if (lane >= o) incl += u; }
+    if (lane == 31) wsum[w] = incl;
+    __syncthreads();
+    unsigned long long wpre = 0;
+    for (int k = 0; k < w; ++k) wpre += wsum[k];
+    const unsigned long long excl = wpre + incl - one;
+    if (c == (int)blockDim.x - 1) {
+        const unsigned long long tot = wpre + incl;
+        for (int k = 0; k < 4; ++k) gtot[k] = (int)((tot >> (16 * k)) & 0xFFFFull);
+    }
+    __syncthreads();
+    int gbase[4], goff[4];
+    {
+        int cols = 0, off = off_val;
+        for (int k = 0; k < 4; ++k) { gbase[k] = cols; goff[k] = off; cols += gtot[k]; off += gtot[k] * 16 * (8 >> k); }
+    }
+    if (c < nc) {
+        const int rank = (int)((excl >> (16 * q)) & 0xFFFFull);
+        reinterpret_cast<uint16_t*>(b + off_dst)[gbase[q] + rank] = (uint16_t)c;
+        // tile row of column c, then its values (16 x size(TilePrec) bytes) into its group
+        int lo = 0, hi = K - 1;
+        while (lo < hi) { const int mid = (lo + hi + 1) / 2; if (hdr[mid] <= c) lo = mid; else hi = mid - 1; }
+        const int64_t src = tr_vb[st.tr0 + lo] + rc.y;
+        const int n16 = 8 >> q;                 // 16-byte chunks per column
+        const uint4* sp = reinterpret_cast<const uint4*>(vstream + src);
+        uint4* dp = reinterpret_cast<uint4*>(b + goff[q] + (int64_t)rank * 16 * (8 >> q));
+        for (int k = 0; k < n16; ++k) dp[k] = sp[k];
+    }
+    if (c == 0) {
+        stg[sidx].boff = boff[sidx];
+        stg[sidx].bbytes = bytes;
+        stg[sidx].off_cw = off_cw;
+        stg[sidx].off_ss = off_ss;
+        stg[sidx].off_dst = off_dst;
+        stg[sidx].off_val = off_val;
+        for (int k = 0; k < 4; ++k) { stg[sidx].gcnt[k] = gtot[k]; stg[sidx].goff[k] = goff[k]; }
+    }
+}
+
 }  // namespace
 
 void destroy_tiles(TileMatrix* A) {
     cudaStream_t s = A->owner_stream;
     void* ptrs[] = {A->TileRowidx, A->TileColidx, A->TilePrec, A->Floor, A->TileNnz, A->Nonrow, A->ValOff,
                     A->TileRowPtr, A->RowIndex, A->CsrRowptr, A->CsrColidx, A->Val64, A->Val32, A->Val16,
-                    A->Val8, A->tr_slot, A->tile_info, A->sidx, A->sslot, A->colw, A->plane64, A->plane32, A->plane16,
-                    A->plane8, A->plan_tr, A->dep_lo, A->dep_hi, A->seg_lo, A->seg_hi};
+                    A->Val8, A->tr_slot, A->tile_info, A->sidx, A->sslot, A->crec, A->plane64, A->plane32, A->plane16,
+                    A->plane8, A->plan_tr, A->dep_lo, A->dep_hi, A->seg_lo, A->seg_hi, A->tr_vb, A->vstream, A->stg,
+                    A->stg_ptr, A->blob};
     for (void* p : ptrs) if (p) dev_free(p, s);
     delete[] A->plan_rows_host;
     *A = TileMatrix();
@@ -424,11 +587,25 @@ mf_status convert_csr(int64_t n_rows, int64_t n_cols, int64_t nnz, const int64_t
     }
     A->tilenum = tot[CNT_TILES];
     A->rownum = tot[CNT_ROWS];
-    // kernel layout: tile-synchronous slices (uniform tile per slice column) unless they cost
-    // more than 30% extra slots over the compact (row-packed) slices
+    // kernel layout: tile-synchronous slices (uniform tile per slice column, streamed by the TMA
+    // pipeline) unless they cost more than 60% extra slots over the compact (row-packed) slices,
+    // or one tile row exceeds a pipeline stage
+    unsigned long long mx[4] = {0, 0, 0, 0};   // max over tile rows: TS width, TS value bytes, tiles, compact width
+    if (ntr > 0) {
+        unsigned long long* dmx = nullptr;
+        MF_TRY(alloc(&dmx, 4, s));
+        MF_CUDA(cudaMemsetAsync(dmx, 0, 4 * sizeof(unsigned long long), s));
+        const unsigned mb = (unsigned)std::min<int64_t>((ntr + 255) / 256, 1184);
+        max2_kernel<<<mb, 256, 0, s>>>(cnt + CNT_WTS * ntr, cnt + CNT_VB * ntr, ntr, dmx);
+        max2_kernel<<<mb, 256, 0, s>>>(cnt + CNT_TILES * ntr, cnt + CNT_WIDTH * ntr, ntr, dmx + 2);
+        MF_CUDA(cudaMemcpyAsync(mx, dmx, sizeof(mx), cudaMemcpyDeviceToHost, s));
+        MF_CUDA(cudaStreamSynchronize(s));
+        dev_free(dmx, s);
+    }
+    const bool ts_fits = mx[0] <= (unsigned long long)mfk::PIPE_CCAP && mx[1] <= (unsigned long long)mfk::PIPE_VCAP;
     if (o.layout == 1) A->ts = 0;
-    else if (o.layout == 2) A->ts = 1;
-    else A->ts = (double)tot[CNT_WTS] <= 1.3 * (double)tot[CNT_WIDTH] ? 1 : 0;
+    else if (o.layout == 2) A->ts = ts_fits ? 1 : 0;
+    else A->ts = ts_fits && (double)tot[CNT_WTS] <= 1.6 * (double)tot[CNT_WIDTH] ? 1 : 0;
     A->slots = A->ts ? tot[CNT_WTS] : tot[CNT_WIDTH];
     for (int q = 0; q < 4; ++q) { A->nval[q] = tot[CNT_NNZP + q]; A->tiles_per_prec[q] = tot[CNT_TILEP + q]; }
 
@@ -443,35 +620,45 @@ mf_status convert_csr(int64_t n_rows, int64_t n_cols, int64_t nnz, const int64_t
     MF_TRY(alloc(&A->Val64, A->nval[0], s)); MF_TRY(alloc(&A->Val32, A->nval[1], s));
     MF_TRY(alloc(&A->Val16, A->nval[2], s)); MF_TRY(alloc(&A->Val8, A->nval[3], s));
     MF_TRY(alloc(&A->tile_info, nt, s));
+    A->vbytes = A->ts ? tot[CNT_VB] : 0;
     if (A->ts) {
-        MF_TRY(alloc(&A->sslot, nslot, s));
-        MF_TRY(alloc(&A->colw, A->slots, s));
+        // padded so that the pipeline's 16-byte aligned bulk copies stay inside the arrays
+        MF_TRY(alloc(&A->sslot, nslot + 16, s));
+        MF_TRY(alloc(&A->crec, A->slots + 8, s));
+        MF_TRY(alloc(&A->vstream, A->vbytes + 64, s));
+        MF_TRY(alloc(&A->tr_vb, ntr + 4, s));
+        MF_CUDA(cudaMemsetAsync(A->sslot, 0, nslot + 16, s));
+        MF_CUDA(cudaMemsetAsync(A->crec, 0, (A->slots + 8) * sizeof(uint2), s));
+        MF_CUDA(cudaMemsetAsync(A->vstream, 0, A->vbytes + 64, s));
+        MF_CUDA(cudaMemsetAsync(A->tr_vb, 0, (ntr + 4) * sizeof(int64_t), s));
+        MF_CUDA(cudaMemcpyAsync(A->tr_vb, off + CNT_VB * S, (ntr + 1) * sizeof(int64_t), cudaMemcpyDeviceToDevice, s));
     } else {
         MF_TRY(alloc(&A->sidx, nslot, s));
     }
-    // value planes: plane q exists when some tile can compute at q (TilePrec <= q)
+    // value planes (compact layout): plane q exists when some tile can compute at q (TilePrec <= q)
     bool need[4] = {false, false, false, false};
-    for (int q = 0; q < 4; ++q)
-        for (int p = 0; p <= q; ++p) if (A->tiles_per_prec[p] > 0) need[q] = true;
+    if (!A->ts)
+        for (int q = 0; q < 4; ++q)
+            for (int p = 0; p <= q; ++p) if (A->tiles_per_prec[p] > 0) need[q] = true;
     // planes padded to whole 8-byte words: the SpMV fetches the aligned 8-byte word around a value
     if (need[0]) MF_TRY(alloc(&A->plane64, nslot + 1, s));
     if (need[1]) MF_TRY(alloc(&A->plane32, nslot + 2, s));
     if (need[2]) MF_TRY(alloc(&A->plane16, nslot + 4, s));
     if (need[3]) MF_TRY(alloc(&A->plane8, nslot + 8, s));
     if (nslot && A->sidx) MF_CUDA(cudaMemsetAsync(A->sidx, 0xFF, nslot * sizeof(uint16_t), s));
-    if (nslot && A->sslot) MF_CUDA(cudaMemsetAsync(A->sslot, 0xFF, nslot, s));
     if (nt == 0) {
         MF_CUDA(cudaMemsetAsync(A->TileNnz, 0, sizeof(int64_t), s));
         MF_CUDA(cudaMemsetAsync(A->Nonrow, 0, sizeof(int64_t), s));
     }
-    MF_TRY(alloc(&A->tr_slot, ntr + 1, s));
+    MF_TRY(alloc(&A->tr_slot, ntr + 4, s));
+    MF_CUDA(cudaMemsetAsync(A->tr_slot, 0, (ntr + 4) * sizeof(int64_t), s));
     MF_CUDA(cudaMemcpyAsync(A->tr_slot, off + (A->ts ? CNT_WTS : CNT_WIDTH) * S, (ntr + 1) * sizeof(int64_t),
                             cudaMemcpyDeviceToDevice, s));
 
     // 4. FILL pass
     Out fo{A->TileRowidx, A->TileColidx, A->TilePrec, A->Floor, A->TileNnz, A->Nonrow, A->ValOff, A->TileRowPtr,
            A->RowIndex, A->CsrRowptr, A->CsrColidx, A->Val64, A->Val32, A->Val16, A->Val8, A->tile_info, A->sidx,
-           A->sslot, A->colw, A->ts, A->plane64, A->plane32, A->plane16, A->plane8, off, ntr};
+           A->sslot, A->crec, A->ts, A->vstream, A->plane64, A->plane32, A->plane16, A->plane8, off, ntr};
     if (ntr > 0) {
         tile_row_kernel<true><<<tblocks, THREADS, 0, s>>>(n_rows, ntr, rowptr, colidx, vals, o.classify, o.loss_tol,
                                                            cnt, d_err, fo);
@@ -479,17 +666,8 @@ mf_status convert_csr(int64_t n_rows, int64_t n_cols, int64_t nnz, const int64_t
     } else {
         MF_CUDA(cudaMemsetAsync(A->TileRowPtr, 0, sizeof(int64_t), s));
     }
-    // max tiles per tile row (host, from the counts)
-    {
-        std::vector<int64_t> hc(ntr);
-        if (ntr) MF_CUDA(cudaMemcpyAsync(hc.data(), cnt + CNT_TILES * ntr, ntr * sizeof(int64_t), cudaMemcpyDeviceToHost, s));
-        MF_CUDA(cudaStreamSynchronize(s));
-        A->max_nt = ntr ? *std::max_element(hc.begin(), hc.end()) : 0;
-        if (ntr) MF_CUDA(cudaMemcpyAsync(hc.data(), cnt + (A->ts ? CNT_WTS : CNT_WIDTH) * ntr, ntr * sizeof(int64_t),
-                                         cudaMemcpyDeviceToHost, s));
-        MF_CUDA(cudaStreamSynchronize(s));
-        A->max_w = ntr ? *std::max_element(hc.begin(), hc.end()) : 0;
-    }
+    A->max_nt = (int64_t)mx[2];
+    A->max_w = (int64_t)(A->ts ? mx[0] : mx[3]);
 
     // 5. launch plan
     int G = o.grid_ctas, B = o.block_threads;
@@ -515,6 +693,47 @@ mf_status convert_csr(int64_t n_rows, int64_t n_cols, int64_t nnz, const int64_t
     deps_kernel<<<G, 256, 0, s>>>(A->plan_tr, G, A->TileRowPtr, A->TileColidx, ntr, A->dep_lo, A->dep_hi, A->seg_lo,
                                   A->seg_hi);
     MF_CUDA(cudaGetLastError());
+    if (A->ts) {   // pipeline stages of every CTA (two passes: count, fill)
+        int32_t* nst = nullptr;
+        MF_TRY(alloc(&nst, G, s));
+        stage_kernel<false><<<G, 32, 0, s>>>(A->plan_tr, G, B / 16, A->tr_slot, A->tr_vb, nst, nullptr, nullptr);
+        MF_CUDA(cudaGetLastError());
+        std::vector<int32_t> nst_h(G), sp_h(G + 1);
+        MF_CUDA(cudaMemcpyAsync(nst_h.data(), nst, G * sizeof(int32_t), cudaMemcpyDeviceToHost, s));
+        MF_CUDA(cudaStreamSynchronize(s));
+        sp_h[0] = 0;
+        for (int g = 0; g < G; ++g) sp_h[g + 1] = sp_h[g] + nst_h[g];
+        A->nstg = sp_h[G];
+        MF_TRY(alloc(&A->stg_ptr, G + 1, s));
+        MF_CUDA(cudaMemcpyAsync(A->stg_ptr, sp_h.data(), (G + 1) * sizeof(int32_t), cudaMemcpyHostToDevice, s));
+        mfk::PipeStage* stg = nullptr;
+        MF_TRY(alloc(&stg, std::max<int64_t>(A->nstg, 1), s));
+        A->stg = stg;
+        stage_kernel<true><<<G, 32, 0, s>>>(A->plan_tr, G, B / 16, A->tr_slot, A->tr_vb, nullptr, A->stg_ptr, stg);
+        MF_CUDA(cudaGetLastError());
+        // blobs: sizes -> offsets -> copies; the per-column source arrays are then released
+        if (A->nstg > 0) {
+            int64_t *bsz = nullptr, *boff = nullptr, *btmp = nullptr;
+            MF_TRY(alloc(&bsz, A->nstg, s));
+            MF_TRY(alloc(&boff, A->nstg + 1, s));
+            MF_TRY(alloc(&btmp, A->nstg / 2048 + 2, s));
+            blob_size_kernel<<<(unsigned)((A->nstg + 255) / 256), 256, 0, s>>>(stg, A->nstg, A->tr_vb, bsz);
+            MF_TRY(scan_excl(bsz, A->nstg, boff, btmp, s));
+            MF_CUDA(cudaMemcpyAsync(&A->blob_bytes, boff + A->nstg, sizeof(int64_t), cudaMemcpyDeviceToHost, s));
+            MF_CUDA(cudaStreamSynchronize(s));
+            MF_TRY(alloc(&A->blob, A->blob_bytes + 64, s));
+            blob_fill_kernel<<<(unsigned)A->nstg, mfk::PIPE_CCAP, 0, s>>>(stg, boff, A->tr_slot, A->tr_vb, A->crec, A->sslot,
+                                                                         A->vstream, A->blob);
+            MF_CUDA(cudaGetLastError());
+            dev_free(bsz, s); dev_free(boff, s); dev_free(btmp, s);
+        }
+        MF_CUDA(cudaStreamSynchronize(s));   // sp_h (pageable) consumed
+        dev_free(nst, s);
+        dev_free(A->sslot, s); A->sslot = nullptr;
+        dev_free(A->crec, s); A->crec = nullptr;
+        dev_free(A->vstream, s); A->vstream = nullptr;
+        dev_free(A->tr_vb, s); A->tr_vb = nullptr;
+    }
     std::vector<int32_t> ptr_h(G + 1);
     MF_CUDA(cudaMemcpyAsync(ptr_h.data(), A->plan_tr, (G + 1) * sizeof(int32_t), cudaMemcpyDeviceToHost, s));
     MF_CUDA(cudaEventRecord(e1, s));
@@ -532,7 +751,8 @@ mf_status convert_csr(int64_t n_rows, int64_t n_cols, int64_t nnz, const int64_t
     A->convert_launches = (n_rows > 0 ? 1 : 0) + (ntr > 0 ? 2 + 1 : 0) + (NCNT + 1) * (ntr > 0 ? 3 : 0) + 2;
     A->canonical_bytes = nt * (4 + 4 + 1 + 1 + 8 + 8 + 8) + 16 + (ntr + 1) * 8 + A->rownum * 2 + nnz +
                          A->nval[0] * 8 + A->nval[1] * 4 + A->nval[2] * 2 + A->nval[3];
-    A->kernel_bytes = (A->ts ? nslot + A->slots * 4 : nslot * 2) + (A->plane64 ? nslot * 8 : 0) + (A->plane32 ? nslot * 4 : 0) +
+    A->kernel_bytes = (A->ts ? A->blob_bytes + A->nstg * (int64_t)sizeof(mfk::PipeStage) : nslot * 2) +
+                      (A->plane64 ? nslot * 8 : 0) + (A->plane32 ? nslot * 4 : 0) +
                       (A->plane16 ? nslot * 2 : 0) + (A->plane8 ? nslot : 0) + nt * 4 + (ntr + 1) * 8;
     return MF_OK;
 }

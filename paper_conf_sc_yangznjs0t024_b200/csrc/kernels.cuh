@@ -23,8 +23,10 @@ struct Mat {
     const int64_t* __restrict__ tr_tile;
     const uint32_t* __restrict__ tile_info;
     const uint16_t* __restrict__ sidx;    // compact layout
-    const uint8_t* __restrict__ sslot;    // tile-synchronous layout
-    const uint32_t* __restrict__ colw;    // tile-synchronous layout
+    const uint8_t* __restrict__ blob;     // tile-synchronous layout: per-stage blobs (the TMA source)
+    const struct PipeStage* __restrict__ stg;   // stages of every CTA
+    const int32_t* __restrict__ stg_ptr;  // [G+1]
+    const int64_t* __restrict__ tile_nnz; // TileNnz (canonical)
     int ts;
     int max_w;                            // widest tile-row slice (slice columns)
     const double* __restrict__ p64;
@@ -71,6 +73,9 @@ struct Counts {
     }
     __device__ __forceinline__ void tile(int e) { bump(t_lo, t_hi, e); }
     __device__ __forceinline__ void nz(int e) { bump(n_lo, n_hi, e); }
+    __device__ __forceinline__ void nzn(int e, int k) {
+        if (e < 3) n_lo += (unsigned long long)k << (21 * e); else n_hi += (unsigned long long)k << (21 * (e - 3));
+    }
     __device__ __forceinline__ static int field(unsigned long long lo, unsigned long long hi, int q) {
         return (int)(((q < 3 ? lo : hi) >> (21 * (q < 3 ? q : q - 3))) & 0x1FFFFFull);
     }
@@ -79,29 +84,22 @@ struct Counts {
 };
 
 // ------------------------------------------------------------------------------------------
-// Windowed SpMV over the contiguous tile rows [tr0, tr1) of one CTA (all B threads call it).
-// A window is up to WIN_TR tile rows (a multiple of H = B/16 so that half-warp h always gets
-// tile rows tr0 + h + kH, the row mapping of the dot-product contract).  Per window the CTA
-// stages in shared memory, with coalesced (cp.async) copies:
-//   compact layout:          the tile codes (tile column + e_t) of the window's tiles;
-//   tile-synchronous layout: the slot bytes and the per-column tile words of the window's
-//                            slice columns (static), plus, once per SpMV, the level bytes of
-//                            the column segments the CTA gathers.
-// Each half-warp then needs one global round trip per chunk of slots (values and x).
+// Compact (row-packed SELL-16) layout: windowed SpMV over the contiguous tile rows [tr0, tr1)
+// of one CTA (all B threads call it).  A window is up to WIN_TR tile rows (a multiple of
+// H = B/16 so that half-warp h always gets tile rows tr0 + h + kH, the row mapping of the
+// dot-product contract); per window the CTA stages the tile codes (tile column + e_t) of the
+// window's tiles in shared memory.  Used for matrices whose tile-synchronous slices would pad
+// too much (scattered patterns, e.g. C4); stencil matrices take the TMA pipeline below.
 constexpr int WIN_TR = 1024;
 constexpr int CODE_CAP = 8192;
-constexpr int COL_CAP = 2048;
-constexpr int LEV_CAP = 16384;
-constexpr int WIN_BUF_BYTES = (COL_CAP * 16 + COL_CAP * 4 + LEV_CAP) > CODE_CAP * 4 ? (COL_CAP * 16 + COL_CAP * 4 + LEV_CAP)
-                                                                                      : CODE_CAP * 4;
+constexpr int WIN_BUF_BYTES = CODE_CAP * 4;
 
 struct WinSmem {
     int32_t* hs;     // [WIN_TR+1] slot (slice column) offset of each tile row, relative to s0
     int32_t* ht;     // [WIN_TR+1] tile offset, relative to t0
     int64_t* misc;   // [4]: -, -, window end, staged
     unsigned long long* pb;   // [4] value-plane base addresses (FP64, FP32, FP16, E4M3)
-    unsigned char* buf;   // [WIN_BUF_BYTES]: compact: uint32 code[CODE_CAP]
-                          //                  TS: uint8 ss[COL_CAP*16] | uint32 cw[COL_CAP] | uint8 lev[LEV_CAP]
+    unsigned char* buf;   // [WIN_BUF_BYTES]: uint32 code[CODE_CAP]
 };
 constexpr size_t WIN_SMEM_BYTES = 2 * (WIN_TR + 1) * 4 + 4 * 8 + 8 + 4 * 8 + WIN_BUF_BYTES + 16;
 
@@ -165,245 +163,366 @@ __device__ __forceinline__ double slot_block(const Mat& A, const unsigned long l
     return acc;
 }
 
-// e_t of a tile-synchronous column word (same rule as tile_code)
-template <bool DYN>
-__device__ __forceinline__ uint32_t col_code(uint32_t word, const uint8_t* lev_s, int32_t seg_lo, bool lev_staged,
-                                             const uint8_t* __restrict__ level, int range_guard) {
-    const uint32_t tc = word >> 4;
-    int e = (int)(word & 3u);
-    if (DYN) {
-        const int lv = lev_staged ? lev_s[tc - seg_lo] : level[tc];
-        if (lv == BYP) return (tc << 3) | BYP;
-        e = max(e, lv);
-        if (range_guard) e = min(e, (int)((word >> 2) & 3u));
-    }
-    return (tc << 3) | (uint32_t)e;
-}
-
-// tile-synchronous layout: columns of one tile row; ss = slot bytes, cd = column codes
-// (tile column << 3 | e_t, uniform across the 16 lanes)
-template <bool COUNT, int N>
-__device__ __forceinline__ double ts_block(const Mat& A, const unsigned long long* w_pb, const uint8_t* ss, const uint32_t* cd, int cnt, int lane,
-                                           int64_t pos0, const double* x, double acc, Counts* cntp) {
-    uint64_t raw[N];
-    double xv[N];
-    int ev[N];
-#pragma unroll
-    for (int q = 0; q < N; ++q) {
-        const uint32_t lc = q < cnt ? ss[q * 16 + lane] : 0xFFu;
-        const uint32_t c = q < cnt ? cd[q] : (uint32_t)BYP;
-        ev[q] = lc == 0xFFu ? BYP : (int)(c & 7u);
-        if (COUNT && lc != 0xFFu) cntp->nz(ev[q]);
-        raw[q] = 0;
-        xv[q] = 0.0;
-        if (ev[q] != BYP) {
-            raw[q] = load_raw(w_pb, ev[q], pos0 + q * 16);
-            xv[q] = x[(int64_t)(c >> 3) * 16 + lc];
-        }
-    }
-#pragma unroll
-    for (int q = 0; q < N; ++q)
-        if (ev[q] != BYP) acc = __fma_rn(decode_val(ev[q], raw[q]), xv[q], acc);
-    return acc;
-}
-
 // ------------------------------------------------------------------------------------------
-// Tile-synchronous SpMV, software-pipelined over windows of 2H tile rows (half-warp h owns tile
-// rows w0+h and w0+H+h of each window -- the dot-contract mapping tr0 + h + kH).
-// Staging of window k+1 overlaps the compute of window k:
-//   * slot bytes: cp.async (16 B per slice column) into the other smem stage;
-//   * per-column records {value pointer at e_t, x offset, e_t}: column words prefetched into
-//     registers before computing window k, turned into records after it.
-// The consumer issues every load of a tile row at once (values: one aligned 8-byte word each; x:
-// one 8-byte load each), then runs the fma chain.  A bypassed / padding slot contributes
-// fma(0, 0, acc) == acc exactly (acc starts at +0 and can never become -0).
-constexpr int TSP_COLS = 1024;   // slice columns per window (cap)
-constexpr int TSP_CPT = 2;       // column words prefetched per thread (TSP_COLS / B for B = 512)
-constexpr int TSP_Q = 9;         // columns per load batch of one tile row
-struct TsRec {
-    unsigned long long vptr;     // plane_e + column slot base * size(e)   (0: bypassed column)
-    int32_t xoff;                // tile column * 16
-    int32_t e;                   // e_t
+// Tile-synchronous (TS) slices streamed through shared memory by the Tensor Memory Accelerator
+// (cp.async.bulk + mbarrier): the B200 form of "load the tiles on chip" and of the
+// one-time on-chip precision conversion.
+//
+// TS layout (convert.cu): tile row TR owns slice columns [tr_slot[TR], tr_slot[TR+1]); a slice
+// column belongs to ONE tile and holds, for lane r = row 16*TR + r, the local column (0 on
+// padding) and the value stored at TilePrec (0 on padding).  The persistent CTA owns the
+// contiguous tile rows [tr0, tr1); conversion cuts them into stages (whole groups of H = B/16
+// tile rows when they fit the caps) and packs each stage into ONE contiguous blob:
+//   [header: int32 column start per tile-row boundary, K+1 entries]
+//   [column words: (tile column << 4) | Floor << 2 | TilePrec, ncol entries]
+//   [local columns: 16 bytes per column]
+//   [destination column of each group entry: u16, grouped FP64 | FP32 | FP16 | E4M3]
+//   [values, grouped by TilePrec (FP64 block, FP32 block, FP16 block, E4M3 block), 16 per column]
+// so that a stage is a single bulk copy (TMA throughput is bounded by copies per second).
+//
+// Per stage: thread 0 keeps PIPE_NST stages in flight (one "full" mbarrier each, refilled when
+// every warp has arrived on the stage's "empty" mbarrier).  After a stage lands:
+//   1. decode pass (all threads, warp-uniform per precision group): 4 values per thread per
+//      step, exact upcast to binary64 into E[col][lane] (the on-chip conversion of P:237); the
+//      dynamic switch (Alg. 5) is applied here: bypassed columns become 0, a column with e_t
+//      below TilePrec is rounded to e_t (RNE_{e_t}(stored value));
+//   2. __syncthreads;
+//   3. FMA pass: half-warp h owns tile rows tr0 + h + kH, lane r = row 16*TR + r (the row mapping
+//      of the dot-product contract) and runs the row's single fma chain in ascending column
+//      order: acc = fma(E[c][r], x[16*tile column + local column], acc) -- a zero (padding or
+//      bypass) term leaves acc unchanged.  x is gathered through L1/L2.  A half-warp runs two
+//      tile rows (two independent chains) at once.
+// Stages hold whole groups of H tile rows (two when they fit), E is single-buffered: two
+// __syncthreads per stage order the decode and FMA passes.
+struct PipeStage {
+    int64_t col0, col1;             // slice-column range of the stage
+    int64_t boff;                   // blob offset in Mat::blob
+    int32_t tr0, tr1;               // tile rows [tr0, tr1)
+    int32_t bbytes;                 // blob bytes (multiple of 16)
+    int32_t off_cw, off_ss, off_dst, off_val;   // section offsets within the blob
+    int32_t gcnt[4];                // columns per precision group (FP64, FP32, FP16, E4M3)
+    int32_t goff[4];                // byte offset of each group's values within the blob
+    int32_t pad[3];
 };
-constexpr size_t TSP_STAGE_BYTES = (size_t)TSP_COLS * 16 + (size_t)TSP_COLS * sizeof(TsRec);
-constexpr size_t TSP_SMEM_BYTES = 2 * ((size_t)TSP_COLS * sizeof(TsRec) + (size_t)TSP_COLS * 16 + (((2 * 512 + 1) * 4 + 15) / 16 * 16)) + LEV_CAP + 64;
-constexpr size_t SPMV_SMEM_BYTES = TSP_SMEM_BYTES > WIN_SMEM_BYTES ? TSP_SMEM_BYTES : WIN_SMEM_BYTES;
+static_assert(sizeof(PipeStage) == 96, "PipeStage is 96 bytes");
 
-// the two SpMV scratch views over one shared-memory region (a matrix uses one layout)
-__device__ __forceinline__ void carve_spmv(unsigned char* p, WinSmem& w, struct TsSmem& ts);
+constexpr int PIPE_NST = 3;        // stages in flight
+constexpr int PIPE_KCAP = 64;      // tile rows per stage
+constexpr int PIPE_CCAP = 600;     // slice columns per stage
+constexpr int PIPE_VCAP = 32768;   // value bytes per stage
+__host__ __device__ constexpr int pipe_r16(int v) { return (v + 15) & ~15; }
+constexpr int PIPE_BLOB_CAP = pipe_r16((PIPE_KCAP + 1) * 4) + pipe_r16(PIPE_CCAP * 4) + PIPE_CCAP * 16 +
+                              pipe_r16(PIPE_CCAP * 2 + 8) + PIPE_VCAP;
+constexpr int PS_INFO = pipe_r16(PIPE_BLOB_CAP);               // int32 tr0, tr1, off_cw, off_ss, off_dst, gcnt[4], goff[4]
+constexpr int PS_BYTES = PS_INFO + 64;
+constexpr int PIPE_E_BYTES = PIPE_CCAP * 128;                  // one decoded stage: FP64 [col][lane]
+constexpr int PIPE_LEV_CAP = 4096;                             // staged level bytes (column segments gathered)
+// region: [NST slots][E][full NST u64][empty NST u64][ctr u64][pad][levels]
+constexpr size_t PIPE_SMEM_BYTES = (size_t)PIPE_NST * PS_BYTES + (size_t)PIPE_E_BYTES + 16 * PIPE_NST + 16 + PIPE_LEV_CAP;
 
-// stage st occupies [base + st*TSP_STRIDE, ...): records | slot bytes | headers; then the levels.
-// (Stage pointers are computed, not looked up: a runtime-indexed pointer array would live in
-// local memory.)
-constexpr size_t TSP_HS_BYTES = ((2 * 512 + 1) * 4 + 15) / 16 * 16;
-constexpr size_t TSP_STRIDE = (size_t)TSP_COLS * sizeof(TsRec) + (size_t)TSP_COLS * 16 + TSP_HS_BYTES;
 struct TsSmem {
     unsigned char* base;
-    __device__ __forceinline__ TsRec* rec(int st) const { return reinterpret_cast<TsRec*>(base + st * TSP_STRIDE); }
-    __device__ __forceinline__ uint8_t* ss(int st) const { return base + st * TSP_STRIDE + (size_t)TSP_COLS * sizeof(TsRec); }
-    __device__ __forceinline__ int32_t* hs(int st) const {
-        return reinterpret_cast<int32_t*>(base + st * TSP_STRIDE + (size_t)TSP_COLS * sizeof(TsRec) + (size_t)TSP_COLS * 16);
+    __device__ __forceinline__ unsigned char* slot(int s) const { return base + (size_t)s * PS_BYTES; }
+    __device__ __forceinline__ unsigned char* E(int b) const { return base + (size_t)PIPE_NST * PS_BYTES + (size_t)b * PIPE_E_BYTES; }
+    __device__ __forceinline__ unsigned long long* full(int s) const {
+        return reinterpret_cast<unsigned long long*>(E(1)) + s;
     }
-    __device__ __forceinline__ uint8_t* lev() const { return base + 2 * TSP_STRIDE; }
+    __device__ __forceinline__ unsigned long long* empty(int s) const { return full(0) + PIPE_NST + s; }
+    __device__ __forceinline__ unsigned long long* ctr() const { return full(0) + 2 * PIPE_NST; }
+    __device__ __forceinline__ uint8_t* lev() const { return reinterpret_cast<uint8_t*>(full(0) + 2 * PIPE_NST + 2); }
 };
 
-__device__ __forceinline__ uint32_t lds_u8(const void* p) {
-    uint32_t v;
-    asm volatile("ld.shared.u8 %0, [%1];" : "=r"(v) : "r"((unsigned)__cvta_generic_to_shared(p)));
+__device__ __forceinline__ unsigned smem_u32(const void* p) { return (unsigned)__cvta_generic_to_shared(p); }
+__device__ __forceinline__ void mbar_init(unsigned long long* b, unsigned cnt) {
+    asm volatile("mbarrier.init.shared::cta.b64 [%0], %1;" ::"r"(smem_u32(b)), "r"(cnt) : "memory");
+}
+__device__ __forceinline__ void mbar_expect_tx(unsigned long long* b, unsigned bytes) {
+    asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(smem_u32(b)), "r"(bytes) : "memory");
+}
+__device__ __forceinline__ void mbar_arrive(unsigned long long* b) {
+    asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];" ::"r"(smem_u32(b)) : "memory");
+}
+__device__ __forceinline__ bool mbar_try(unsigned long long* b, unsigned parity) {
+    unsigned ok;
+    asm volatile("{\n\t.reg .pred p;\n\tmbarrier.try_wait.parity.shared::cta.b64 p, [%1], %2;\n\tselp.u32 %0, 1, 0, p;\n\t}"
+                 : "=r"(ok) : "r"(smem_u32(b)), "r"(parity) : "memory");
+    return ok != 0;
+}
+// bounded wait: a pipeline that cannot complete traps (kernel error) instead of hanging the GPU
+static __device__ __noinline__ void mbar_wait_slow(unsigned long long* b, unsigned parity) {
+    unsigned long long t0;
+    asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t0));
+    for (unsigned k = 1;; ++k) {
+        if (mbar_try(b, parity)) return;
+        if ((k & 1023u) == 0) {
+            unsigned long long t1;
+            asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t1));
+            if (t1 - t0 > 20ull * 1000000000ull) __trap();
+        }
+    }
+}
+__device__ __forceinline__ void mbar_wait(unsigned long long* b, unsigned parity) {
+    if (!mbar_try(b, parity)) mbar_wait_slow(b, parity);
+}
+__device__ __forceinline__ unsigned long long policy_evict_first() {
+    unsigned long long p;
+    asm volatile("createpolicy.fractional.L2::evict_first.b64 %0, 1.0;" : "=l"(p));
+    return p;
+}
+// the matrix is read once per SpMV -> L2 evict_first (keeps the solver's vectors L2-resident)
+__device__ __forceinline__ void bulk_g2s_ef(void* dst, const void* src, unsigned bytes, unsigned long long* bar,
+                                            unsigned long long pol) {
+    asm volatile("cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes.L2::cache_hint [%0], [%1], %2, [%3], %4;"
+                 ::"r"(smem_u32(dst)), "l"(src), "r"(bytes), "r"(smem_u32(bar)), "l"(pol) : "memory");
+}
+
+// all threads; followed by a __syncthreads of the caller before the first SpMV
+__device__ __forceinline__ void pipe_init(const TsSmem& sm) {
+    if (threadIdx.x == 0) {
+        for (int s = 0; s < PIPE_NST; ++s) {
+            mbar_init(sm.full(s), 1);
+            mbar_init(sm.empty(s), blockDim.x >> 5);
+        }
+        *sm.ctr() = 0ull;
+        asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+    }
+}
+
+// thread 0: stage st -> slot (one bulk copy)
+__device__ __forceinline__ void pipe_issue(const Mat& A, const PipeStage& st, unsigned char* slot, unsigned long long* full,
+                                           unsigned long long pol) {
+    int32_t* info = reinterpret_cast<int32_t*>(slot + PS_INFO);
+    info[0] = st.tr0;
+    info[1] = st.tr1;
+    info[2] = st.off_cw;
+    info[3] = st.off_ss;
+    info[4] = st.off_dst;
+#pragma unroll
+    for (int q = 0; q < 4; ++q) { info[5 + q] = st.gcnt[q]; info[9 + q] = st.goff[q]; }
+    mbar_expect_tx(full, (unsigned)st.bbytes);
+    bulk_g2s_ef(slot, A.blob + st.boff, (unsigned)st.bbytes, full, pol);
+}
+
+__device__ __forceinline__ int lds_i32(unsigned a) {
+    int v;
+    asm volatile("ld.shared.s32 %0, [%1];" : "=r"(v) : "r"(a));
     return v;
 }
-__device__ __forceinline__ void lds_rec(const void* p, unsigned long long& vptr, int& xoff, int& e) {
-    unsigned lo, hi, xo, ee;
-    asm volatile("ld.shared.v4.u32 {%0, %1, %2, %3}, [%4];"
-                 : "=r"(lo), "=r"(hi), "=r"(xo), "=r"(ee) : "r"((unsigned)__cvta_generic_to_shared(p)));
-    vptr = ((unsigned long long)hi << 32) | lo;
-    xoff = (int)xo;
-    e = (int)ee;
+__device__ __forceinline__ uint32_t lds_u32(unsigned a) {
+    uint32_t v;
+    asm volatile("ld.shared.u32 %0, [%1];" : "=r"(v) : "r"(a));
+    return v;
+}
+__device__ __forceinline__ uint32_t lds_u16(unsigned a) {
+    uint32_t v;
+    asm volatile("ld.shared.u16 %0, [%1];" : "=r"(v) : "r"(a));
+    return v;
+}
+__device__ __forceinline__ uint32_t lds_u8(unsigned a) {
+    uint32_t v;
+    asm volatile("ld.shared.u8 %0, [%1];" : "=r"(v) : "r"(a));
+    return v;
+}
+__device__ __forceinline__ double lds_f64(unsigned a) {
+    double v;
+    asm volatile("ld.shared.f64 %0, [%1];" : "=d"(v) : "r"(a));
+    return v;
+}
+__device__ __forceinline__ uint2 lds_v2(unsigned a) {
+    uint2 v;
+    asm volatile("ld.shared.v2.u32 {%0, %1}, [%2];" : "=r"(v.x), "=r"(v.y) : "r"(a));
+    return v;
+}
+__device__ __forceinline__ uint4 lds_v4(unsigned a) {
+    uint4 v;
+    asm volatile("ld.shared.v4.u32 {%0, %1, %2, %3}, [%4];" : "=r"(v.x), "=r"(v.y), "=r"(v.z), "=r"(v.w) : "r"(a));
+    return v;
+}
+__device__ __forceinline__ void sts_d2(unsigned a, double u, double v) {
+    asm volatile("st.shared.v2.f64 [%0], {%1, %2};" ::"r"(a), "d"(u), "d"(v) : "memory");
 }
 
-// one tile row of a window: all its slots' loads are issued before the fma chain.  Padding and
-// bypassed slots load a zero value word (their x load reads a valid element of the same
-// segment), so every slot is one unconditional fma: fma(0, x, acc) == acc exactly.
-template <bool COUNT>
-__device__ __forceinline__ double ts_row(const uint8_t* ss, const TsRec* rec, int a, int W, int lane,
-                                         const double* x, Counts* cntp) {
-    double acc = 0.0;
-    for (int k = 0; k < W; k += TSP_Q) {
-        unsigned long long wv[TSP_Q];
-        double xv[TSP_Q];
-        uint32_t meta[TSP_Q];          // ((addr & 7) << 11) | e
-        const int n = W - k;
-#pragma unroll
-        for (int q = 0; q < TSP_Q; ++q) {
-            // columns past the tile row (q >= n) read column a (always staged) and are masked
-            const bool in = q < n;
-            const int c = in ? a + k + q : a;
-            const uint32_t lc = lds_u8(ss + c * 16 + lane);
-            unsigned long long vptr;
-            int xoff, e;
-            lds_rec(rec + c, vptr, xoff, e);
-            if (COUNT && in && lc != 0xFFu) cntp->nz(e);
-            const bool ok = in && lc != 0xFFu && e != BYP;
-            const unsigned long long ad = vptr + ((unsigned long long)lane << (3 - (e & 3)));
-            meta[q] = ((uint32_t)(ad & 7ull) << 11) | (uint32_t)(e & 3);
-            unsigned long long w = 0ull;
-            asm volatile("{\n\t.reg .pred p;\n\tsetp.ne.u32 p, %2, 0;\n\t@p ld.global.nc.u64 %0, [%1];\n\t}"
-                         : "+l"(w) : "l"(ad & ~7ull), "r"((unsigned)ok));
-            wv[q] = w;
-            xv[q] = x[xoff + (int)(lc & 15u)];
+// level of tile column tc for the dynamic switch
+__device__ __forceinline__ int col_level(uint32_t tc, const uint8_t* __restrict__ level, unsigned lev_s, bool lev_staged,
+                                         int32_t seg_lo) {
+    return lev_staged ? (int)lds_u8(lev_s + (tc - (uint32_t)seg_lo)) : (int)level[tc];
+}
+
+__device__ __forceinline__ double e4m3_lo(uint32_t w2) {   // the E4M3 byte in bits 0..7 -> binary64 (exact)
+    const __half_raw h = __nv_cvt_fp8_to_halfraw((__nv_fp8_storage_t)(w2 & 0xFFu), __NV_E4M3);
+    return (double)__half2float(__half(h));
+}
+__device__ __forceinline__ double h16(uint32_t bits) { return (double)__half2float(__ushort_as_half((unsigned short)bits)); }
+
+// decode pass: group Q (0 FP64 .. 3 E4M3) of the stage in slot -> E.  Unit = 4 lanes of one column.
+template <int Q, bool DYN>
+__device__ __forceinline__ void pipe_decode_group(unsigned slot, unsigned Eb, int ncol_q, unsigned goff, unsigned dst_q, unsigned cw,
+                                                  const uint8_t* __restrict__ level, unsigned lev_s, bool lev_staged,
+                                                  int32_t seg_lo, int range_guard) {
+    const int units = ncol_q * 4;
+    for (int u = threadIdx.x; u < units; u += blockDim.x) {
+        const int j = u >> 2, r0 = (u & 3) * 4;
+        const unsigned d = lds_u16(dst_q + 2u * (unsigned)j);          // destination column in the stage
+        const unsigned src = slot + goff + (unsigned)((j * 16 + r0) << (3 - Q));
+        double v[4];
+        if (Q == 0) {
+            const uint4 a = lds_v4(src), b = lds_v4(src + 16);
+            v[0] = __hiloint2double((int)a.y, (int)a.x); v[1] = __hiloint2double((int)a.w, (int)a.z);
+            v[2] = __hiloint2double((int)b.y, (int)b.x); v[3] = __hiloint2double((int)b.w, (int)b.z);
+        } else if (Q == 1) {
+            const uint4 a = lds_v4(src);
+            v[0] = (double)__uint_as_float(a.x); v[1] = (double)__uint_as_float(a.y);
+            v[2] = (double)__uint_as_float(a.z); v[3] = (double)__uint_as_float(a.w);
+        } else if (Q == 2) {
+            const uint2 a = lds_v2(src);
+            v[0] = h16(a.x); v[1] = h16(a.x >> 16); v[2] = h16(a.y); v[3] = h16(a.y >> 16);
+        } else {
+            const uint32_t a = lds_u32(src);
+            v[0] = e4m3_lo(a); v[1] = e4m3_lo(a >> 8); v[2] = e4m3_lo(a >> 16); v[3] = e4m3_lo(a >> 24);
         }
+        if (DYN) {   // e_t = bypass | max(TilePrec, level), range guard e_t <= Floor (Alg. 5)
+            const uint32_t word = lds_u32(cw + 4u * d);
+            const int lv = col_level(word >> 4, level, lev_s, lev_staged, seg_lo);
+            if (lv > Q) {
+                if (lv == BYP) { v[0] = v[1] = v[2] = v[3] = 0.0; }
+                else {
+                    int e = lv;
+                    if (range_guard) e = min(e, (int)((word >> 2) & 3u));
+                    if (e != Q) {
 #pragma unroll
-        for (int q = 0; q < TSP_Q; ++q)
-            acc = __fma_rn(decode_val((int)(meta[q] & 3u), wv[q] >> (meta[q] >> 8)), xv[q], acc);
+                        for (int k = 0; k < 4; ++k) v[k] = round_to(v[k], e);
+                    }
+                }
+            }
+        }
+        const unsigned ea = Eb + d * 128u + (unsigned)r0 * 8u;
+        sts_d2(ea, v[0], v[1]);
+        sts_d2(ea + 16, v[2], v[3]);
     }
-    return acc;
 }
 
+template <bool DYN>
+__device__ __forceinline__ void pipe_decode(unsigned slot, unsigned Eb, const uint8_t* __restrict__ level, unsigned lev_s, bool lev_staged,
+                                            int32_t seg_lo, int range_guard) {
+    const unsigned cw = slot + (unsigned)lds_i32(slot + PS_INFO + 8);
+    unsigned dst = slot + (unsigned)lds_i32(slot + PS_INFO + 16);
+    const int g0 = lds_i32(slot + PS_INFO + 20), g1 = lds_i32(slot + PS_INFO + 24), g2 = lds_i32(slot + PS_INFO + 28),
+              g3 = lds_i32(slot + PS_INFO + 32);
+    pipe_decode_group<0, DYN>(slot, Eb, g0, (unsigned)lds_i32(slot + PS_INFO + 36), dst, cw, level, lev_s, lev_staged, seg_lo, range_guard);
+    dst += 2u * (unsigned)g0;
+    pipe_decode_group<1, DYN>(slot, Eb, g1, (unsigned)lds_i32(slot + PS_INFO + 40), dst, cw, level, lev_s, lev_staged, seg_lo, range_guard);
+    dst += 2u * (unsigned)g1;
+    pipe_decode_group<2, DYN>(slot, Eb, g2, (unsigned)lds_i32(slot + PS_INFO + 44), dst, cw, level, lev_s, lev_staged, seg_lo, range_guard);
+    dst += 2u * (unsigned)g2;
+    pipe_decode_group<3, DYN>(slot, Eb, g3, (unsigned)lds_i32(slot + PS_INFO + 48), dst, cw, level, lev_s, lev_staged, seg_lo, range_guard);
+}
+
+// four columns [c, c+4) of one tile row with n valid (past the row: re-read column c, masked)
+struct PipeRow {
+    unsigned a;      // first column (stage-relative)
+    int W;           // columns
+    double acc;
+};
+__device__ __forceinline__ void pipe_load4(unsigned cw, unsigned ssl, unsigned El, unsigned c, int n, const double* __restrict__ x,
+                                           double (&ev)[4], double (&xv)[4]) {
+    const unsigned b4 = 4u * c, b16 = 16u * c, b128 = 128u * c;
+#pragma unroll
+    for (int q = 0; q < 4; ++q) {
+        const unsigned o = q < n ? (unsigned)q : 0u;
+        const uint32_t word = lds_u32(cw + b4 + 4u * o);
+        const uint32_t lc = lds_u8(ssl + b16 + 16u * o);
+        ev[q] = lds_f64(El + b128 + 128u * o);
+        xv[q] = x[(word & ~15u) | lc];
+    }
+}
+
+// FMA pass of one stage: half-warp h takes its tile rows (TR = tr0c + h (mod H)) in ascending
+// order, two at a time (two independent fma chains per lane).
+template <class Emit>
+__device__ __forceinline__ void pipe_fma(const Mat& A, unsigned slot, unsigned Eb, int64_t tr0c, const double* __restrict__ x,
+                                         const double* __restrict__ own, Emit& emit) {
+    const int t = threadIdx.x, H = blockDim.x >> 4, h = t >> 4, lane = t & 15;
+    const int32_t S0 = lds_i32(slot + PS_INFO), S1 = lds_i32(slot + PS_INFO + 4);
+    const unsigned cw = slot + (unsigned)lds_i32(slot + PS_INFO + 8);
+    const unsigned ssl = slot + (unsigned)lds_i32(slot + PS_INFO + 12) + (unsigned)lane;
+    const unsigned El = Eb + 8u * (unsigned)lane;
+    const int off0 = (int)((S0 - tr0c) % H);
+    for (int64_t TR = S0 + (h - off0 + H) % H; TR < S1; TR += 2 * H) {
+        const bool two = TR + H < S1;
+        const int k0 = (int)(TR - S0), k1 = two ? k0 + H : k0;
+        const int a0 = lds_i32(slot + 4u * k0), W0 = lds_i32(slot + 4u * (k0 + 1)) - a0;
+        const int a1 = lds_i32(slot + 4u * k1), W1 = two ? lds_i32(slot + 4u * (k1 + 1)) - a1 : 0;
+        const int64_t i0 = TR * 16 + lane, i1 = i0 + 16 * H;
+        const double ov0 = (own != nullptr && i0 < A.n_rows) ? own[i0] : 0.0;
+        const double ov1 = (own != nullptr && two && i1 < A.n_rows) ? own[i1] : 0.0;
+        double acc0 = 0.0, acc1 = 0.0;
+        const int Wm = max(W0, W1);
+        for (int cb = 0; cb < Wm; cb += 4) {
+            double e0[4], x0[4], e1[4], x1[4];
+            const int n0 = W0 - cb, n1 = W1 - cb;
+            pipe_load4(cw, ssl, El, (unsigned)(a0 + (n0 > 0 ? cb : 0)), n0, x, e0, x0);
+            pipe_load4(cw, ssl, El, (unsigned)(a1 + (n1 > 0 ? cb : 0)), n1, x, e1, x1);
+#pragma unroll
+            for (int q = 0; q < 4; ++q) {
+                if (q < n0) acc0 = __fma_rn(e0[q], x0[q], acc0);
+                if (q < n1) acc1 = __fma_rn(e1[q], x1[q], acc1);
+            }
+        }
+        emit(TR, lane, acc0, ov0);
+        if (two) emit(TR + H, lane, acc1, ov1);
+    }
+}
+
+// the whole SpMV of one CTA (all threads), tile rows [tr0c, tr1c) = the CTA's plan range
 template <bool DYN, bool COUNT, class Emit>
-__device__ __forceinline__ void spmv_ts_pipe(const Mat& A, int64_t tr0, int64_t tr1, const double* x, const uint8_t* __restrict__ level,
-                             int range_guard, const TsSmem& sm, Counts* cnt, int32_t seg_lo, int32_t seg_hi, Emit emit) {
-    const int t = threadIdx.x, B = blockDim.x, H = B >> 4, h = t >> 4, lane = t & 15;
-    const int NW = 2 * H;                       // tile rows per window
+__device__ __forceinline__ void spmv_pipe(const Mat& A, int64_t tr0c, int64_t tr1c, const double* __restrict__ x,
+                                          const uint8_t* __restrict__ level, int range_guard, const TsSmem& sm, Counts* cnt,
+                                          int32_t seg_lo, int32_t seg_hi, const double* __restrict__ own, Emit& emit) {
+    const int t = threadIdx.x, B = blockDim.x;
+    const int32_t s_begin = A.stg_ptr[blockIdx.x], ns = A.stg_ptr[blockIdx.x + 1] - s_begin;
     const int32_t nlev = seg_hi - seg_lo + 1;
-    const bool lev_staged = DYN && nlev > 0 && nlev <= LEV_CAP;
-    const unsigned long long pb0 = (unsigned long long)A.p64, pb1 = (unsigned long long)A.p32,
-                             pb2 = (unsigned long long)A.p16, pb3 = (unsigned long long)A.p8;
-    __syncthreads();
+    const bool lev_staged = DYN && nlev > 0 && nlev <= PIPE_LEV_CAP;
+    __syncthreads();                          // smem users of the previous phase are done
+    const unsigned u0 = (unsigned)*sm.ctr();
+    unsigned long long pol = 0;
+    if (t == 0) {
+        pol = policy_evict_first();
+        for (int k = 0; k < min(ns, PIPE_NST); ++k) {
+            const unsigned u = u0 + (unsigned)k, sl = u % PIPE_NST, mm = u / PIPE_NST;
+            if (mm > 0) mbar_wait(sm.empty(sl), (mm - 1) & 1u);
+            pipe_issue(A, A.stg[s_begin + k], sm.slot(sl), sm.full(sl), pol);
+        }
+    }
     if (lev_staged)
         for (int i = t; i < nlev; i += B) sm.lev()[i] = level[seg_lo + i];
     if (COUNT)
-        for (int64_t i = A.tr_tile[tr0] + t; i < A.tr_tile[tr1]; i += B)
-            cnt->tile(tile_code<DYN>(A.tile_info[i], level, range_guard) & 7u);
-    // prefetch state for the next window: header (thread i <= NW) and column words (registers)
-    uint32_t cw0 = 0u, cw1 = 0u;
-    static_assert(TSP_CPT == 2, "two column words per thread");
-#define TSP_FETCH_HDR(W0, HDR)                                                               \
-    {                                                                                       \
-        const int64_t nw_ = min((int64_t)NW, tr1 - (W0));                                   \
-        HDR = t <= nw_ ? A.tr_slot[(W0) + t] : A.tr_slot[(W0) + nw_];                       \
-    }
-#define TSP_PUBLISH_HDR(ST, W0, HDR)                                                         \
-    {                                                                                       \
-        const int64_t nw_ = min((int64_t)NW, tr1 - (W0));                                   \
-        if (t <= nw_) sm.hs(ST)[t] = (int32_t)((HDR) - A.tr_slot[W0]);                      \
-    }
-#define TSP_ISSUE(ST, SBASE, NCOL)                                                           \
-    {                                                                                       \
-        for (int c_ = t; c_ < (NCOL); c_ += B) cp_async16(sm.ss(ST) + c_ * 16, A.sslot + ((SBASE) + c_) * 16); \
-        cw0 = t < (NCOL) ? __ldg(A.colw + (SBASE) + t) : 0u;                                \
-        cw1 = t + B < (NCOL) ? __ldg(A.colw + (SBASE) + t + B) : 0u;                        \
-    }
-    auto build_rec = [&](int st, int64_t sbase, int c, uint32_t word) {
-        const uint32_t tc = word >> 4;
-        int e = (int)(word & 3u);
-        if (DYN) {
-            const int lv = lev_staged ? sm.lev()[tc - seg_lo] : level[tc];
-            if (lv == BYP) e = BYP;
-            else {
-                e = max(e, lv);
-                if (range_guard) e = min(e, (int)((word >> 2) & 3u));
-            }
+        for (int64_t i = A.tr_tile[tr0c] + t; i < A.tr_tile[tr1c]; i += B) {
+            const int e = (int)(tile_code<DYN>(A.tile_info[i], level, range_guard) & 7u);
+            cnt->tile(e);
+            cnt->nzn(e, (int)(A.tile_nnz[i + 1] - A.tile_nnz[i]));
         }
-        const unsigned long long pbase = e == 0 ? pb0 : e == 1 ? pb1 : e == 2 ? pb2 : pb3;
-        const unsigned long long vptr = pbase + ((unsigned long long)((sbase + c) * 16) << (3 - (e & 3)));
-        sm.rec(st)[c] = TsRec{e == BYP ? 0ull : vptr, (int32_t)(tc * 16), e};
-    };
-#define TSP_BUILD(ST, SBASE, NCOL)                                                           \
-    {                                                                                       \
-        if (t < (NCOL)) build_rec(ST, SBASE, t, cw0);                                       \
-        if (t + B < (NCOL)) build_rec(ST, SBASE, t + B, cw1);                               \
-    }
-    // window 0: staged synchronously
-    int64_t w0 = tr0;
-    int stage = 0;
-    int64_t hdr = 0;
-    if (w0 < tr1) TSP_FETCH_HDR(w0, hdr)
     __syncthreads();
-    if (w0 < tr1) {
-        const int64_t nw = min((int64_t)NW, tr1 - w0);
-        TSP_PUBLISH_HDR(0, w0, hdr)
-        __syncthreads();
-        const int ncol = sm.hs(0)[nw];
-        const int64_t sbase = A.tr_slot[w0];
-        TSP_ISSUE(0, sbase, ncol)
-        TSP_BUILD(0, sbase, ncol)
-        cp_async_wait_all();
-        __syncthreads();
-    }
-    while (w0 < tr1) {
-        const int64_t nw = min((int64_t)NW, tr1 - w0);
-        const int64_t w1 = w0 + nw;
-        // prefetch window k+1: header, slot bytes (cp.async), column words (registers)
-        int ncol1 = 0;
-        int64_t sbase1 = 0;
-        if (w1 < tr1) {
-            TSP_FETCH_HDR(w1, hdr)
-            TSP_PUBLISH_HDR(stage ^ 1, w1, hdr)
-            __syncthreads();
-            const int64_t nw1 = min((int64_t)NW, tr1 - w1);
-            ncol1 = sm.hs(stage ^ 1)[nw1];
-            sbase1 = A.tr_slot[w1];
-            TSP_ISSUE(stage ^ 1, sbase1, ncol1)
+    const unsigned lev_s = smem_u32(sm.lev());
+    PipeStage nxt;
+    for (int k = 0; k < ns; ++k) {
+        const unsigned u = u0 + (unsigned)k, sl = u % PIPE_NST, mm = u / PIPE_NST;
+        const bool refill = t == 0 && k + PIPE_NST < ns;
+        if (refill) nxt = A.stg[s_begin + k + PIPE_NST];
+        mbar_wait(sm.full(sl), mm & 1u);
+        const unsigned slot = smem_u32(sm.slot(sl)), Eb = smem_u32(sm.E(0));
+        if (k > 0) __syncthreads();           // E free: every warp is done with the previous stage
+        pipe_decode<DYN>(slot, Eb, level, lev_s, lev_staged, seg_lo, range_guard);
+        __syncthreads();                      // E complete
+        pipe_fma(A, slot, Eb, tr0c, x, own, emit);
+        __syncwarp();
+        if ((t & 31) == 0) mbar_arrive(sm.empty(sl));
+        if (refill) {
+            mbar_wait(sm.empty(sl), mm & 1u);
+            pipe_issue(A, nxt, sm.slot(sl), sm.full(sl), pol);
         }
-        // compute window k: half-warp h owns rows w0 + h and w0 + H + h
-        {
-            const int32_t* hs = sm.hs(stage);
-            for (int li = h; li < nw; li += H) {
-                const int a = hs[li], W = hs[li + 1] - a;
-                const double acc = ts_row<COUNT>(sm.ss(stage), sm.rec(stage), a, W, lane, x, cnt);
-                emit(w0 + li, lane, acc);
-            }
-        }
-        if (w1 < tr1) TSP_BUILD(stage ^ 1, sbase1, ncol1)
-        cp_async_wait_all();
-        __syncthreads();
-        stage ^= 1;
-        w0 = w1;
     }
-#undef TSP_FETCH_HDR
-#undef TSP_PUBLISH_HDR
-#undef TSP_ISSUE
-#undef TSP_BUILD
+    __syncthreads();
+    if (t == 0) *sm.ctr() = (unsigned long long)(u0 + (unsigned)ns);
 }
 
 __device__ __forceinline__ void carve_spmv(unsigned char* base, WinSmem& w, TsSmem& ts) {
@@ -418,31 +537,25 @@ __device__ __forceinline__ void carve_spmv(unsigned char* base, WinSmem& w, TsSm
     p += (WIN_TR + 1) * 4;
     p = reinterpret_cast<unsigned char*>((reinterpret_cast<uintptr_t>(p) + 15) & ~uintptr_t(15));
     w.buf = p;
-    ts.base = base;
+    ts.base = base;    // the two views overlap: a matrix uses one layout
 }
+constexpr size_t SPMV_SMEM_BYTES = PIPE_SMEM_BYTES > WIN_SMEM_BYTES ? PIPE_SMEM_BYTES : WIN_SMEM_BYTES;
 
-// emit(TR, lane, value) is called by every lane for each of its tile rows, in ascending TR.
-// seg_lo/seg_hi: the column segments this CTA's tiles gather (tile-synchronous level staging).
+// emit(TR, lane, value, own[row]) is called by every lane for each of its tile rows, in ascending
+// TR; own (nullable) is a vector the caller's fused dot needs at the row (prefetched).
+// seg_lo/seg_hi: the column segments this CTA's tiles gather (level staging).
 template <bool DYN, bool COUNT, int PF, class Emit>
 __device__ __forceinline__ void spmv_cta(const Mat& A, int64_t tr0, int64_t tr1, const double* x, const uint8_t* __restrict__ level,
                          int range_guard, const WinSmem& w, const TsSmem& tsm, Counts* cnt, int32_t seg_lo,
-                         int32_t seg_hi, Emit emit) {
-    const int t = threadIdx.x, B = blockDim.x, H = B >> 4, h = t >> 4, lane = t & 15;
-    // tile-synchronous slices whose windows of 2H tile rows fit the staging buffers
-    if (A.ts && (int64_t)A.max_w * 2 * H <= min(TSP_COLS, TSP_CPT * B) && 2 * H <= 2 * 512) {
-        spmv_ts_pipe<DYN, COUNT>(A, tr0, tr1, x, level, range_guard, tsm, cnt, seg_lo, seg_hi, emit);
+                         int32_t seg_hi, const double* own, Emit emit) {
+    if (A.ts) {
+        spmv_pipe<DYN, COUNT>(A, tr0, tr1, x, level, range_guard, tsm, cnt, seg_lo, seg_hi, own, emit);
         return;
     }
-    uint8_t* ss = w.buf;
-    uint32_t* cw = reinterpret_cast<uint32_t*>(w.buf + COL_CAP * 16);
-    uint8_t* lev_s = w.buf + COL_CAP * 16 + COL_CAP * 4;
-    const int32_t nlev = seg_hi - seg_lo + 1;
-    const bool lev_staged = DYN && A.ts && nlev > 0 && nlev <= LEV_CAP;
+    const int t = threadIdx.x, B = blockDim.x, H = B >> 4, h = t >> 4, lane = t & 15;
     __syncthreads();
     if (t < 4) w.pb[t] = t == 0 ? (unsigned long long)A.p64 : t == 1 ? (unsigned long long)A.p32
                        : t == 2 ? (unsigned long long)A.p16 : (unsigned long long)A.p8;
-    if (lev_staged)
-        for (int i = t; i < nlev; i += B) lev_s[i] = level[seg_lo + i];
     for (int64_t w0 = tr0; w0 < tr1;) {
         const int64_t wmax = min(tr1 - w0, (int64_t)WIN_TR);
         __syncthreads();   // previous window fully consumed
@@ -453,57 +566,20 @@ __device__ __forceinline__ void spmv_cta(const Mat& A, int64_t tr0, int64_t tr1,
         }
         __syncthreads();
         if (t == 0) {
-            // largest multiple of H (or the whole rest) whose tiles / columns fit the buffer
-            const int32_t* lim = A.ts ? w.hs : w.ht;
-            const int cap = A.ts ? COL_CAP : CODE_CAP;
+            // largest multiple of H (or the whole rest) whose tiles fit the code buffer
             int64_t nw = wmax;
-            if (lim[nw] > cap) {
+            if (w.ht[nw] > CODE_CAP) {
                 nw = (int64_t)H;
-                while (nw + H <= wmax && lim[nw + H] <= cap) nw += H;
+                while (nw + H <= wmax && w.ht[nw + H] <= CODE_CAP) nw += H;
                 if (nw > wmax) nw = wmax;
             }
             w.misc[2] = nw;
-            w.misc[3] = lim[nw] <= cap;
+            w.misc[3] = w.ht[nw] <= CODE_CAP;
         }
         __syncthreads();
         const int64_t nw = w.misc[2];
         const bool staged = w.misc[3] != 0;
         const int nt = w.ht[nw];
-        if (A.ts) {
-            const int ncol = w.hs[nw];
-            if (COUNT)
-                for (int i = t; i < nt; i += B) cnt->tile(tile_code<DYN>(A.tile_info[t0 + i], level, range_guard) & 7u);
-            if (staged) {
-                for (int c = t; c < ncol; c += B) cp_async16(ss + c * 16, A.sslot + (s0 + c) * 16);
-                for (int c = t; c < ncol; c += B)     // column words -> column codes (tc << 3 | e_t)
-                    cw[c] = col_code<DYN>(__ldg(A.colw + s0 + c), lev_s, seg_lo, lev_staged, level, range_guard);
-                cp_async_wait_all();
-            }
-            __syncthreads();
-            for (int64_t li = h; li < nw; li += H) {
-                const int32_t a = w.hs[li];
-                const int W = w.hs[li + 1] - a;
-                const int64_t sb = s0 + a;
-                double acc = 0.0;
-                for (int k = 0; k < W; k += PF) {
-                    if (staged) {
-                        acc = ts_block<COUNT, PF>(A, w.pb, ss + (a + k) * 16, cw + a + k, min(W - k, PF), lane,
-                                                  (sb + k) * 16 + lane, x, acc, cnt);
-                    } else {
-                        uint32_t cdl[PF];
-#pragma unroll
-                        for (int q = 0; q < PF; ++q)
-                            cdl[q] = k + q < W ? col_code<DYN>(__ldg(A.colw + sb + k + q), lev_s, seg_lo, lev_staged, level,
-                                                                range_guard) : (uint32_t)BYP;
-                        acc = ts_block<COUNT, PF>(A, w.pb, A.sslot + (sb + k) * 16, cdl, min(W - k, PF), lane,
-                                                  (sb + k) * 16 + lane, x, acc, cnt);
-                    }
-                }
-                emit(w0 + li, lane, acc);
-            }
-            w0 += nw;
-            continue;
-        }
         uint32_t* code = reinterpret_cast<uint32_t*>(w.buf);
         for (int i = t; i < nt; i += B) {
             const uint32_t c = tile_code<DYN>(A.tile_info[t0 + i], level, range_guard);
@@ -514,7 +590,12 @@ __device__ __forceinline__ void spmv_cta(const Mat& A, int64_t tr0, int64_t tr1,
         // half-warp h: tile rows w0 + h + kH, the next row's first PF slot words prefetched
         uint16_t nxt[PF];
         int64_t li = h;
-#define CMP_LOAD_FIRST(L)                                                                           {                                                                                               const int32_t a_ = w.hs[L], W_ = w.hs[(L) + 1] - a_;                                        const uint16_t* sp_ = A.sidx + (s0 + a_) * 16 + lane;                                       _Pragma("unroll") for (int q = 0; q < PF; ++q) nxt[q] = q < W_ ? __ldg(sp_ + q * 16) : mf::SLOT_PAD;         }
+#define CMP_LOAD_FIRST(L)                                                                           \
+    {                                                                                               \
+        const int32_t a_ = w.hs[L], W_ = w.hs[(L) + 1] - a_;                                        \
+        const uint16_t* sp_ = A.sidx + (s0 + a_) * 16 + lane;                                       \
+        _Pragma("unroll") for (int q = 0; q < PF; ++q) nxt[q] = q < W_ ? __ldg(sp_ + q * 16) : mf::SLOT_PAD; \
+    }
         if (li < nw) CMP_LOAD_FIRST(li)
         for (; li < nw; li += H) {
             uint16_t cur[PF];
@@ -526,6 +607,8 @@ __device__ __forceinline__ void spmv_cta(const Mat& A, int64_t tr0, int64_t tr1,
             const int64_t sb = s0 + a;
             const int64_t tb_abs = t0 + w.ht[li];
             const uint32_t* cd = code + w.ht[li];
+            const int64_t i = (w0 + li) * 16 + lane;
+            const double ov = (own != nullptr && i < A.n_rows) ? own[i] : 0.0;
             double acc = 0.0;
             acc = slot_block<DYN, COUNT, PF>(A, w.pb, cur, min(W, PF), sb * 16 + lane, cd, staged, tb_abs, level,
                                               range_guard, x, acc, cnt);
@@ -537,7 +620,7 @@ __device__ __forceinline__ void spmv_cta(const Mat& A, int64_t tr0, int64_t tr1,
                 acc = slot_block<DYN, COUNT, PF>(A, w.pb, more, min(W - k, PF), (sb + k) * 16 + lane, cd, staged, tb_abs,
                                                   level, range_guard, x, acc, cnt);
             }
-            emit(w0 + li, lane, acc);
+            emit(w0 + li, lane, acc, ov);
         }
 #undef CMP_LOAD_FIRST
         w0 += nw;

@@ -75,8 +75,17 @@ struct TileMatrix {
     uint32_t* tile_info = nullptr;   // [tilenum] (TileColidx << 4) | (Floor << 2) | TilePrec
     int ts = 0;                      // 1: tile-synchronous slices
     uint16_t* sidx = nullptr;        // compact: [16*slots] (tile index in tile row << 4) | local column
-    uint8_t* sslot = nullptr;        // tile-synchronous: [16*slots] local column or 0xFF
-    uint32_t* colw = nullptr;        // tile-synchronous: [slots] (tile column << 4) | (Floor << 2) | TilePrec per slice column
+    uint8_t* sslot = nullptr;        // tile-synchronous: [16*slots] local column (0 on padding)
+    uint2* crec = nullptr;           // tile-synchronous: [slots] static column record (see kernels.cuh)
+    int64_t* tr_vb = nullptr;        // tile-synchronous: [ntr+1] value-byte start of each tile row in vstream
+    uint8_t* vstream = nullptr;      // tile-synchronous: values at TilePrec, 16*size(TilePrec) bytes per slice column
+    int64_t vbytes = 0;              // bytes of vstream
+    uint8_t* blob = nullptr;         // tile-synchronous: per-stage blobs streamed by the TMA pipeline
+    int64_t blob_bytes = 0;
+    void* stg = nullptr;             // tile-synchronous: mfk::PipeStage per stage of every CTA
+    int32_t* stg_ptr = nullptr;      // device [G+1]
+    int64_t nstg = 0;
+    // compact layout only: value planes RNE_q(stored value) per slot
     double* plane64 = nullptr;       // [16*slots] value at FP64 (tiles with TilePrec == FP64)
     float* plane32 = nullptr;        // value rounded to FP32 (tiles with TilePrec <= FP32)
     __half* plane16 = nullptr;       // ... FP16

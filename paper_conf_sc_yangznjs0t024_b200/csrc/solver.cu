@@ -239,6 +239,7 @@ __device__ __forceinline__ Smem carve(const SolveArgs& a, int nvec) {
     unsigned char* p = reinterpret_cast<unsigned char*>(s.timer + NPHASE + 1);
     p = reinterpret_cast<unsigned char*>((reinterpret_cast<uintptr_t>(p) + 15) & ~uintptr_t(15));
     mfk::carve_spmv(p, s.win, s.ts);
+    mfk::pipe_init(s.ts);      // ordered before the first SpMV by the caller's __syncthreads (Timer::start)
     p += mfk::SPMV_SMEM_BYTES;
     p = reinterpret_cast<unsigned char*>((reinterpret_cast<uintptr_t>(p) + 15) & ~uintptr_t(15));
     s.mu = reinterpret_cast<double*>(p);
@@ -298,11 +299,11 @@ __global__ void __launch_bounds__(MAXT, 1) cg_persistent(SolveArgs a) {
 
     // init: r = b - A~ x0 at TilePrec; p = r; partial (b,b), (r,r)
     double v2[2] = {0.0, 0.0};
-    mfk::spmv_cta<false, false, PF>(a.A, tr0, tr1, X, nullptr, 0, sm.win, sm.ts, nullptr, 0, -1,
-                                [&](int64_t TR, int ln, double ax) {
+    mfk::spmv_cta<false, false, PF>(a.A, tr0, tr1, X, nullptr, 0, sm.win, sm.ts, nullptr, 0, -1, a.b,
+                                [&](int64_t TR, int ln, double ax, double bi) {
                                     const int64_t i = TR * 16 + ln;
                                     if (i < n) {
-                                        const double bi = a.b[i], ri = __dsub_rn(bi, ax);
+                                        const double ri = __dsub_rn(bi, ax);
                                         Rv[i] = ri;
                                         P[i] = ri;
                                         v2[0] = __fma_rn(bi, bi, v2[0]);
@@ -338,13 +339,13 @@ __global__ void __launch_bounds__(MAXT, 1) cg_persistent(SolveArgs a) {
             tm.tick(0);
             // step A: mu = A~_j p_j (own tile rows) with the fused partial (mu, p)
             double sg[1] = {0.0};
-            mfk::spmv_cta<DYN, COUNT, PF>(a.A, tr0, tr1, P, a.lev_p, a.range_guard, sm.win, sm.ts, &cnt, a.seg_lo[blockIdx.x], a.seg_hi[blockIdx.x],
-                                      [&](int64_t TR, int ln, double mv) {
+            mfk::spmv_cta<DYN, COUNT, PF>(a.A, tr0, tr1, P, a.lev_p, a.range_guard, sm.win, sm.ts, &cnt, a.seg_lo[blockIdx.x], a.seg_hi[blockIdx.x], P,
+                                      [&](int64_t TR, int ln, double mv, double ov) {
                                           const int64_t i = TR * 16 + ln;
                                           if (i < n) {
                                               const int64_t li = i - R0;
                                               if (li < mu_cap) MUs[li] = mv; else MUg[i] = mv;
-                                              sg[0] = __fma_rn(mv, P[i], sg[0]);
+                                              sg[0] = __fma_rn(mv, ov, sg[0]);
                                           }
                                       });
             flush_counts<COUNT>(a, c, cnt, sm.ired);
@@ -452,11 +453,11 @@ __global__ void __launch_bounds__(MAXT, 1) bicgstab_persistent(SolveArgs a) {
 
     // init: r = b - A~ x0; r0* = r; p = r; partial (b,b), (r,r), (r,r0*)
     double v3[3] = {0.0, 0.0, 0.0};
-    mfk::spmv_cta<false, false, PF>(a.A, tr0, tr1, X, nullptr, 0, sm.win, sm.ts, nullptr, 0, -1,
-                                [&](int64_t TR, int ln, double ax) {
+    mfk::spmv_cta<false, false, PF>(a.A, tr0, tr1, X, nullptr, 0, sm.win, sm.ts, nullptr, 0, -1, a.b,
+                                [&](int64_t TR, int ln, double ax, double bi) {
                                     const int64_t i = TR * 16 + ln;
                                     if (i < n) {
-                                        const double bi = a.b[i], ri = __dsub_rn(bi, ax);
+                                        const double ri = __dsub_rn(bi, ax);
                                         Rv[i] = ri; a.rh[i] = ri; P[i] = ri;
                                         v3[0] = __fma_rn(bi, bi, v3[0]);
                                         v3[1] = __fma_rn(ri, ri, v3[1]);
@@ -493,10 +494,10 @@ __global__ void __launch_bounds__(MAXT, 1) bicgstab_persistent(SolveArgs a) {
             tm.tick(0);
             // mu = A~ p ; partial (mu, r0*)
             double eta[1] = {0.0};
-            mfk::spmv_cta<DYN, COUNT, PF>(a.A, tr0, tr1, P, a.lev_p, a.range_guard, sm.win, sm.ts, &cnt, a.seg_lo[blockIdx.x], a.seg_hi[blockIdx.x],
-                                      [&](int64_t TR, int ln, double mv) {
+            mfk::spmv_cta<DYN, COUNT, PF>(a.A, tr0, tr1, P, a.lev_p, a.range_guard, sm.win, sm.ts, &cnt, a.seg_lo[blockIdx.x], a.seg_hi[blockIdx.x], RH,
+                                      [&](int64_t TR, int ln, double mv, double ov) {
                                           const int64_t i = TR * 16 + ln;
-                                          if (i < n) { mu_at(i - R0) = mv; eta[0] = __fma_rn(mv, RH[i], eta[0]); }
+                                          if (i < n) { mu_at(i - R0) = mv; eta[0] = __fma_rn(mv, ov, eta[0]); }
                                       });
             flush_counts<COUNT>(a, c, cnt, sm.ired);
             __syncthreads();
@@ -521,13 +522,13 @@ __global__ void __launch_bounds__(MAXT, 1) bicgstab_persistent(SolveArgs a) {
             tm.tick(4);
             // theta = A~ s ; partial (theta, theta), (theta, s)
             double tt[2] = {0.0, 0.0};
-            mfk::spmv_cta<DYN, COUNT, PF>(a.A, tr0, tr1, S, a.lev_s, a.range_guard, sm.win, sm.ts, &cnt, a.seg_lo[blockIdx.x], a.seg_hi[blockIdx.x],
-                                      [&](int64_t TR, int ln, double tv) {
+            mfk::spmv_cta<DYN, COUNT, PF>(a.A, tr0, tr1, S, a.lev_s, a.range_guard, sm.win, sm.ts, &cnt, a.seg_lo[blockIdx.x], a.seg_hi[blockIdx.x], S,
+                                      [&](int64_t TR, int ln, double tv, double ov) {
                                           const int64_t i = TR * 16 + ln;
                                           if (i < n) {
                                               th_at(i - R0) = tv;
                                               tt[0] = __fma_rn(tv, tv, tt[0]);
-                                              tt[1] = __fma_rn(tv, S[i], tt[1]);
+                                              tt[1] = __fma_rn(tv, ov, tt[1]);
                                           }
                                       });
             flush_counts<COUNT>(a, c, cnt, sm.ired);
@@ -688,11 +689,11 @@ __global__ void __launch_bounds__(MAXT, 1) pcg_persistent(SolveArgs a) {
     (void)h;
 
     double v2[2] = {0.0, 0.0};
-    mfk::spmv_cta<false, false, PF>(a.A, tr0, tr1, X, nullptr, 0, sm.win, sm.ts, nullptr, 0, -1,
-                                    [&](int64_t TR, int ln, double ax) {
+    mfk::spmv_cta<false, false, PF>(a.A, tr0, tr1, X, nullptr, 0, sm.win, sm.ts, nullptr, 0, -1, a.b,
+                                    [&](int64_t TR, int ln, double ax, double bi) {
                                         const int64_t i = TR * 16 + ln;
                                         if (i < n) {
-                                            const double bi = a.b[i], ri = __dsub_rn(bi, ax);
+                                            const double ri = __dsub_rn(bi, ax);
                                             Rv[i] = ri;
                                             v2[0] = __fma_rn(bi, bi, v2[0]);
                                             v2[1] = __fma_rn(ri, ri, v2[1]);
@@ -731,13 +732,13 @@ __global__ void __launch_bounds__(MAXT, 1) pcg_persistent(SolveArgs a) {
             if (!wait_deps(a, (unsigned)(j + 1))) { status = MF_ERR_DEADLOCK; break; }
             tm.tick(0);
             double sg[1] = {0.0};
-            mfk::spmv_cta<DYN, COUNT, PF>(a.A, tr0, tr1, P, a.lev_p, a.range_guard, sm.win, sm.ts, &cnt, a.seg_lo[blockIdx.x], a.seg_hi[blockIdx.x],
-                                          [&](int64_t TR, int ln, double mv) {
+            mfk::spmv_cta<DYN, COUNT, PF>(a.A, tr0, tr1, P, a.lev_p, a.range_guard, sm.win, sm.ts, &cnt, a.seg_lo[blockIdx.x], a.seg_hi[blockIdx.x], P,
+                                          [&](int64_t TR, int ln, double mv, double ov) {
                                               const int64_t i = TR * 16 + ln;
                                               if (i < n) {
                                                   const int64_t li = i - R0;
                                                   if (li < mu_cap) MUs[li] = mv; else a.mu_g[i] = mv;
-                                                  sg[0] = __fma_rn(mv, P[i], sg[0]);
+                                                  sg[0] = __fma_rn(mv, ov, sg[0]);
                                               }
                                           });
             flush_counts<COUNT>(a, c, cnt, sm.ired);
@@ -821,11 +822,11 @@ __global__ void __launch_bounds__(MAXT, 1) pbicgstab_persistent(SolveArgs a) {
     auto th_at = [&](int64_t li) -> double& { return li < mu_cap ? THs[li] : a.th_g[R0 + li]; };
 
     double v3[3] = {0.0, 0.0, 0.0};
-    mfk::spmv_cta<false, false, PF>(a.A, tr0, tr1, X, nullptr, 0, sm.win, sm.ts, nullptr, 0, -1,
-                                    [&](int64_t TR, int ln, double ax) {
+    mfk::spmv_cta<false, false, PF>(a.A, tr0, tr1, X, nullptr, 0, sm.win, sm.ts, nullptr, 0, -1, a.b,
+                                    [&](int64_t TR, int ln, double ax, double bi) {
                                         const int64_t i = TR * 16 + ln;
                                         if (i < n) {
-                                            const double bi = a.b[i], ri = __dsub_rn(bi, ax);
+                                            const double ri = __dsub_rn(bi, ax);
                                             Rv[i] = ri; a.rh[i] = ri; P[i] = ri;
                                             v3[0] = __fma_rn(bi, bi, v3[0]);
                                             v3[1] = __fma_rn(ri, ri, v3[1]);
@@ -862,10 +863,10 @@ __global__ void __launch_bounds__(MAXT, 1) pbicgstab_persistent(SolveArgs a) {
             if (!wait_deps(a, epoch)) { status = MF_ERR_DEADLOCK; break; }
             tm.tick(0);
             double eta[1] = {0.0};
-            mfk::spmv_cta<DYN, COUNT, PF>(a.A, tr0, tr1, PH, a.lev_p, a.range_guard, sm.win, sm.ts, &cnt, a.seg_lo[blockIdx.x], a.seg_hi[blockIdx.x],
-                                          [&](int64_t TR, int ln, double mv) {
+            mfk::spmv_cta<DYN, COUNT, PF>(a.A, tr0, tr1, PH, a.lev_p, a.range_guard, sm.win, sm.ts, &cnt, a.seg_lo[blockIdx.x], a.seg_hi[blockIdx.x], RH,
+                                          [&](int64_t TR, int ln, double mv, double ov) {
                                               const int64_t i = TR * 16 + ln;
-                                              if (i < n) { mu_at(i - R0) = mv; eta[0] = __fma_rn(mv, RH[i], eta[0]); }
+                                              if (i < n) { mu_at(i - R0) = mv; eta[0] = __fma_rn(mv, ov, eta[0]); }
                                           });
             flush_counts<COUNT>(a, c, cnt, sm.ired);
             __syncthreads();
@@ -886,13 +887,13 @@ __global__ void __launch_bounds__(MAXT, 1) pbicgstab_persistent(SolveArgs a) {
             if (!wait_deps(a, epoch)) { status = MF_ERR_DEADLOCK; break; }
             tm.tick(4);
             double tt[2] = {0.0, 0.0};
-            mfk::spmv_cta<DYN, COUNT, PF>(a.A, tr0, tr1, SH, a.lev_s, a.range_guard, sm.win, sm.ts, &cnt, a.seg_lo[blockIdx.x], a.seg_hi[blockIdx.x],
-                                          [&](int64_t TR, int ln, double tv) {
+            mfk::spmv_cta<DYN, COUNT, PF>(a.A, tr0, tr1, SH, a.lev_s, a.range_guard, sm.win, sm.ts, &cnt, a.seg_lo[blockIdx.x], a.seg_hi[blockIdx.x], S,
+                                          [&](int64_t TR, int ln, double tv, double ov) {
                                               const int64_t i = TR * 16 + ln;
                                               if (i < n) {
                                                   th_at(i - R0) = tv;
                                                   tt[0] = __fma_rn(tv, tv, tt[0]);
-                                                  tt[1] = __fma_rn(tv, S[i], tt[1]);
+                                                  tt[1] = __fma_rn(tv, ov, tt[1]);
                                               }
                                           });
             flush_counts<COUNT>(a, c, cnt, sm.ired);
@@ -969,13 +970,15 @@ __global__ void __launch_bounds__(1024) spmv_kernel(Mat A, const int32_t* __rest
     mfk::WinSmem w;
     mfk::TsSmem tsm;
     mfk::carve_spmv(smem_raw + 64, w, tsm);
+    mfk::pipe_init(tsm);
+    __syncthreads();
     Counts cnt;
     cnt.zero();
     if (COUNT && threadIdx.x < 10) ired[threadIdx.x] = 0;
     const int64_t tr0 = plan_tr[blockIdx.x], tr1 = plan_tr[blockIdx.x + 1];
     const int64_t n = A.n_rows;
-    mfk::spmv_cta<DYN, COUNT, 4>(A, tr0, tr1, x, level, range_guard, w, tsm, &cnt, seg_lo[blockIdx.x], seg_hi[blockIdx.x],
-                                 [&](int64_t TR, int ln, double v) {
+    mfk::spmv_cta<DYN, COUNT, 4>(A, tr0, tr1, x, level, range_guard, w, tsm, &cnt, seg_lo[blockIdx.x], seg_hi[blockIdx.x], nullptr,
+                                 [&](int64_t TR, int ln, double v, double) {
         const int64_t i = TR * 16 + ln;
         if (i < n) y[i] = v;
     });
@@ -1038,7 +1041,8 @@ void* pick_kernel(bool bicg, bool dyn, bool count, bool pre) {
 }
 
 Mat mat_view(const TileMatrix& A) {
-    return Mat{A.n_rows, A.n_cols, A.ntr, A.tr_slot, A.TileRowPtr, A.tile_info, A.sidx, A.sslot, A.colw, A.ts, (int)A.max_w,
+    return Mat{A.n_rows, A.n_cols, A.ntr, A.tr_slot, A.TileRowPtr, A.tile_info, A.sidx, A.blob,
+               reinterpret_cast<const mfk::PipeStage*>(A.stg), A.stg_ptr, A.TileNnz, A.ts, (int)A.max_w,
                A.plane64, A.plane32, A.plane16, A.plane8};
 }
 
@@ -1132,6 +1136,9 @@ mf_status run_solve(const TileMatrix& A, bool bicg, const double* b, double* x, 
     (void)H;
     int64_t cap = ((int64_t)smem_optin - (int64_t)fixed - 64) / (8 * nvec);
     cap = std::max<int64_t>(0, std::min(cap, max_rows));
+    // the TMA pipeline (tile-synchronous layout) spends shared memory on stages in flight; the SpMV
+    // outputs then live in global memory (L2-resident: the matrix streams with evict_first)
+    if (A.ts) cap = 0;
     if (const char* ev = getenv("MF_MU_ONCHIP")) if (atoi(ev) == 0) cap = 0;   // tuning: trade smem for L1
     const size_t pre_smem = pre ? (size_t)B * 12 + 32 : 0;
     cap = std::max<int64_t>(0, std::min<int64_t>(cap, ((int64_t)smem_optin - (int64_t)fixed - (int64_t)pre_smem - 64) / (8 * nvec)));
@@ -1258,7 +1265,12 @@ mf_status run_solve(const TileMatrix& A, bool bicg, const double* b, double* x, 
     // vectors: CG 48n per iteration (read p,x,r; write x,r,p); BiCGSTAB 72n (read p,x,r,r0*,s;
     // write s,x,r,p); + 16n per SpMV output that cannot stay on chip (capacity rule)
     const double vec = bicg ? 72.0 : 48.0;
-    const double spill_b = spill ? (bicg ? 32.0 : 16.0) : 0.0;
+    // capacity rule: the SpMV outputs count as HBM traffic only when they cannot fit
+    // the GPU's shared memory, whatever this launch chose to do with them
+    int smem_sm = 0;
+    MF_CUDA(cudaDeviceGetAttribute(&smem_sm, cudaDevAttrMaxSharedMemoryPerMultiprocessor, dev));
+    const bool over_cap = 8.0 * (double)n * (double)nvec > (double)sms * (double)smem_sm;
+    const double spill_b = over_cap ? (bicg ? 32.0 : 16.0) : 0.0;
     info->model_bytes = model + (vec + spill_b) * (double)n * (double)iters;
     if (pre) {   // per apply: L and U values + column indices, row pointers, the vectors in/y/out
         const double apply_b = 12.0 * (double)(P->nnz_l + P->nnz_u) + 16.0 * (double)n + 8.0 * n + 32.0 * (double)n;
