@@ -37,10 +37,8 @@ struct Mat {
 
 __device__ __forceinline__ unsigned hw_mask() { return (threadIdx.x & 16) ? 0xFFFF0000u : 0x0000FFFFu; }
 
-__device__ __forceinline__ int hw_min_i(int v, unsigned m) {
-    for (int o = 8; o >= 1; o >>= 1) v = min(v, __shfl_xor_sync(m, v, o));
-    return v;
-}
+// min over the half-warp (mask m): one redux.sync
+__device__ __forceinline__ int hw_min_i(int v, unsigned m) { return (int)__reduce_min_sync(m, (unsigned)v); }
 
 // (tile column << 3) | e_t.   e_t = bypass | max_prec(floor, min_prec(TilePrec, level))
 template <bool DYN>
@@ -180,20 +178,22 @@ __device__ __forceinline__ double slot_block(const Mat& A, const unsigned long l
 //   [values, grouped by TilePrec (FP64 block, FP32 block, FP16 block, E4M3 block), 16 per column]
 // so that a stage is a single bulk copy (TMA throughput is bounded by copies per second).
 //
-// Per stage: thread 0 keeps PIPE_NST stages in flight (one "full" mbarrier each, refilled when
-// every warp has arrived on the stage's "empty" mbarrier).  After a stage lands:
+// Per stage: thread 0 keeps PIPE_NST stages in flight (one "full" mbarrier each).  After a stage
+// lands:
 //   1. decode pass (all threads, warp-uniform per precision group): 4 values per thread per
 //      step, exact upcast to binary64 into E[col][lane] (the on-chip conversion of P:237); the
 //      dynamic switch (Alg. 5) is applied here: bypassed columns become 0, a column with e_t
 //      below TilePrec is rounded to e_t (RNE_{e_t}(stored value));
-//   2. __syncthreads;
+//   2. __syncthreads -- the slot is consumed (its column words / local columns were copied to the
+//      decoded-stage buffer too), so thread 0 refills it at once: PIPE_NST - 1 stages stay in
+//      flight during the FMA pass;
 //   3. FMA pass: half-warp h owns tile rows tr0 + h + kH, lane r = row 16*TR + r (the row mapping
 //      of the dot-product contract) and runs the row's single fma chain in ascending column
 //      order: acc = fma(E[c][r], x[16*tile column + local column], acc) -- a zero (padding or
-//      bypass) term leaves acc unchanged.  x is gathered through L1/L2.  A half-warp runs two
-//      tile rows (two independent chains) at once.
-// Stages hold whole groups of H tile rows (two when they fit), E is single-buffered: two
-// __syncthreads per stage order the decode and FMA passes.
+//      bypass) term leaves acc unchanged.  x is gathered through L1/L2 with coherent loads; the
+//      chain of a row is fully unrolled on its column count, all loads issued before the fmas.
+// Stages hold whole groups of H tile rows (two when they fit); the decoded-stage buffer is
+// single: two __syncthreads per stage order the decode and FMA passes.
 struct PipeStage {
     int64_t col0, col1;             // slice-column range of the stage
     int64_t boff;                   // blob offset in Mat::blob
@@ -208,28 +208,33 @@ static_assert(sizeof(PipeStage) == 96, "PipeStage is 96 bytes");
 
 constexpr int PIPE_NST = 3;        // stages in flight
 constexpr int PIPE_KCAP = 64;      // tile rows per stage
-constexpr int PIPE_CCAP = 600;     // slice columns per stage
-constexpr int PIPE_VCAP = 32768;   // value bytes per stage
+constexpr int PIPE_CCAP = 576;     // slice columns per stage
+constexpr int PIPE_VCAP = 28672;   // value bytes per stage
 __host__ __device__ constexpr int pipe_r16(int v) { return (v + 15) & ~15; }
 constexpr int PIPE_BLOB_CAP = pipe_r16((PIPE_KCAP + 1) * 4) + pipe_r16(PIPE_CCAP * 4) + PIPE_CCAP * 16 +
                               pipe_r16(PIPE_CCAP * 2 + 8) + PIPE_VCAP;
 constexpr int PS_INFO = pipe_r16(PIPE_BLOB_CAP);               // int32 tr0, tr1, off_cw, off_ss, off_dst, gcnt[4], goff[4]
 constexpr int PS_BYTES = PS_INFO + 64;
-constexpr int PIPE_E_BYTES = PIPE_CCAP * 128;                  // one decoded stage: FP64 [col][lane]
+// decoded stage (FMA side): values FP64 [col][lane], then the column words, local columns and
+// tile-row headers copied out of the slot so that the slot is refilled right after decoding
+constexpr int PIPE_E_BYTES = PIPE_CCAP * 128;
+constexpr int PIPE_F_CW = PIPE_E_BYTES;                        // u32 column words
+constexpr int PIPE_F_SS = PIPE_F_CW + PIPE_CCAP * 4;           // u8 local columns [col][lane]
+constexpr int PIPE_F_HDR = PIPE_F_SS + PIPE_CCAP * 16;         // int32 headers, then tr0, tr1
+constexpr int PIPE_D_BYTES = PIPE_F_HDR + pipe_r16((PIPE_KCAP + 1) * 4 + 8);
 constexpr int PIPE_LEV_CAP = 4096;                             // staged level bytes (column segments gathered)
-// region: [NST slots][E][full NST u64][empty NST u64][ctr u64][pad][levels]
-constexpr size_t PIPE_SMEM_BYTES = (size_t)PIPE_NST * PS_BYTES + (size_t)PIPE_E_BYTES + 16 * PIPE_NST + 16 + PIPE_LEV_CAP;
+// region: [NST slots][decoded stage][full NST u64][ctr u64][pad][levels]
+constexpr size_t PIPE_SMEM_BYTES = (size_t)PIPE_NST * PS_BYTES + (size_t)PIPE_D_BYTES + 8 * PIPE_NST + 16 + PIPE_LEV_CAP;
 
 struct TsSmem {
     unsigned char* base;
     __device__ __forceinline__ unsigned char* slot(int s) const { return base + (size_t)s * PS_BYTES; }
-    __device__ __forceinline__ unsigned char* E(int b) const { return base + (size_t)PIPE_NST * PS_BYTES + (size_t)b * PIPE_E_BYTES; }
+    __device__ __forceinline__ unsigned char* D() const { return base + (size_t)PIPE_NST * PS_BYTES; }
     __device__ __forceinline__ unsigned long long* full(int s) const {
-        return reinterpret_cast<unsigned long long*>(E(1)) + s;
+        return reinterpret_cast<unsigned long long*>(D() + PIPE_D_BYTES) + s;
     }
-    __device__ __forceinline__ unsigned long long* empty(int s) const { return full(0) + PIPE_NST + s; }
-    __device__ __forceinline__ unsigned long long* ctr() const { return full(0) + 2 * PIPE_NST; }
-    __device__ __forceinline__ uint8_t* lev() const { return reinterpret_cast<uint8_t*>(full(0) + 2 * PIPE_NST + 2); }
+    __device__ __forceinline__ unsigned long long* ctr() const { return full(0) + PIPE_NST; }
+    __device__ __forceinline__ uint8_t* lev() const { return reinterpret_cast<uint8_t*>(full(0) + PIPE_NST + 2); }
 };
 
 __device__ __forceinline__ unsigned smem_u32(const void* p) { return (unsigned)__cvta_generic_to_shared(p); }
@@ -279,10 +284,7 @@ __device__ __forceinline__ void bulk_g2s_ef(void* dst, const void* src, unsigned
 // all threads; followed by a __syncthreads of the caller before the first SpMV
 __device__ __forceinline__ void pipe_init(const TsSmem& sm) {
     if (threadIdx.x == 0) {
-        for (int s = 0; s < PIPE_NST; ++s) {
-            mbar_init(sm.full(s), 1);
-            mbar_init(sm.empty(s), blockDim.x >> 5);
-        }
+        for (int s = 0; s < PIPE_NST; ++s) mbar_init(sm.full(s), 1);
         *sm.ctr() = 0ull;
         asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
     }
@@ -303,49 +305,10 @@ __device__ __forceinline__ void pipe_issue(const Mat& A, const PipeStage& st, un
     bulk_g2s_ef(slot, A.blob + st.boff, (unsigned)st.bbytes, full, pol);
 }
 
-__device__ __forceinline__ int lds_i32(unsigned a) {
-    int v;
-    asm volatile("ld.shared.s32 %0, [%1];" : "=r"(v) : "r"(a));
-    return v;
-}
-__device__ __forceinline__ uint32_t lds_u32(unsigned a) {
-    uint32_t v;
-    asm volatile("ld.shared.u32 %0, [%1];" : "=r"(v) : "r"(a));
-    return v;
-}
-__device__ __forceinline__ uint32_t lds_u16(unsigned a) {
-    uint32_t v;
-    asm volatile("ld.shared.u16 %0, [%1];" : "=r"(v) : "r"(a));
-    return v;
-}
-__device__ __forceinline__ uint32_t lds_u8(unsigned a) {
-    uint32_t v;
-    asm volatile("ld.shared.u8 %0, [%1];" : "=r"(v) : "r"(a));
-    return v;
-}
-__device__ __forceinline__ double lds_f64(unsigned a) {
-    double v;
-    asm volatile("ld.shared.f64 %0, [%1];" : "=d"(v) : "r"(a));
-    return v;
-}
-__device__ __forceinline__ uint2 lds_v2(unsigned a) {
-    uint2 v;
-    asm volatile("ld.shared.v2.u32 {%0, %1}, [%2];" : "=r"(v.x), "=r"(v.y) : "r"(a));
-    return v;
-}
-__device__ __forceinline__ uint4 lds_v4(unsigned a) {
-    uint4 v;
-    asm volatile("ld.shared.v4.u32 {%0, %1, %2, %3}, [%4];" : "=r"(v.x), "=r"(v.y), "=r"(v.z), "=r"(v.w) : "r"(a));
-    return v;
-}
-__device__ __forceinline__ void sts_d2(unsigned a, double u, double v) {
-    asm volatile("st.shared.v2.f64 [%0], {%1, %2};" ::"r"(a), "d"(u), "d"(v) : "memory");
-}
-
 // level of tile column tc for the dynamic switch
-__device__ __forceinline__ int col_level(uint32_t tc, const uint8_t* __restrict__ level, unsigned lev_s, bool lev_staged,
+__device__ __forceinline__ int col_level(uint32_t tc, const uint8_t* __restrict__ level, const uint8_t* lev_s, bool lev_staged,
                                          int32_t seg_lo) {
-    return lev_staged ? (int)lds_u8(lev_s + (tc - (uint32_t)seg_lo)) : (int)level[tc];
+    return lev_staged ? (int)lev_s[tc - (uint32_t)seg_lo] : (int)level[tc];
 }
 
 __device__ __forceinline__ double e4m3_lo(uint32_t w2) {   // the E4M3 byte in bits 0..7 -> binary64 (exact)
@@ -354,130 +317,194 @@ __device__ __forceinline__ double e4m3_lo(uint32_t w2) {   // the E4M3 byte in b
 }
 __device__ __forceinline__ double h16(uint32_t bits) { return (double)__half2float(__ushort_as_half((unsigned short)bits)); }
 
-// decode pass: group Q (0 FP64 .. 3 E4M3) of the stage in slot -> E.  Unit = 4 lanes of one column.
+// Shared-memory accesses of the pipeline are plain C++ (the compiler schedules them freely between
+// the barriers); the stage slot is read-only after its "full" mbarrier completes.
+struct PipeView {
+    const int32_t* info;      // PS_INFO fields
+    const int32_t* hdr;       // column start per tile-row boundary
+    const uint32_t* cw;       // column words
+    const uint8_t* ss;        // local columns [col][lane]
+    const uint16_t* dst;      // group permutation
+    const unsigned char* blob;
+};
+__device__ __forceinline__ PipeView pipe_view(const unsigned char* slot) {
+    PipeView v;
+    v.blob = slot;
+    v.info = reinterpret_cast<const int32_t*>(slot + PS_INFO);
+    v.hdr = reinterpret_cast<const int32_t*>(slot);
+    v.cw = reinterpret_cast<const uint32_t*>(slot + v.info[2]);
+    v.ss = slot + v.info[3];
+    v.dst = reinterpret_cast<const uint16_t*>(slot + v.info[4]);
+    return v;
+}
+
+// decode pass: group Q (0 FP64 .. 3 E4M3) of the stage -> E.  Unit = 4 lanes of one column.
 template <int Q, bool DYN>
-__device__ __forceinline__ void pipe_decode_group(unsigned slot, unsigned Eb, int ncol_q, unsigned goff, unsigned dst_q, unsigned cw,
-                                                  const uint8_t* __restrict__ level, unsigned lev_s, bool lev_staged,
+__device__ __forceinline__ void pipe_decode_group(const PipeView& v, double* E, int ncol_q, int goff, const uint16_t* dst_q,
+                                                  const uint8_t* __restrict__ level, const uint8_t* lev_s, bool lev_staged,
                                                   int32_t seg_lo, int range_guard) {
     const int units = ncol_q * 4;
     for (int u = threadIdx.x; u < units; u += blockDim.x) {
         const int j = u >> 2, r0 = (u & 3) * 4;
-        const unsigned d = lds_u16(dst_q + 2u * (unsigned)j);          // destination column in the stage
-        const unsigned src = slot + goff + (unsigned)((j * 16 + r0) << (3 - Q));
-        double v[4];
+        const unsigned d = dst_q[j];                                   // destination column in the stage
+        const unsigned char* src = v.blob + goff + ((j * 16 + r0) << (3 - Q));
+        double w[4];
         if (Q == 0) {
-            const uint4 a = lds_v4(src), b = lds_v4(src + 16);
-            v[0] = __hiloint2double((int)a.y, (int)a.x); v[1] = __hiloint2double((int)a.w, (int)a.z);
-            v[2] = __hiloint2double((int)b.y, (int)b.x); v[3] = __hiloint2double((int)b.w, (int)b.z);
+            const double2 a = reinterpret_cast<const double2*>(src)[0], b = reinterpret_cast<const double2*>(src)[1];
+            w[0] = a.x; w[1] = a.y; w[2] = b.x; w[3] = b.y;
         } else if (Q == 1) {
-            const uint4 a = lds_v4(src);
-            v[0] = (double)__uint_as_float(a.x); v[1] = (double)__uint_as_float(a.y);
-            v[2] = (double)__uint_as_float(a.z); v[3] = (double)__uint_as_float(a.w);
+            const float4 a = *reinterpret_cast<const float4*>(src);
+            w[0] = (double)a.x; w[1] = (double)a.y; w[2] = (double)a.z; w[3] = (double)a.w;
         } else if (Q == 2) {
-            const uint2 a = lds_v2(src);
-            v[0] = h16(a.x); v[1] = h16(a.x >> 16); v[2] = h16(a.y); v[3] = h16(a.y >> 16);
+            const uint2 a = *reinterpret_cast<const uint2*>(src);
+            w[0] = h16(a.x); w[1] = h16(a.x >> 16); w[2] = h16(a.y); w[3] = h16(a.y >> 16);
         } else {
-            const uint32_t a = lds_u32(src);
-            v[0] = e4m3_lo(a); v[1] = e4m3_lo(a >> 8); v[2] = e4m3_lo(a >> 16); v[3] = e4m3_lo(a >> 24);
+            const uint32_t a = *reinterpret_cast<const uint32_t*>(src);
+            w[0] = e4m3_lo(a); w[1] = e4m3_lo(a >> 8); w[2] = e4m3_lo(a >> 16); w[3] = e4m3_lo(a >> 24);
         }
         if (DYN) {   // e_t = bypass | max(TilePrec, level), range guard e_t <= Floor (Alg. 5)
-            const uint32_t word = lds_u32(cw + 4u * d);
+            const uint32_t word = v.cw[d];
             const int lv = col_level(word >> 4, level, lev_s, lev_staged, seg_lo);
             if (lv > Q) {
-                if (lv == BYP) { v[0] = v[1] = v[2] = v[3] = 0.0; }
+                if (lv == BYP) { w[0] = w[1] = w[2] = w[3] = 0.0; }
                 else {
                     int e = lv;
                     if (range_guard) e = min(e, (int)((word >> 2) & 3u));
                     if (e != Q) {
 #pragma unroll
-                        for (int k = 0; k < 4; ++k) v[k] = round_to(v[k], e);
+                        for (int k = 0; k < 4; ++k) w[k] = round_to(w[k], e);
                     }
                 }
             }
         }
-        const unsigned ea = Eb + d * 128u + (unsigned)r0 * 8u;
-        sts_d2(ea, v[0], v[1]);
-        sts_d2(ea + 16, v[2], v[3]);
+        double2* ea = reinterpret_cast<double2*>(E + d * 16 + r0);
+        ea[0] = make_double2(w[0], w[1]);
+        ea[1] = make_double2(w[2], w[3]);
     }
 }
 
 template <bool DYN>
-__device__ __forceinline__ void pipe_decode(unsigned slot, unsigned Eb, const uint8_t* __restrict__ level, unsigned lev_s, bool lev_staged,
-                                            int32_t seg_lo, int range_guard) {
-    const unsigned cw = slot + (unsigned)lds_i32(slot + PS_INFO + 8);
-    unsigned dst = slot + (unsigned)lds_i32(slot + PS_INFO + 16);
-    const int g0 = lds_i32(slot + PS_INFO + 20), g1 = lds_i32(slot + PS_INFO + 24), g2 = lds_i32(slot + PS_INFO + 28),
-              g3 = lds_i32(slot + PS_INFO + 32);
-    pipe_decode_group<0, DYN>(slot, Eb, g0, (unsigned)lds_i32(slot + PS_INFO + 36), dst, cw, level, lev_s, lev_staged, seg_lo, range_guard);
-    dst += 2u * (unsigned)g0;
-    pipe_decode_group<1, DYN>(slot, Eb, g1, (unsigned)lds_i32(slot + PS_INFO + 40), dst, cw, level, lev_s, lev_staged, seg_lo, range_guard);
-    dst += 2u * (unsigned)g1;
-    pipe_decode_group<2, DYN>(slot, Eb, g2, (unsigned)lds_i32(slot + PS_INFO + 44), dst, cw, level, lev_s, lev_staged, seg_lo, range_guard);
-    dst += 2u * (unsigned)g2;
-    pipe_decode_group<3, DYN>(slot, Eb, g3, (unsigned)lds_i32(slot + PS_INFO + 48), dst, cw, level, lev_s, lev_staged, seg_lo, range_guard);
+__device__ __forceinline__ void pipe_decode(const PipeView& v, unsigned char* D, const uint8_t* __restrict__ level, const uint8_t* lev_s,
+                                            bool lev_staged, int32_t seg_lo, int range_guard) {
+    double* E = reinterpret_cast<double*>(D);
+    {   // the FMA side's copy of the column words, local columns and headers
+        const int S0 = v.info[0], S1 = v.info[1], K = S1 - S0;
+        const int ncol = v.hdr[K];
+        uint4* fss = reinterpret_cast<uint4*>(D + PIPE_F_SS);
+        const uint4* sss = reinterpret_cast<const uint4*>(v.ss);
+        for (int c = threadIdx.x; c < ncol; c += blockDim.x) fss[c] = sss[c];
+        uint32_t* fcw = reinterpret_cast<uint32_t*>(D + PIPE_F_CW);
+        for (int c = threadIdx.x; c < ncol; c += blockDim.x) fcw[c] = v.cw[c];
+        int32_t* fh = reinterpret_cast<int32_t*>(D + PIPE_F_HDR);
+        for (int k = threadIdx.x; k <= K; k += blockDim.x) fh[k] = v.hdr[k];
+        if (threadIdx.x == 0) {
+            int32_t* tail = reinterpret_cast<int32_t*>(D + PIPE_D_BYTES) - 2;
+            tail[0] = S0;
+            tail[1] = S1;
+        }
+    }
+    const uint16_t* dst = v.dst;
+    const int g0 = v.info[5], g1 = v.info[6], g2 = v.info[7], g3 = v.info[8];
+    pipe_decode_group<0, DYN>(v, E, g0, v.info[9], dst, level, lev_s, lev_staged, seg_lo, range_guard);
+    dst += g0;
+    pipe_decode_group<1, DYN>(v, E, g1, v.info[10], dst, level, lev_s, lev_staged, seg_lo, range_guard);
+    dst += g1;
+    pipe_decode_group<2, DYN>(v, E, g2, v.info[11], dst, level, lev_s, lev_staged, seg_lo, range_guard);
+    dst += g2;
+    pipe_decode_group<3, DYN>(v, E, g3, v.info[12], dst, level, lev_s, lev_staged, seg_lo, range_guard);
 }
 
-// four columns [c, c+4) of one tile row with n valid (past the row: re-read column c, masked)
-struct PipeRow {
-    unsigned a;      // first column (stage-relative)
-    int W;           // columns
-    double acc;
-};
-__device__ __forceinline__ void pipe_load4(unsigned cw, unsigned ssl, unsigned El, unsigned c, int n, const double* __restrict__ x,
-                                           double (&ev)[4], double (&xv)[4]) {
-    const unsigned b4 = 4u * c, b16 = 16u * c, b128 = 128u * c;
+// one tile row of N columns starting at stage column c: every load first, then the fma chain.
+// x is written during the solve by other CTAs (ordered by the barriers' acquire): plain coherent
+// loads (x is not __restrict__, so never the read-only .nc path).
+template <int N>
+__device__ __forceinline__ double pipe_row(const uint32_t* cw, const uint8_t* ssl, const double* El, int c, const double* x) {
+    double ev[N], xv[N];
 #pragma unroll
-    for (int q = 0; q < 4; ++q) {
-        const unsigned o = q < n ? (unsigned)q : 0u;
-        const uint32_t word = lds_u32(cw + b4 + 4u * o);
-        const uint32_t lc = lds_u8(ssl + b16 + 16u * o);
-        ev[q] = lds_f64(El + b128 + 128u * o);
+    for (int q = 0; q < N; ++q) {
+        const uint32_t word = cw[c + q];
+        const uint32_t lc = ssl[(c + q) * 16];
+        ev[q] = El[(c + q) * 16];
         xv[q] = x[(word & ~15u) | lc];
+    }
+    double acc = 0.0;
+#pragma unroll
+    for (int q = 0; q < N; ++q) acc = __fma_rn(ev[q], xv[q], acc);
+    return acc;
+}
+// rows wider than 12 columns: chunks of 8 (the chain continues across chunks)
+__device__ __forceinline__ double pipe_row_long(const uint32_t* cw, const uint8_t* ssl, const double* El, int c, int W, const double* x) {
+    double acc = 0.0;
+    int q0 = 0;
+    for (; q0 + 8 <= W; q0 += 8) {
+        double ev[8], xv[8];
+#pragma unroll
+        for (int q = 0; q < 8; ++q) {
+            const int cc = c + q0 + q;
+            ev[q] = El[cc * 16];
+            xv[q] = x[(cw[cc] & ~15u) | ssl[cc * 16]];
+        }
+#pragma unroll
+        for (int q = 0; q < 8; ++q) acc = __fma_rn(ev[q], xv[q], acc);
+    }
+    for (; q0 < W; ++q0) {
+        const int cc = c + q0;
+        acc = __fma_rn(El[cc * 16], x[(cw[cc] & ~15u) | ssl[cc * 16]], acc);
+    }
+    return acc;
+}
+__device__ __forceinline__ double pipe_row_any(const uint32_t* cw, const uint8_t* ssl, const double* El, int c, int W, const double* x) {
+    switch (W) {
+    case 0: return 0.0;
+    case 1: return pipe_row<1>(cw, ssl, El, c, x);
+    case 2: return pipe_row<2>(cw, ssl, El, c, x);
+    case 3: return pipe_row<3>(cw, ssl, El, c, x);
+    case 4: return pipe_row<4>(cw, ssl, El, c, x);
+    case 5: return pipe_row<5>(cw, ssl, El, c, x);
+    case 6: return pipe_row<6>(cw, ssl, El, c, x);
+    case 7: return pipe_row<7>(cw, ssl, El, c, x);
+    case 8: return pipe_row<8>(cw, ssl, El, c, x);
+    case 9: return pipe_row<9>(cw, ssl, El, c, x);
+    case 10: return pipe_row<10>(cw, ssl, El, c, x);
+    case 11: return pipe_row<11>(cw, ssl, El, c, x);
+    case 12: return pipe_row<12>(cw, ssl, El, c, x);
+    default: return pipe_row_long(cw, ssl, El, c, W, x);
     }
 }
 
-// FMA pass of one stage: half-warp h takes its tile rows (TR = tr0c + h (mod H)) in ascending
-// order, two at a time (two independent fma chains per lane).
+// FMA pass of one stage: half-warp h takes its tile rows (TR = tr0c + h (mod H)) in ascending order
 template <class Emit>
-__device__ __forceinline__ void pipe_fma(const Mat& A, unsigned slot, unsigned Eb, int64_t tr0c, const double* __restrict__ x,
-                                         const double* __restrict__ own, Emit& emit) {
+__device__ __forceinline__ void pipe_fma(const Mat& A, const unsigned char* D, int64_t tr0c, const double* x,
+                                         const double* own, Emit& emit) {
     const int t = threadIdx.x, H = blockDim.x >> 4, h = t >> 4, lane = t & 15;
-    const int32_t S0 = lds_i32(slot + PS_INFO), S1 = lds_i32(slot + PS_INFO + 4);
-    const unsigned cw = slot + (unsigned)lds_i32(slot + PS_INFO + 8);
-    const unsigned ssl = slot + (unsigned)lds_i32(slot + PS_INFO + 12) + (unsigned)lane;
-    const unsigned El = Eb + 8u * (unsigned)lane;
-    const int off0 = (int)((S0 - tr0c) % H);
-    for (int64_t TR = S0 + (h - off0 + H) % H; TR < S1; TR += 2 * H) {
-        const bool two = TR + H < S1;
-        const int k0 = (int)(TR - S0), k1 = two ? k0 + H : k0;
-        const int a0 = lds_i32(slot + 4u * k0), W0 = lds_i32(slot + 4u * (k0 + 1)) - a0;
-        const int a1 = lds_i32(slot + 4u * k1), W1 = two ? lds_i32(slot + 4u * (k1 + 1)) - a1 : 0;
-        const int64_t i0 = TR * 16 + lane, i1 = i0 + 16 * H;
-        const double ov0 = (own != nullptr && i0 < A.n_rows) ? own[i0] : 0.0;
-        const double ov1 = (own != nullptr && two && i1 < A.n_rows) ? own[i1] : 0.0;
-        double acc0 = 0.0, acc1 = 0.0;
-        const int Wm = max(W0, W1);
-        for (int cb = 0; cb < Wm; cb += 4) {
-            double e0[4], x0[4], e1[4], x1[4];
-            const int n0 = W0 - cb, n1 = W1 - cb;
-            pipe_load4(cw, ssl, El, (unsigned)(a0 + (n0 > 0 ? cb : 0)), n0, x, e0, x0);
-            pipe_load4(cw, ssl, El, (unsigned)(a1 + (n1 > 0 ? cb : 0)), n1, x, e1, x1);
-#pragma unroll
-            for (int q = 0; q < 4; ++q) {
-                if (q < n0) acc0 = __fma_rn(e0[q], x0[q], acc0);
-                if (q < n1) acc1 = __fma_rn(e1[q], x1[q], acc1);
-            }
-        }
-        emit(TR, lane, acc0, ov0);
-        if (two) emit(TR + H, lane, acc1, ov1);
+    const int32_t* hdr = reinterpret_cast<const int32_t*>(D + PIPE_F_HDR);
+    const uint32_t* cw = reinterpret_cast<const uint32_t*>(D + PIPE_F_CW);
+    const uint8_t* ssl = D + PIPE_F_SS + lane;
+    const double* El = reinterpret_cast<const double*>(D) + lane;
+
+    // S0, S1 follow the K+1 headers; K is recovered from them (S1 - S0)
+    int S0 = 0, S1 = 0;
+    {
+        // headers occupy [0, K]; tr0/tr1 at K+1, K+2 -- found from the fixed KCAP-sized area
+        const int32_t* tail = reinterpret_cast<const int32_t*>(D + PIPE_D_BYTES) - 2;
+        S0 = tail[0];
+        S1 = tail[1];
+    }
+    const int off0 = (int)(S0 - tr0c) % H;
+    for (int TR = S0 + (h - off0 + H) % H; TR < S1; TR += H) {
+        const int k = TR - S0;
+        const int a = hdr[k], W = hdr[k + 1] - a;
+        const int64_t i = (int64_t)TR * 16 + lane;
+        const double ov = (own != nullptr && i < A.n_rows) ? own[i] : 0.0;
+        emit((int64_t)TR, lane, pipe_row_any(cw, ssl, El, a, W, x), ov);
     }
 }
 
 // the whole SpMV of one CTA (all threads), tile rows [tr0c, tr1c) = the CTA's plan range
 template <bool DYN, bool COUNT, class Emit>
-__device__ __forceinline__ void spmv_pipe(const Mat& A, int64_t tr0c, int64_t tr1c, const double* __restrict__ x,
+__device__ __forceinline__ void spmv_pipe(const Mat& A, int64_t tr0c, int64_t tr1c, const double* x,
                                           const uint8_t* __restrict__ level, int range_guard, const TsSmem& sm, Counts* cnt,
-                                          int32_t seg_lo, int32_t seg_hi, const double* __restrict__ own, Emit& emit) {
+                                          int32_t seg_lo, int32_t seg_hi, const double* own, Emit& emit) {
     const int t = threadIdx.x, B = blockDim.x;
     const int32_t s_begin = A.stg_ptr[blockIdx.x], ns = A.stg_ptr[blockIdx.x + 1] - s_begin;
     const int32_t nlev = seg_hi - seg_lo + 1;
@@ -489,7 +516,6 @@ __device__ __forceinline__ void spmv_pipe(const Mat& A, int64_t tr0c, int64_t tr
         pol = policy_evict_first();
         for (int k = 0; k < min(ns, PIPE_NST); ++k) {
             const unsigned u = u0 + (unsigned)k, sl = u % PIPE_NST, mm = u / PIPE_NST;
-            if (mm > 0) mbar_wait(sm.empty(sl), (mm - 1) & 1u);
             pipe_issue(A, A.stg[s_begin + k], sm.slot(sl), sm.full(sl), pol);
         }
     }
@@ -502,24 +528,19 @@ __device__ __forceinline__ void spmv_pipe(const Mat& A, int64_t tr0c, int64_t tr
             cnt->nzn(e, (int)(A.tile_nnz[i + 1] - A.tile_nnz[i]));
         }
     __syncthreads();
-    const unsigned lev_s = smem_u32(sm.lev());
+    const uint8_t* lev_s = sm.lev();
+    unsigned char* D = sm.D();
     PipeStage nxt;
     for (int k = 0; k < ns; ++k) {
         const unsigned u = u0 + (unsigned)k, sl = u % PIPE_NST, mm = u / PIPE_NST;
         const bool refill = t == 0 && k + PIPE_NST < ns;
         if (refill) nxt = A.stg[s_begin + k + PIPE_NST];
+        if (k > 0) __syncthreads();           // the decoded-stage buffer is free (previous FMA pass done)
         mbar_wait(sm.full(sl), mm & 1u);
-        const unsigned slot = smem_u32(sm.slot(sl)), Eb = smem_u32(sm.E(0));
-        if (k > 0) __syncthreads();           // E free: every warp is done with the previous stage
-        pipe_decode<DYN>(slot, Eb, level, lev_s, lev_staged, seg_lo, range_guard);
-        __syncthreads();                      // E complete
-        pipe_fma(A, slot, Eb, tr0c, x, own, emit);
-        __syncwarp();
-        if ((t & 31) == 0) mbar_arrive(sm.empty(sl));
-        if (refill) {
-            mbar_wait(sm.empty(sl), mm & 1u);
-            pipe_issue(A, nxt, sm.slot(sl), sm.full(sl), pol);
-        }
+        pipe_decode<DYN>(pipe_view(sm.slot(sl)), D, level, lev_s, lev_staged, seg_lo, range_guard);
+        __syncthreads();                      // decoded stage complete; slot sl no longer read
+        if (refill) pipe_issue(A, nxt, sm.slot(sl), sm.full(sl), pol);
+        pipe_fma(A, D, tr0c, x, own, emit);
     }
     __syncthreads();
     if (t == 0) *sm.ctr() = (unsigned long long)(u0 + (unsigned)ns);

@@ -388,16 +388,16 @@ __global__ void __launch_bounds__(MAXT, 1) cg_persistent(SolveArgs a) {
             const double beta = __ddiv_rn(rr[0], rho);
             rho = rr[0];
             // step D: p = r + beta p (own rows) and the levels of its segments (Alg. 4)
-            for (int64_t TR0 = tr0 + h; TR0 < tr1; TR0 += 2 * (int64_t)H) {
-                double pv[2], rv[2];
+            for (int64_t TR0 = tr0 + h; TR0 < tr1; TR0 += 4 * (int64_t)H) {
+                double pv[4], rv[4];
 #pragma unroll
-                for (int q = 0; q < 2; ++q) {
+                for (int q = 0; q < 4; ++q) {
                     const int64_t i = (TR0 + q * H) * 16 + lane;
                     pv[q] = 0.0; rv[q] = 0.0;
                     if (TR0 + q * H < tr1 && i < n) { pv[q] = P[i]; rv[q] = Rv[i]; }
                 }
 #pragma unroll
-                for (int q = 0; q < 2; ++q) {
+                for (int q = 0; q < 4; ++q) {
                     const int64_t TR = TR0 + q * H;
                     if (TR < tr1) {                            // uniform per half-warp
                         const int64_t i = TR * 16 + lane;
@@ -445,7 +445,7 @@ __global__ void __launch_bounds__(MAXT, 1) bicgstab_persistent(SolveArgs a) {
     double* __restrict__ Rv = a.r;
     double* __restrict__ P = a.p;
     double* __restrict__ S = a.s;
-    const double* __restrict__ RH = a.rh;
+    const double* RH = a.rh;   // written at init in this kernel: no read-only (.nc) loads
     double* __restrict__ MUs = sm.mu;
     double* __restrict__ THs = sm.th;
     auto mu_at = [&](int64_t li) -> double& { return li < mu_cap ? MUs[li] : a.mu_g[R0 + li]; };
@@ -815,7 +815,7 @@ __global__ void __launch_bounds__(MAXT, 1) pbicgstab_persistent(SolveArgs a) {
     double* __restrict__ S = a.s;
     double* PH = a.pz;
     double* SH = a.ps;
-    const double* __restrict__ RH = a.rh;
+    const double* RH = a.rh;   // written at init in this kernel: no read-only (.nc) loads
     double* __restrict__ MUs = sm.mu;
     double* __restrict__ THs = sm.th;
     auto mu_at = [&](int64_t li) -> double& { return li < mu_cap ? MUs[li] : a.mu_g[R0 + li]; };
