@@ -10,8 +10,9 @@ convergence (mf_cg_solve).  value = CG iterations per second over the timed step
 
   python bench.py [--gpus N] [--steps K] [--warmup W] [--config C2] [--impl reference]
 
-N > 1 (torchrun, one process per GPU): every rank solves its own instance (weak scaling, no
-data-path collective), timed on the device, max over ranks.
+N > 1 (torchrun, one process per GPU): ONE solve of the config's matrix partitioned into row
+blocks over the N GPUs (dist.py: NCCL halo exchange + rank-ordered scalar reductions; strong
+scaling), timed on the device, max over ranks.
 --impl reference: the oracle (oracle/, plain C, binary64) on the host cores, same metric and
 config, each step a bounded sample of the workload (the first --ref-iters CG iterations).
 """
@@ -239,6 +240,106 @@ def gpu_arm(args, rank, world):
     return line
 
 
+def dist_arm(args, rank, world):
+    """N > 1: ONE solve of the config's matrix row-partitioned over the N GPUs (SURVEY 8(e),
+    paper_conf_sc_yangznjs0t024_b200/dist.py): NCCL halo exchange of p + rank-ordered scalar
+    reductions, per-rank work in libmf kernels.  Strong scaling: value = CG iterations per second
+    of the distributed solve; a step = per-rank conversion of its rows + the solve."""
+    import torch
+    import torch.distributed as td
+
+    import paper_conf_sc_yangznjs0t024_b200 as mf
+    import workloads as W
+    from paper_conf_sc_yangznjs0t024_b200 import dist
+
+    dev = torch.device("cuda", rank % max(torch.cuda.device_count(), 1))
+    torch.cuda.set_device(dev)
+    mf.build()
+    mf.lib()
+    spec, desc = _config(args.config)
+    if spec["solver"] != "cg":
+        raise SystemExit("row-partitioned multi-GPU path: CG configs (C1, C2, C5)")
+    A = W.make(args.config)
+    b_h = W.rhs_ones(A)
+    bnd = dist.partition_rows(A.n_rows, world, A.rowptr)
+    rb, re = bnd[rank], bnd[rank + 1]
+    rp, ci, va = dist.local_rows(A, rb, re)
+    b = torch.from_numpy(b_h[rb:re].copy()).to(dev)
+    comm = dist.Comm()
+    eng = dist.CudaEngine(dev)
+
+    def step():
+        D = dist.DistMatrix(eng, comm, A.n_rows, rb, re, rp, ci, va)
+        return D, dist.cg_solve(D, b, tol=1e-10, max_iter=spec["max_iter"], mode="dynamic")
+
+    for _ in range(args.warmup):
+        D, r = step()
+        conv_launches = D.M.info()["convert_launches"]
+        D.M.close()
+    torch.cuda.synchronize()
+    td.barrier()
+    stream = torch.cuda.current_stream()
+    e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    with Clocks(dev.index) as clk:
+        torch.cuda.synchronize()
+        e0.record(stream)
+        iters = 0
+        for _ in range(args.steps):
+            D, r = step()
+            assert r.converged
+            iters += r.iterations
+            D.M.close()
+        e1.record(stream)
+        torch.cuda.synchronize()
+    ms = torch.tensor([e0.elapsed_time(e1)], dtype=torch.float64, device=dev)
+    td.all_reduce(ms, op=td.ReduceOp.MAX)
+    total_ms = float(ms.item())
+    value = iters / (total_ms / 1e3)
+    # e2e through the public API with host inputs: this rank's CSR rows and b slice (host) ->
+    # device inside the timed region, conversion + solve, x back to pinned host memory
+    bh = torch.from_numpy(b_h[rb:re].copy()).pin_memory()
+    xh = torch.empty(re - rb, dtype=torch.float64).pin_memory()
+    td.barrier()
+    torch.cuda.synchronize()
+    f0, f1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    f0.record(stream)
+    e2e_it = 0
+    for _ in range(args.steps):
+        bd = bh.to(dev, non_blocking=True)
+        D = dist.DistMatrix(eng, comm, A.n_rows, rb, re, rp, ci, va)
+        r = dist.cg_solve(D, bd, tol=1e-10, max_iter=spec["max_iter"], mode="dynamic")
+        xh.copy_(r.x, non_blocking=True)
+        e2e_it += r.iterations
+        D.M.close()
+    f1.record(stream)
+    torch.cuda.synchronize()
+    ms2 = torch.tensor([f0.elapsed_time(f1)], dtype=torch.float64, device=dev)
+    td.all_reduce(ms2, op=td.ReduceOp.MAX)
+    peaks = _peaks()
+    n = A.n_rows
+    # byte model per iteration (global, all ranks): static TilePrec bytes + 48n vectors + halo planes
+    line = {
+        "metric": METRIC, "value": round(value, 3), "unit": UNIT, "n_gpus": world, "steps": args.steps,
+        "warmup": args.warmup, "ms_per_step": round(total_ms / args.steps, 4), "higher_is_better": True,
+        "scaling": "strong", "vs_baseline": None, "dtype": "f64", "data": "synthetic (seeded workloads.py)",
+        "config": {"workload": desc, "n": n, "nnz": A.nnz, "solver": "cg", "tol": 1e-10,
+                   "mode": "dynamic mixed (FP64/FP32/FP16/E4M3 tiles + bypass)",
+                   "step": "per-rank conversion of its rows + one distributed solve",
+                   "parallelism": f"row blocks over {world} GPUs (NCCL halo of p + rank-ordered scalar all-gathers)",
+                   "partition_rows": bnd, "l2": "inputs larger than L2 per step (whole solve)"},
+        "iterations": r.iterations,
+        "halo_bytes_per_iteration_rank0": D.plan.bytes_per_exchange(),
+        "e2e": {"value": round(e2e_it / (float(ms2.item()) / 1e3), 3), "unit": UNIT,
+                "h2d_bytes_per_step": int(rp.nbytes + ci.nbytes + va.nbytes + 8 * (re - rb)),
+                "d2h_bytes_per_step": int(8 * (re - rb))},
+        # libmf kernels per step on this rank: conversion, 2 init dots (2 kernels each), and per
+        # iteration levels + SpMV + dot (2) + fused x/r update (2) + p update
+        "gpu_launches": int(args.steps * (conv_launches + 4 + 7 * r.iterations)),
+        "clocks": clk.summary(),
+    }
+    return line
+
+
 def cpu_baseline(args, sample_iters):
     import oracle
     import workloads as W
@@ -285,6 +386,25 @@ def reference_arm(args):
             "e2e": {"value": round(value, 4), "unit": UNIT, "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
 
 
+def torch_dist_ready():
+    import torch.distributed as td
+    return td.is_available() and td.is_initialized()
+
+
+def init_single_rank_group():
+    """--dist with one process: a one-rank NCCL group (exercises the multi-GPU path on 1 GPU)."""
+    import socket
+
+    import torch
+    s = socket.socket()
+    s.bind(("127.0.0.1", 0))
+    port = s.getsockname()[1]
+    s.close()
+    os.environ.setdefault("MASTER_ADDR", "127.0.0.1")
+    os.environ.setdefault("MASTER_PORT", str(port))
+    torch.distributed.init_process_group("nccl", rank=0, world_size=1, device_id=torch.device("cuda", 0))
+
+
 def main():
     ap = argparse.ArgumentParser()
     ap.add_argument("--gpus", type=int, default=1)
@@ -295,6 +415,7 @@ def main():
     ap.add_argument("--ref-iters", type=int, default=12, help="oracle iterations per reference step")
     ap.add_argument("--cpu-sample-iters", type=int, default=100)
     ap.add_argument("--no-cpu-baseline", action="store_true")
+    ap.add_argument("--dist", action="store_true", help="row-partitioned multi-GPU path even with one rank")
     args = ap.parse_args()
     world = int(os.environ.get("WORLD_SIZE", "1"))
     rank = int(os.environ.get("RANK", "0"))
@@ -306,12 +427,17 @@ def main():
     if world > 1:
         import torch
         torch.distributed.init_process_group("nccl", device_id=torch.device("cuda", int(os.environ.get("LOCAL_RANK", rank))))
-    line = gpu_arm(args, int(os.environ.get("LOCAL_RANK", rank)), world)
+    if world > 1 or args.dist:
+        if not torch_dist_ready():
+            init_single_rank_group()
+        line = dist_arm(args, int(os.environ.get("LOCAL_RANK", rank)), world)
+    else:
+        line = gpu_arm(args, int(os.environ.get("LOCAL_RANK", rank)), world)
     if rank == 0:
         if world == 1 and not args.no_cpu_baseline:
             line["cpu_baseline"] = cpu_baseline(args, args.cpu_sample_iters)
         print(json.dumps(line), flush=True)
-    if world > 1:
+    if torch_dist_ready():
         import torch
         torch.distributed.destroy_process_group()
 

@@ -11,7 +11,7 @@
  *    detail string.  Argument and CSR validation happen before any device work.
  *  - The caller owns every input buffer; buffers are read, never retained, and must stay
  *    valid until `stream` has passed the call.  The library owns handles (mf_tile_matrix,
- *    mf_precond, mf_comm) and their workspaces; *_destroy frees them.  Workspace memory
+ *    mf_precond) and their workspaces; *_destroy frees them.  Workspace memory
  *    comes from the allocator installed with mf_set_allocator (default: cudaMallocAsync).
  *  - At most one solve may be in flight per mf_tile_matrix.
  *  - Requires compute capability 10.0 (B200, sm_100a); otherwise MF_ERR_UNSUPPORTED_DEVICE.
@@ -58,7 +58,6 @@ typedef enum { MF_PRECOND_NONE = 0, MF_PRECOND_ILU0 = 1 } mf_precond_kind;
 
 typedef struct mf_tile_matrix mf_tile_matrix;
 typedef struct mf_precond mf_precond;
-typedef struct mf_comm mf_comm;
 
 /* ---------------------------------------------------------------- conversion */
 typedef struct {
@@ -178,20 +177,19 @@ mf_status mf_cg_solve(const mf_tile_matrix* A, const double* b, double* x, const
 mf_status mf_bicgstab_solve(const mf_tile_matrix* A, const double* b, double* x, const mf_solve_opts* opts,
                             mf_solve_info* info, mf_stream stream);
 
-/* ---------------------------------------------------------------- multi-GPU (row blocks) */
-/* One process per GPU.  nccl_unique_id: host, 128 bytes (from mf_comm_unique_id on rank 0,
- * broadcast by the caller, e.g. over a torch.distributed process group). */
-mf_status mf_comm_unique_id(void* out128 /* host */);
-mf_status mf_comm_create(const void* nccl_unique_id, int32_t nranks, int32_t rank, mf_comm** out);
-mf_status mf_comm_destroy(mf_comm* c);
-/* This rank's rows [row_begin, row_end) of an n_global x n_global matrix; colidx global. */
-mf_status mf_tile_matrix_from_csr_dist(mf_comm* c, int64_t n_global, int64_t row_begin, int64_t row_end,
-                                       int64_t nnz_local, const int64_t* rowptr, const int32_t* colidx,
-                                       const double* vals, const mf_convert_opts* opts, mf_stream stream,
-                                       mf_tile_matrix** out);
-/* b, x: this rank's local slices. */
-mf_status mf_cg_solve_dist(const mf_tile_matrix* A, const double* b, double* x, const mf_solve_opts* opts,
-                           mf_solve_info* info, mf_stream stream);
+/* ---------------------------------------------------------------- multi-GPU (row blocks)
+ * One process per GPU; rank k owns the tile-aligned rows [row_begin, row_end) of the global
+ * matrix and converts them as a local n_local x n_ext matrix whose columns are the contiguous
+ * range [xlo, xhi) of global columns its rows gather (xlo a multiple of 16, so local and global
+ * 16-segments coincide).  The halo exchange of the search direction and the scalar reductions
+ * run over NCCL from the Python layer (torch.distributed); every arithmetic step runs in these
+ * kernels, with the launch plan's reduction tree (rank partials are then summed in rank order).
+ * Alg. 1 steps C and D: */
+/* x += alpha p ; r = fma(-alpha, mu, r) on the matrix's rows; *rr (host) = (r, r), plan tree. */
+mf_status mf_cg_update_xr(const mf_tile_matrix* A, double alpha, const double* p, const double* mu, double* x,
+                          double* r, double* rr, mf_stream stream);
+/* p = fma(beta, p, r) on the matrix's rows. */
+mf_status mf_cg_update_p(const mf_tile_matrix* A, double beta, const double* r, double* p, mf_stream stream);
 
 const char* mf_status_string(mf_status s);
 const char* mf_last_error(void);

@@ -33,8 +33,7 @@ STATUS = {0: "MF_OK", 1: "MF_ERR_INVALID_ARG", 2: "MF_ERR_UNSORTED_CSR", 3: "MF_
 SYMBOLS = ["mf_default_convert_opts", "mf_default_solve_opts", "mf_set_allocator", "mf_tile_matrix_from_csr",
            "mf_tile_matrix_destroy", "mf_tile_matrix_info", "mf_tile_matrix_export", "mf_spmv", "mf_levels",
            "mf_dot", "mf_precond_create", "mf_precond_destroy", "mf_precond_apply", "mf_cg_solve",
-           "mf_bicgstab_solve", "mf_comm_unique_id", "mf_comm_create", "mf_comm_destroy",
-           "mf_tile_matrix_from_csr_dist", "mf_cg_solve_dist", "mf_status_string", "mf_last_error",
+           "mf_bicgstab_solve", "mf_cg_update_xr", "mf_cg_update_p", "mf_status_string", "mf_last_error",
            "mf_abi_version"]
 
 NVCC_FLAGS = ["-gencode", "arch=compute_100a,code=sm_100a", "-O3", "-lineinfo", "-std=c++17", "-fmad=false",
@@ -143,12 +142,8 @@ def lib():
         L.mf_precond_apply.argtypes = [vp, vp, vp, vp]
         L.mf_cg_solve.argtypes = [vp, vp, vp, C.POINTER(SolveOpts), C.POINTER(SolveInfo), vp]
         L.mf_bicgstab_solve.argtypes = [vp, vp, vp, C.POINTER(SolveOpts), C.POINTER(SolveInfo), vp]
-        L.mf_comm_unique_id.argtypes = [vp]
-        L.mf_comm_create.argtypes = [vp, i32, i32, C.POINTER(vp)]
-        L.mf_comm_destroy.argtypes = [vp]
-        L.mf_tile_matrix_from_csr_dist.argtypes = [vp, i64, i64, i64, i64, vp, vp, vp, C.POINTER(ConvertOpts), vp,
-                                                   C.POINTER(vp)]
-        L.mf_cg_solve_dist.argtypes = [vp, vp, vp, C.POINTER(SolveOpts), C.POINTER(SolveInfo), vp]
+        L.mf_cg_update_xr.argtypes = [vp, d, vp, vp, vp, vp, C.POINTER(d), vp]
+        L.mf_cg_update_p.argtypes = [vp, d, vp, vp, vp]
         _lib = L
         return L
 
@@ -277,6 +272,26 @@ class TileMatrix:
         out = C.c_double()
         _check(lib().mf_dot(self._h, _ptr(u), _ptr(v), C.byref(out), _stream_ptr(stream)))
         return out.value
+
+
+    # CG steps C and D (Alg. 1) on this matrix's rows -- the per-rank kernels of the
+    # row-block multi-GPU driver (dist.py); same reduction tree as dot().
+    def cg_update_xr(self, alpha, p, mu, x, r, stream=None) -> float:
+        """x += alpha p ; r = fma(-alpha, mu, r) ; returns (r, r)."""
+        import torch
+        for t, nm in ((p, "p"), (mu, "mu"), (x, "x"), (r, "r")):
+            _need_cuda(t, torch.float64, nm)
+        out = C.c_double()
+        _check(lib().mf_cg_update_xr(self._h, float(alpha), _ptr(p), _ptr(mu), _ptr(x), _ptr(r), C.byref(out),
+                                     _stream_ptr(stream)))
+        return out.value
+
+    def cg_update_p(self, beta, r, p, stream=None):
+        """p = fma(beta, p, r)."""
+        import torch
+        _need_cuda(r, torch.float64, "r")
+        _need_cuda(p, torch.float64, "p")
+        _check(lib().mf_cg_update_p(self._h, float(beta), _ptr(r), _ptr(p), _stream_ptr(stream)))
 
 
 def levels(v, th, stream=None):

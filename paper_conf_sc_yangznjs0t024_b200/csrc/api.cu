@@ -232,6 +232,17 @@ mf_status mf_dot(const mf_tile_matrix* A, const double* u, const double* v, doub
     return run_dot(A->m, u, v, out, (cudaStream_t)stream);
 }
 
+mf_status mf_cg_update_xr(const mf_tile_matrix* A, double alpha, const double* p, const double* mu, double* x, double* r,
+                          double* rr, mf_stream stream) {
+    if (!A || !rr || (A->m.n_rows > 0 && (!p || !mu || !x || !r))) return fail(MF_ERR_INVALID_ARG, "NULL argument");
+    return run_cg_xr(A->m, alpha, p, mu, x, r, rr, (cudaStream_t)stream);
+}
+
+mf_status mf_cg_update_p(const mf_tile_matrix* A, double beta, const double* r, double* p, mf_stream stream) {
+    if (!A || (A->m.n_rows > 0 && (!r || !p))) return fail(MF_ERR_INVALID_ARG, "NULL argument");
+    return run_cg_p(A->m, beta, r, p, (cudaStream_t)stream);
+}
+
 static mf_status solve_common(const mf_tile_matrix* A, bool bicg, const double* b, double* x,
                               const mf_solve_opts* opts, mf_solve_info* info, mf_stream stream) {
     if (!A || !info || (A->m.n_rows > 0 && (!b || !x))) return fail(MF_ERR_INVALID_ARG, "NULL argument");
@@ -241,7 +252,6 @@ static mf_status solve_common(const mf_tile_matrix* A, bool bicg, const double* 
     if (!(o.tol >= 0) || o.max_iter < 0) return fail(MF_ERR_INVALID_ARG, "tol must be >= 0 and max_iter >= 0");
     if (o.mode < MF_MODE_FP64 || o.mode > MF_MODE_DYNAMIC_MIXED) return fail(MF_ERR_INVALID_ARG, "bad mode");
     *info = mf_solve_info{};
-    if (A->m.comm) return fail(MF_ERR_INVALID_ARG, "distributed matrix: use mf_cg_solve_dist");
     return run_solve(A->m, bicg, b, x, o, info, (cudaStream_t)stream);
 }
 

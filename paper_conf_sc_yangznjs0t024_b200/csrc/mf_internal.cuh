@@ -98,9 +98,6 @@ struct TileMatrix {
     int32_t* seg_lo = nullptr;       // device [G] first column segment gathered by CTA g
     int32_t* seg_hi = nullptr;       // device [G] last column segment gathered (-1: none)
     int64_t* plan_rows_host = nullptr;  // host [G+1]
-    // distributed (row block of a larger matrix); row_begin == 0 and halo empty on 1 GPU
-    mf_comm* comm = nullptr;
-    int64_t row_begin = 0, n_global = 0;
     // byte bookkeeping
     int64_t canonical_bytes = 0, kernel_bytes = 0;
     cudaStream_t owner_stream = nullptr;
@@ -114,6 +111,9 @@ mf_status run_spmv(const TileMatrix& A, const double* x, double* y, const uint8_
                    int64_t* counts_host, cudaStream_t s);
 mf_status run_levels(const double* v, int64_t n, const double* th, uint8_t* level, cudaStream_t s);
 mf_status run_dot(const TileMatrix& A, const double* u, const double* v, double* out_host, cudaStream_t s);
+mf_status run_cg_xr(const TileMatrix& A, double alpha, const double* p, const double* mu, double* x, double* r,
+                    double* rr_host, cudaStream_t s);
+mf_status run_cg_p(const TileMatrix& A, double beta, const double* r, double* p, cudaStream_t s);
 mf_status run_solve(const TileMatrix& A, bool bicg, const double* b, double* x, const mf_solve_opts& o,
                     mf_solve_info* info, cudaStream_t s);
 

@@ -18,6 +18,7 @@
 
 #include <algorithm>
 #include <cmath>
+#include <cstdio>
 #include <cstdlib>
 #include <vector>
 
@@ -1021,6 +1022,32 @@ __global__ void dot_partial_kernel(const int32_t* __restrict__ plan_tr, int64_t 
         if (threadIdx.x == 0) slots[blockIdx.x] = ct;
     }
 }
+// CG vector steps for the row-block multi-GPU driver (same plan tree as the persistent kernel):
+//   xr: x += alpha p, r = fma(-alpha, mu, r), partial (r, r);   p: p = fma(beta, p, r)
+__global__ void cg_xr_kernel(const int32_t* __restrict__ plan_tr, int64_t n, double alpha, const double* p, const double* mu,
+                             double* x, double* r, double* slots) {
+    __shared__ double red[32];
+    const int64_t R0 = (int64_t)plan_tr[blockIdx.x] * 16, Rend = min((int64_t)plan_tr[blockIdx.x + 1] * 16, n);
+    double acc = 0.0;
+    for (int64_t i = R0 + threadIdx.x; i < Rend; i += blockDim.x) {
+        x[i] = __fma_rn(alpha, p[i], x[i]);
+        const double ri = __fma_rn(-alpha, mu[i], r[i]);
+        r[i] = ri;
+        acc = __fma_rn(ri, ri, acc);
+    }
+    const double wt = mfk::butterfly32(acc);
+    if ((threadIdx.x & 31) == 0) red[threadIdx.x >> 5] = wt;
+    __syncthreads();
+    if (threadIdx.x < 32) {
+        const double ct = mfk::tree32(red, blockDim.x >> 5);
+        if (threadIdx.x == 0) slots[blockIdx.x] = ct;
+    }
+}
+__global__ void cg_p_kernel(int64_t n, double beta, const double* r, double* p) {
+    for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x)
+        p[i] = __fma_rn(beta, p[i], r[i]);
+}
+
 __global__ void dot_final_kernel(const double* __restrict__ slots, int G, double* out) {
     const double gt = mfk::tree32(slots, G);
     if (threadIdx.x == 0) *out = gt;
@@ -1097,6 +1124,27 @@ mf_status run_dot(const TileMatrix& A, const double* u, const double* v, double*
     MF_CUDA(cudaMemcpyAsync(out_host, slots + A.G, sizeof(double), cudaMemcpyDeviceToHost, s));
     MF_CUDA(cudaStreamSynchronize(s));
     dev_free(slots, s);
+    return MF_OK;
+}
+
+mf_status run_cg_xr(const TileMatrix& A, double alpha, const double* p, const double* mu, double* x, double* r,
+                    double* rr_host, cudaStream_t s) {
+    double* slots = nullptr;
+    MF_TRY(alloc(&slots, A.G + 1, s));
+    cg_xr_kernel<<<A.G, A.B, 0, s>>>(A.plan_tr, A.n_rows, alpha, p, mu, x, r, slots);
+    dot_final_kernel<<<1, 32, 0, s>>>(slots, A.G, slots + A.G);
+    MF_CUDA(cudaGetLastError());
+    MF_CUDA(cudaMemcpyAsync(rr_host, slots + A.G, sizeof(double), cudaMemcpyDeviceToHost, s));
+    MF_CUDA(cudaStreamSynchronize(s));
+    dev_free(slots, s);
+    return MF_OK;
+}
+
+mf_status run_cg_p(const TileMatrix& A, double beta, const double* r, double* p, cudaStream_t s) {
+    if (A.n_rows == 0) return MF_OK;
+    const int blocks = (int)std::min<int64_t>((A.n_rows + 255) / 256, 148 * 8);
+    cg_p_kernel<<<blocks, 256, 0, s>>>(A.n_rows, beta, r, p);
+    MF_CUDA(cudaGetLastError());
     return MF_OK;
 }
 
@@ -1280,6 +1328,18 @@ mf_status run_solve(const TileMatrix& A, bool bicg, const double* b, double* x, 
         double sum = 0;
         for (int g = 0; g < G; ++g) sum += (double)ph[(size_t)g * NPHASE + k];
         info->phase_ms[k] = sum / G / 1e6;
+    }
+    if (getenv("MF_PHASE_DUMP")) {   // diagnostics: per-phase min / mean / max over CTAs (ms)
+        for (int k = 0; k < NPHASE; ++k) {
+            double mn = 1e300, mx = 0, sum = 0;
+            for (int g = 0; g < G; ++g) { const double v = (double)ph[(size_t)g * NPHASE + k] / 1e6; mn = std::min(mn, v); mx = std::max(mx, v); sum += v; }
+            if (mx > 0) fprintf(stderr, "phase %2d: min %.3f mean %.3f max %.3f ms\n", k, mn, sum / G, mx);
+        }
+        fprintf(stderr, "spmv per CTA:");
+        for (int g = 0; g < G; ++g) fprintf(stderr, " %.2f", (double)ph[(size_t)g * NPHASE + 1] / 1e6);
+        fprintf(stderr, "\nrows per CTA:");
+        for (int g = 0; g < G; ++g) fprintf(stderr, " %lld", (long long)(A.plan_rows_host[g + 1] - A.plan_rows_host[g]));
+        fprintf(stderr, "\n");
     }
     {
         double sum = 0;
