@@ -675,7 +675,9 @@ mf_status convert_csr(int64_t n_rows, int64_t n_cols, int64_t nnz, const int64_t
     if (B % 32 || B > 1024 || B < 32) {
         return fail(MF_ERR_INVALID_ARG, "block_threads must be a multiple of 32 in [32, 1024]");
     }
-    if (G <= 0) G = (int)std::max<int64_t>(1, std::min<int64_t>(sms, ntr / 64));
+    // auto plan: one CTA per SM; small matrices get at least 8 tile rows per CTA (latency-bound:
+    // more CTAs shorten the per-CTA chain more than the extra barrier participants cost)
+    if (G <= 0) G = (int)std::max<int64_t>(1, std::min<int64_t>(sms, (ntr + 7) / 8));
     if (G > sms * 2) G = sms * 2;
     if (ntr > 0 && G > ntr) G = (int)ntr;
     if (G < 1) G = 1;

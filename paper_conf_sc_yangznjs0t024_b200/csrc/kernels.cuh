@@ -234,6 +234,7 @@ struct TsSmem {
         return reinterpret_cast<unsigned long long*>(D() + PIPE_D_BYTES) + s;
     }
     __device__ __forceinline__ unsigned long long* ctr() const { return full(0) + PIPE_NST; }
+    __device__ __forceinline__ unsigned long long* resident() const { return full(0) + PIPE_NST + 1; }
     __device__ __forceinline__ uint8_t* lev() const { return reinterpret_cast<uint8_t*>(full(0) + PIPE_NST + 2); }
 };
 
@@ -286,6 +287,7 @@ __device__ __forceinline__ void pipe_init(const TsSmem& sm) {
     if (threadIdx.x == 0) {
         for (int s = 0; s < PIPE_NST; ++s) mbar_init(sm.full(s), 1);
         *sm.ctr() = 0ull;
+        *sm.resident() = 0ull;
         asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
     }
 }
@@ -510,6 +512,35 @@ __device__ __forceinline__ void spmv_pipe(const Mat& A, int64_t tr0c, int64_t tr
     const int32_t nlev = seg_hi - seg_lo + 1;
     const bool lev_staged = DYN && nlev > 0 && nlev <= PIPE_LEV_CAP;
     __syncthreads();                          // smem users of the previous phase are done
+    if (ns <= PIPE_NST) {
+        // every stage of this CTA fits the ring: load once, keep the slots resident across SpMVs
+        // (small matrices, e.g. C1: no TMA round trip per SpMV)
+        const bool loaded = *sm.resident() != 0ull;
+        if (!loaded && t == 0) {
+            const unsigned long long pol = policy_evict_first();
+            for (int k = 0; k < ns; ++k) pipe_issue(A, A.stg[s_begin + k], sm.slot(k), sm.full(k), pol);
+        }
+        if (lev_staged)
+            for (int i = t; i < nlev; i += B) sm.lev()[i] = level[seg_lo + i];
+        if (COUNT)
+            for (int64_t i = A.tr_tile[tr0c] + t; i < A.tr_tile[tr1c]; i += B) {
+                const int e = (int)(tile_code<DYN>(A.tile_info[i], level, range_guard) & 7u);
+                cnt->tile(e);
+                cnt->nzn(e, (int)(A.tile_nnz[i + 1] - A.tile_nnz[i]));
+            }
+        __syncthreads();
+        unsigned char* D = sm.D();
+        for (int k = 0; k < ns; ++k) {
+            if (k > 0) __syncthreads();
+            if (!loaded) mbar_wait(sm.full(k), 0u);
+            pipe_decode<DYN>(pipe_view(sm.slot(k)), D, level, sm.lev(), lev_staged, seg_lo, range_guard);
+            __syncthreads();
+            pipe_fma(A, D, tr0c, x, own, emit);
+        }
+        __syncthreads();
+        if (t == 0) *sm.resident() = 1ull;
+        return;
+    }
     const unsigned u0 = (unsigned)*sm.ctr();
     unsigned long long pol = 0;
     if (t == 0) {
