@@ -26,7 +26,7 @@ def mf():
 def test_header_declares_the_paper_calls():
     fns = header_functions()
     for name in ("mf_tile_matrix_from_csr", "mf_cg_solve", "mf_bicgstab_solve", "mf_precond_create",
-                 "mf_spmv", "mf_levels", "mf_dot", "mf_cg_solve_dist"):
+                 "mf_spmv", "mf_levels", "mf_dot", "mf_cg_update_xr", "mf_cg_update_p"):
         assert name in fns
 
 
