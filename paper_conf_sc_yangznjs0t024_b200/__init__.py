@@ -37,7 +37,7 @@ SYMBOLS = ["mf_default_convert_opts", "mf_default_solve_opts", "mf_set_allocator
            "mf_abi_version"]
 
 NVCC_FLAGS = ["-gencode", "arch=compute_100a,code=sm_100a", "-O3", "-lineinfo", "-std=c++17", "-fmad=false",
-              "-Xcompiler", "-fPIC", "-shared"]
+              "-Xcompiler", "-fPIC"]
 
 
 class MFError(RuntimeError):
@@ -55,12 +55,22 @@ def build(force: bool = False, verbose: bool = False) -> str:
             os.path.getmtime(LIB_PATH) >= max(os.path.getmtime(d) for d in deps):
         return LIB_PATH
     nccl_inc, nccl_lib = _nccl_paths()
-    tmp = LIB_PATH + f".{os.getpid()}.tmp"
-    cmd = ["nvcc", *NVCC_FLAGS, "-I", INCLUDE, "-I", nccl_inc, "-o", tmp, *srcs,
-           "-L", nccl_lib, "-l:libnccl.so.2", f"-Xlinker=-rpath={nccl_lib}"]
+    # one nvcc per translation unit, in parallel (no relocatable device code: each kernel's
+    # device code lives in the object of its host stub), then one shared-library link
+    from concurrent.futures import ThreadPoolExecutor
+    objdir = os.path.join(HERE, "build")
+    os.makedirs(objdir, exist_ok=True)
+    objs = [os.path.join(objdir, os.path.basename(s)[:-3] + ".o") for s in srcs]
+    cmds = [["nvcc", *NVCC_FLAGS, "-I", INCLUDE, "-I", nccl_inc, "-c", "-o", o, s] for s, o in zip(srcs, objs)]
     if verbose:
-        print(" ".join(cmd))
-    subprocess.check_call(cmd)
+        for c in cmds:
+            print(" ".join(c))
+    with ThreadPoolExecutor(len(cmds)) as ex:
+        for f in [ex.submit(subprocess.check_call, c) for c in cmds]:
+            f.result()
+    tmp = LIB_PATH + f".{os.getpid()}.tmp"
+    subprocess.check_call(["nvcc", "-gencode", "arch=compute_100a,code=sm_100a", "-shared", "-o", tmp, *objs,
+                           "-L", nccl_lib, "-l:libnccl.so.2", f"-Xlinker=-rpath={nccl_lib}"])
     os.replace(tmp, LIB_PATH)
     return LIB_PATH
 

@@ -587,7 +587,7 @@ __device__ __forceinline__ void carve_spmv(unsigned char* base, WinSmem& w, TsSm
     p += (WIN_TR + 1) * 4;
     w.ht = reinterpret_cast<int32_t*>(p);
     p += (WIN_TR + 1) * 4;
-    p = reinterpret_cast<unsigned char*>((reinterpret_cast<uintptr_t>(p) + 15) & ~uintptr_t(15));
+    p = base + pipe_r16((int)(p - base));    // base is 16-aligned; no integer round trip of the pointer
     w.buf = p;
     ts.base = base;    // the two views overlap: a matrix uses one layout
 }

@@ -237,12 +237,13 @@ __device__ __forceinline__ Smem carve(const SolveArgs& a, int nvec) {
     s.red = d;
     s.ired = reinterpret_cast<int*>(d + 4 * 32 + 8);
     s.timer = reinterpret_cast<unsigned long long*>(s.ired + 16);
-    unsigned char* p = reinterpret_cast<unsigned char*>(s.timer + NPHASE + 1);
-    p = reinterpret_cast<unsigned char*>((reinterpret_cast<uintptr_t>(p) + 15) & ~uintptr_t(15));
+    // alignment by offsets from smem_raw (never through an integer cast of the pointer): the
+    // compiler keeps the shared address space and emits LDS/STS with 32-bit addresses
+    unsigned char* p = smem_raw + mfk::pipe_r16((int)(reinterpret_cast<unsigned char*>(s.timer + NPHASE + 1) - smem_raw));
     mfk::carve_spmv(p, s.win, s.ts);
     mfk::pipe_init(s.ts);      // ordered before the first SpMV by the caller's __syncthreads (Timer::start)
     p += mfk::SPMV_SMEM_BYTES;
-    p = reinterpret_cast<unsigned char*>((reinterpret_cast<uintptr_t>(p) + 15) & ~uintptr_t(15));
+    p = smem_raw + mfk::pipe_r16((int)(p - smem_raw));
     s.mu = reinterpret_cast<double*>(p);
     s.th = s.mu + a.mu_cap;
     s.tys = s.mu + (size_t)nvec * a.mu_cap;
