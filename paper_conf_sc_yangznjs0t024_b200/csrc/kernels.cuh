@@ -33,6 +33,8 @@ struct Mat {
     const float* __restrict__ p32;
     const __half* __restrict__ p16;
     const uint8_t* __restrict__ p8;
+    uint8_t* stk;                         // sticky variant (P:237 literal), TS layout: per slice column,
+                                          // bit L set = the column's values were lowered to L in place
 };
 
 __device__ __forceinline__ unsigned hw_mask() { return (threadIdx.x & 16) ? 0xFFFF0000u : 0x0000FFFFu; }
@@ -303,6 +305,7 @@ __device__ __forceinline__ void pipe_issue(const Mat& A, const PipeStage& st, un
     info[4] = st.off_dst;
 #pragma unroll
     for (int q = 0; q < 4; ++q) { info[5 + q] = st.gcnt[q]; info[9 + q] = st.goff[q]; }
+    info[13] = (int32_t)st.col0;
     mbar_expect_tx(full, (unsigned)st.bbytes);
     bulk_g2s_ef(slot, A.blob + st.boff, (unsigned)st.bbytes, full, pol);
 }
@@ -344,7 +347,7 @@ __device__ __forceinline__ PipeView pipe_view(const unsigned char* slot) {
 template <int Q, bool DYN>
 __device__ __forceinline__ void pipe_decode_group(const PipeView& v, double* E, int ncol_q, int goff, const uint16_t* dst_q,
                                                   const uint8_t* __restrict__ level, const uint8_t* lev_s, bool lev_staged,
-                                                  int32_t seg_lo, int range_guard) {
+                                                  int32_t seg_lo, int range_guard, uint8_t* stk) {
     const int units = ncol_q * 4;
     for (int u = threadIdx.x; u < units; u += blockDim.x) {
         const int j = u >> 2, r0 = (u & 3) * 4;
@@ -364,7 +367,32 @@ __device__ __forceinline__ void pipe_decode_group(const PipeView& v, double* E, 
             const uint32_t a = *reinterpret_cast<const uint32_t*>(src);
             w[0] = e4m3_lo(a); w[1] = e4m3_lo(a >> 8); w[2] = e4m3_lo(a >> 16); w[3] = e4m3_lo(a >> 24);
         }
-        if (DYN) {   // e_t = bypass | max(TilePrec, level), range guard e_t <= Floor (Alg. 5)
+        if (DYN && stk != nullptr) {
+            // sticky variant (P:237 literal; oracle spmv_tiles): e_t = max(cur, level) with the
+            // range guard; a new lower e_t lowers the tile's working values in place for good --
+            // the working value is RNE applied at every level the column has been lowered to, in
+            // ascending order (successive rounding, as the in-place copy has it)
+            const uint32_t word = v.cw[d];
+            const int lv = col_level(word >> 4, level, lev_s, lev_staged, seg_lo);
+            if (lv == BYP) { w[0] = w[1] = w[2] = w[3] = 0.0; }
+            else {
+                uint8_t* sp = stk + (v.info[13] + (int)d);
+                unsigned mask = *sp;
+                const int cur = mask ? 31 - __clz(mask) : Q;
+                int e = max(lv, cur);
+                if (range_guard) e = min(e, (int)((word >> 2) & 3u));
+                if (e > cur) {
+                    mask |= 1u << e;
+                    if (r0 == 0) *sp = (uint8_t)mask;   // every unit of the column computes the same mask
+                }
+#pragma unroll
+                for (int L = Q + 1; L <= 3; ++L)
+                    if (mask & (1u << L)) {
+#pragma unroll
+                        for (int k = 0; k < 4; ++k) w[k] = round_to(w[k], L);
+                    }
+            }
+        } else if (DYN) {   // e_t = bypass | max(TilePrec, level), range guard e_t <= Floor (Alg. 5)
             const uint32_t word = v.cw[d];
             const int lv = col_level(word >> 4, level, lev_s, lev_staged, seg_lo);
             if (lv > Q) {
@@ -387,7 +415,7 @@ __device__ __forceinline__ void pipe_decode_group(const PipeView& v, double* E, 
 
 template <bool DYN>
 __device__ __forceinline__ void pipe_decode(const PipeView& v, unsigned char* D, const uint8_t* __restrict__ level, const uint8_t* lev_s,
-                                            bool lev_staged, int32_t seg_lo, int range_guard) {
+                                            bool lev_staged, int32_t seg_lo, int range_guard, uint8_t* stk) {
     double* E = reinterpret_cast<double*>(D);
     {   // the FMA side's copy of the column words, local columns and headers
         const int S0 = v.info[0], S1 = v.info[1], K = S1 - S0;
@@ -407,13 +435,13 @@ __device__ __forceinline__ void pipe_decode(const PipeView& v, unsigned char* D,
     }
     const uint16_t* dst = v.dst;
     const int g0 = v.info[5], g1 = v.info[6], g2 = v.info[7], g3 = v.info[8];
-    pipe_decode_group<0, DYN>(v, E, g0, v.info[9], dst, level, lev_s, lev_staged, seg_lo, range_guard);
+    pipe_decode_group<0, DYN>(v, E, g0, v.info[9], dst, level, lev_s, lev_staged, seg_lo, range_guard, stk);
     dst += g0;
-    pipe_decode_group<1, DYN>(v, E, g1, v.info[10], dst, level, lev_s, lev_staged, seg_lo, range_guard);
+    pipe_decode_group<1, DYN>(v, E, g1, v.info[10], dst, level, lev_s, lev_staged, seg_lo, range_guard, stk);
     dst += g1;
-    pipe_decode_group<2, DYN>(v, E, g2, v.info[11], dst, level, lev_s, lev_staged, seg_lo, range_guard);
+    pipe_decode_group<2, DYN>(v, E, g2, v.info[11], dst, level, lev_s, lev_staged, seg_lo, range_guard, stk);
     dst += g2;
-    pipe_decode_group<3, DYN>(v, E, g3, v.info[12], dst, level, lev_s, lev_staged, seg_lo, range_guard);
+    pipe_decode_group<3, DYN>(v, E, g3, v.info[12], dst, level, lev_s, lev_staged, seg_lo, range_guard, stk);
 }
 
 // one tile row of N columns starting at stage column c: every load first, then the fma chain.
@@ -533,7 +561,7 @@ __device__ __forceinline__ void spmv_pipe(const Mat& A, int64_t tr0c, int64_t tr
         for (int k = 0; k < ns; ++k) {
             if (k > 0) __syncthreads();
             if (!loaded) mbar_wait(sm.full(k), 0u);
-            pipe_decode<DYN>(pipe_view(sm.slot(k)), D, level, sm.lev(), lev_staged, seg_lo, range_guard);
+            pipe_decode<DYN>(pipe_view(sm.slot(k)), D, level, sm.lev(), lev_staged, seg_lo, range_guard, A.stk);
             __syncthreads();
             pipe_fma(A, D, tr0c, x, own, emit);
         }
@@ -568,7 +596,7 @@ __device__ __forceinline__ void spmv_pipe(const Mat& A, int64_t tr0c, int64_t tr
         if (refill) nxt = A.stg[s_begin + k + PIPE_NST];
         if (k > 0) __syncthreads();           // the decoded-stage buffer is free (previous FMA pass done)
         mbar_wait(sm.full(sl), mm & 1u);
-        pipe_decode<DYN>(pipe_view(sm.slot(sl)), D, level, lev_s, lev_staged, seg_lo, range_guard);
+        pipe_decode<DYN>(pipe_view(sm.slot(sl)), D, level, lev_s, lev_staged, seg_lo, range_guard, A.stk);
         __syncthreads();                      // decoded stage complete; slot sl no longer read
         if (refill) pipe_issue(A, nxt, sm.slot(sl), sm.full(sl), pol);
         pipe_fma(A, D, tr0c, x, own, emit);

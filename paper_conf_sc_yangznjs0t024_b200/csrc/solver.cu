@@ -1071,7 +1071,7 @@ void* pick_kernel(bool bicg, bool dyn, bool count, bool pre) {
 Mat mat_view(const TileMatrix& A) {
     return Mat{A.n_rows, A.n_cols, A.ntr, A.tr_slot, A.TileRowPtr, A.tile_info, A.sidx, A.blob,
                reinterpret_cast<const mfk::PipeStage*>(A.stg), A.stg_ptr, A.TileNnz, A.ts, (int)A.max_w,
-               A.plane64, A.plane32, A.plane16, A.plane8};
+               A.plane64, A.plane32, A.plane16, A.plane8, nullptr};
 }
 
 }  // namespace
@@ -1164,7 +1164,11 @@ static double spmv_model_bytes(const TileMatrix& A, const unsigned long long* c1
 mf_status run_solve(const TileMatrix& A, bool bicg, const double* b, double* x, const mf_solve_opts& o,
                     mf_solve_info* info, cudaStream_t s) {
     if (A.n_rows != A.n_cols) return fail(MF_ERR_INVALID_ARG, "solve needs a square matrix");
-    if (o.sticky) return fail(MF_ERR_NOT_IMPLEMENTED, "sticky (in-place) downgrade is not implemented on the GPU path");
+    // sticky variant (P:237 literal): dynamic mode only (as in the oracle), tile-synchronous layout
+    const bool sticky = o.sticky && o.mode == MF_MODE_DYNAMIC_MIXED;
+    if (sticky && !A.ts) return fail(MF_ERR_NOT_IMPLEMENTED, "sticky downgrade is implemented for the tile-synchronous layout only");
+    if (sticky && (o.tile_level_counts != nullptr || o.collect_stats))
+        return fail(MF_ERR_NOT_IMPLEMENTED, "sticky downgrade does not collect per-SpMV level statistics");
     Precond* P = o.M ? const_cast<Precond*>(&o.M->p) : nullptr;
     const bool pre = P != nullptr;
     if (pre && P->n != A.n_rows) return fail(MF_ERR_INVALID_ARG, "preconditioner built for another matrix size");
@@ -1225,8 +1229,14 @@ mf_status run_solve(const TileMatrix& A, bool bicg, const double* b, double* x, 
     MF_CUDA(cudaMemsetAsync(out, 0, 8 * sizeof(double), s));
     if (count) MF_CUDA(cudaMemsetAsync(lcounts, 0, (size_t)lc_cap * 10 * sizeof(unsigned long long), s));
 
+    uint8_t* stk = nullptr;
+    if (sticky) {
+        MF_TRY(alloc(&stk, (size_t)A.slots + 1, s));
+        MF_CUDA(cudaMemsetAsync(stk, 0, (size_t)A.slots + 1, s));
+    }
     SolveArgs a{};
     a.A = mat_view(A);
+    a.A.stk = stk;
     a.G = G; a.plan_tr = A.plan_tr; a.dep_lo = A.dep_lo; a.dep_hi = A.dep_hi; a.seg_lo = A.seg_lo; a.seg_hi = A.seg_hi;
     a.n = n; a.b = b; a.x = x; a.r = r; a.p = p; a.mu_g = mu_g; a.lev_p = lev_p;
     a.rh = rh; a.s = sv; a.th_g = th_g; a.lev_s = lev_s;
@@ -1351,7 +1361,7 @@ mf_status run_solve(const TileMatrix& A, bool bicg, const double* b, double* x, 
     dev_free(r, s); dev_free(p, s); dev_free(mu_g, s); dev_free(lev_p, s); dev_free(rh, s); dev_free(sv, s);
     dev_free(lev_s, s); dev_free(th_g, s); dev_free(slots, s); dev_free(hist, s); dev_free(out, s);
     dev_free(sync, s); dev_free(bar_ns, s); dev_free(phase_ns, s); dev_free(lcounts, s);
-    dev_free(pz, s); dev_free(psh, s);
+    dev_free(pz, s); dev_free(psh, s); dev_free(stk, s);
     if (st == MF_ERR_BREAKDOWN) return fail(st, "numerical breakdown");
     if (st == MF_ERR_DEADLOCK) return fail(st, "grid-barrier watchdog expired");
     return st;
