@@ -117,8 +117,8 @@ typedef struct {
     int32_t switch_absolute;    /* 0: tau = eps*||v0||/sqrt(n) (reading R8); 1: tau = eps (Alg. 1 l.3) */
     int32_t sticky;             /* 1 (dynamic mode): one-time in-place downgrade (P:237 literal) -- a tile
                                    lowered to e_t keeps its values rounded to e_t for the rest of the solve
-                                   (successive RNE, oracle spmv_tiles).  Tile-synchronous layout only, and
-                                   without level statistics: otherwise MF_ERR_NOT_IMPLEMENTED */
+                                   (successive RNE, oracle spmv_tiles).  Both kernel layouts; not combined
+                                   with level statistics (MF_ERR_NOT_IMPLEMENTED) */
     int32_t range_guard;        /* 1 (default): never lower a tile below its range floor */
     const mf_precond* M;        /* NULL = no preconditioner; else PCG / right-preconditioned PBiCGSTAB */
     double* residual_history;   /* host, optional: relres_0 .. relres_k (k+1 values) */

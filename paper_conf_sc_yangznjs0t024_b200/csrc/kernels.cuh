@@ -33,8 +33,8 @@ struct Mat {
     const float* __restrict__ p32;
     const __half* __restrict__ p16;
     const uint8_t* __restrict__ p8;
-    uint8_t* stk;                         // sticky variant (P:237 literal), TS layout: per slice column,
-                                          // bit L set = the column's values were lowered to L in place
+    uint8_t* stk;                         // sticky variant (P:237 literal): per slice column (TS layout) or
+                                          // per tile (compact), bit L set = values lowered to L in place
 };
 
 __device__ __forceinline__ unsigned hw_mask() { return (threadIdx.x & 16) ? 0xFFFF0000u : 0x0000FFFFu; }
@@ -55,6 +55,28 @@ __device__ __forceinline__ uint32_t tile_code(uint32_t info, const uint8_t* __re
     }
     return (tc << 3) | (uint32_t)e;
 }
+
+// sticky variant, compact layout (P:237 literal; oracle spmv_tiles): per-tile mask of the levels
+// the tile was lowered to in place.  Code = (tile column << 3) | e_t | TilePrec << 27 | mask << 29
+// (mask bits L = 1..3 stored as mask >> 1; tile column < 2^24); `update` (the window's code staging, one thread per tile) records a new
+// lowering, the per-slot recomputation of an unstaged window only reads the updated mask.
+__device__ __forceinline__ uint32_t sticky_code(const Mat& A, int64_t tile, const uint8_t* __restrict__ level, int range_guard,
+                                                bool update) {
+    const uint32_t info = A.tile_info[tile];
+    const uint32_t tc = info >> 4, prec = info & 3u;
+    const int lv = level[tc];
+    if (lv == BYP) return (tc << 3) | BYP;
+    unsigned mask = A.stk[tile];
+    const int cur = mask ? 31 - __clz(mask) : (int)prec;
+    int e = max(lv, cur);
+    if (range_guard) e = min(e, (int)((info >> 2) & 3u));
+    if (e > cur) {
+        mask |= 1u << e;
+        if (update) A.stk[tile] = (uint8_t)mask;
+    }
+    return (tc << 3) | (uint32_t)e | (prec << 27) | ((mask >> 1) << 29);   // mask bits 1..3
+}
+constexpr uint32_t CODE_TC_MASK = 0x00FFFFFFu;   // tile column field of a code (after >> 3)
 
 __device__ __forceinline__ double load_val(const Mat& A, int e, int64_t pos) {
     if (e == 0) return A.p64[pos];
@@ -148,18 +170,34 @@ __device__ __forceinline__ double slot_block(const Mat& A, const unsigned long l
         xv[q] = 0.0;
         if (q < cnt && s[q] != mf::SLOT_PAD) {
             const int j = s[q] >> 4;
-            const uint32_t c = staged ? code[j] : tile_code<DYN>(A.tile_info[tb_abs + j], level, range_guard);
+            const uint32_t c = staged ? code[j]
+                               : (DYN && A.stk != nullptr) ? sticky_code(A, tb_abs + j, level, range_guard, false)
+                                                           : tile_code<DYN>(A.tile_info[tb_abs + j], level, range_guard);
             ev[q] = (int)(c & 7u);
             if (COUNT) cntp->nz(ev[q]);
             if (ev[q] != BYP) {
-                raw[q] = load_raw(w_pb, ev[q], pos0 + q * 16);
-                xv[q] = x[(int64_t)(c >> 3) * 16 + (s[q] & 15)];
+                // sticky: the stored value (plane TilePrec), lowered in slot_value below
+                raw[q] = load_raw(w_pb, (DYN && A.stk != nullptr) ? (int)((c >> 27) & 3u) : ev[q], pos0 + q * 16);
+                xv[q] = x[(int64_t)((c >> 3) & CODE_TC_MASK) * 16 + (s[q] & 15)];
+                if (DYN && A.stk != nullptr) ev[q] |= (int)(c >> 24) & 0xF8;   // TilePrec << 3 | (mask >> 1) << 5
             }
         }
     }
 #pragma unroll
     for (int q = 0; q < N; ++q)
-        if (ev[q] != BYP) acc = __fma_rn(decode_val(ev[q], raw[q]), xv[q], acc);
+        if ((ev[q] & 7) != BYP) {
+            double v;
+            if (DYN && A.stk != nullptr) {   // successive RNE at every level the tile was lowered to
+                const int prec = (ev[q] >> 3) & 3, m1 = ev[q] >> 5;   // m1 bit L-1 = lowered to L
+                v = decode_val(prec, raw[q]);
+#pragma unroll
+                for (int L = 1; L <= 3; ++L)
+                    if (L > prec && (m1 & (1 << (L - 1)))) v = round_to(v, L);
+            } else {
+                v = decode_val(ev[q], raw[q]);
+            }
+            acc = __fma_rn(v, xv[q], acc);
+        }
     return acc;
 }
 
@@ -662,7 +700,8 @@ __device__ __forceinline__ void spmv_cta(const Mat& A, int64_t tr0, int64_t tr1,
         const int nt = w.ht[nw];
         uint32_t* code = reinterpret_cast<uint32_t*>(w.buf);
         for (int i = t; i < nt; i += B) {
-            const uint32_t c = tile_code<DYN>(A.tile_info[t0 + i], level, range_guard);
+            const uint32_t c = (DYN && A.stk != nullptr) ? sticky_code(A, t0 + i, level, range_guard, true)
+                                                         : tile_code<DYN>(A.tile_info[t0 + i], level, range_guard);
             if (staged) code[i] = c;
             if (COUNT) cnt->tile((int)(c & 7u));
         }

@@ -1166,7 +1166,8 @@ mf_status run_solve(const TileMatrix& A, bool bicg, const double* b, double* x, 
     if (A.n_rows != A.n_cols) return fail(MF_ERR_INVALID_ARG, "solve needs a square matrix");
     // sticky variant (P:237 literal): dynamic mode only (as in the oracle), tile-synchronous layout
     const bool sticky = o.sticky && o.mode == MF_MODE_DYNAMIC_MIXED;
-    if (sticky && !A.ts) return fail(MF_ERR_NOT_IMPLEMENTED, "sticky downgrade is implemented for the tile-synchronous layout only");
+    if (sticky && !A.ts && (A.n_cols + 15) / 16 > ((int64_t)1 << 24))
+        return fail(MF_ERR_NOT_IMPLEMENTED, "sticky downgrade, compact layout: more than 2^24 tile columns");
     if (sticky && (o.tile_level_counts != nullptr || o.collect_stats))
         return fail(MF_ERR_NOT_IMPLEMENTED, "sticky downgrade does not collect per-SpMV level statistics");
     Precond* P = o.M ? const_cast<Precond*>(&o.M->p) : nullptr;
@@ -1231,8 +1232,9 @@ mf_status run_solve(const TileMatrix& A, bool bicg, const double* b, double* x, 
 
     uint8_t* stk = nullptr;
     if (sticky) {
-        MF_TRY(alloc(&stk, (size_t)A.slots + 1, s));
-        MF_CUDA(cudaMemsetAsync(stk, 0, (size_t)A.slots + 1, s));
+        const size_t nst = (size_t)(A.ts ? A.slots : A.tilenum) + 1;   // per slice column (TS) / per tile (compact)
+        MF_TRY(alloc(&stk, nst, s));
+        MF_CUDA(cudaMemsetAsync(stk, 0, nst, s));
     }
     SolveArgs a{};
     a.A = mat_view(A);

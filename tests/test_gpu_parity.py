@@ -347,16 +347,19 @@ STICKY_CASES = [
     ("C2-32-sticky-148", lambda: W.make("C2", 32), "cg", 148, 128),
     ("ragged-sticky", lambda: W.poisson2d(33), "cg", 3, 64),
     ("C3-64-sticky", lambda: W.make("C3", 64), "bicgstab", 8, 512),
+    ("C4ind-sticky", lambda: W.make("C4ind", 1 << 12), "bicgstab", 6, 256),
 ]
 
 
+@pytest.mark.parametrize("layout", [1, 2])
 @pytest.mark.parametrize("name,make,solver,G,B", STICKY_CASES, ids=[c[0] for c in STICKY_CASES])
-def test_sticky_downgrade_parity(mf, orc, name, make, solver, G, B):
+def test_sticky_downgrade_parity(mf, orc, name, make, solver, G, B, layout):
     """Sticky variant (P:237 literal, oracle spmv_tiles' in-place successive rounding): histories,
-    iteration counts and x bit-identical to the oracle's kernel-order emulation."""
+    iteration counts and x bit-identical to the oracle's kernel-order emulation, both layouts
+    (state per slice column on the TMA pipeline, per tile on the compact layout)."""
     A = make()
     b = W.rhs_ones(A)
-    Gm = mf.TileMatrix.from_host_csr(A, grid_ctas=G, block_threads=B, layout=2)
+    Gm = mf.TileMatrix.from_host_csr(A, grid_ctas=G, block_threads=B, layout=layout)
     g, bb, R = Gm.plan()
     T = oracle_tiles(orc, A, True)
     ofn = orc.cg if solver == "cg" else orc.bicgstab
@@ -378,9 +381,6 @@ def test_sticky_downgrade_parity(mf, orc, name, make, solver, G, B):
 def test_sticky_unsupported_combinations(mf):
     A = W.make("C2", 16)
     b = dev(W.rhs_ones(A))
-    Gc = mf.TileMatrix.from_host_csr(A, grid_ctas=4, block_threads=256, layout=1)
-    with pytest.raises(mf.MFError):
-        mf.cg_solve(Gc, b, mode=2, sticky=True)
     Gt = mf.TileMatrix.from_host_csr(A, grid_ctas=4, block_threads=256, layout=2)
     with pytest.raises(mf.MFError):
         mf.cg_solve(Gt, b, mode=2, sticky=True, level_counts=True)
