@@ -113,8 +113,8 @@ typedef struct {
     double tol;                 /* stop when ||r_j|| / ||b|| < tol (1e-10) */
     int64_t max_iter;           /* 1000 */
     mf_mode mode;               /* default MF_MODE_DYNAMIC_MIXED */
-    double switch_eps;          /* eps of P:174; < 0 = default (= 1e-2 * tol, reading R8) */
-    int32_t switch_absolute;    /* 0: tau = eps*||v0||/sqrt(n) (reading R8); 1: tau = eps (Alg. 1 l.3) */
+    double switch_eps;          /* eps of P:174; < 0 = default (= tol, reading R8); tau = eps*||v0||_2 */
+    int32_t switch_absolute;    /* 0: tau = eps*||v0||_2 (reading R8); 1: tau = eps (Alg. 1 l.3) */
     int32_t sticky;             /* 1 (dynamic mode): one-time in-place downgrade (P:237 literal) -- a tile
                                    lowered to e_t keeps its values rounded to e_t for the rest of the solve
                                    (successive RNE, oracle spmv_tiles).  Both kernel layouts; not combined

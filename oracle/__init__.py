@@ -68,6 +68,10 @@ class _Info(C.Structure):
                 ("rel_residual", C.c_double), ("n_spmv", C.c_int64)]
 
 
+class _Sticky(C.Structure):
+    _fields_ = [("cur", C.POINTER(C.c_uint8)), ("wv", C.POINTER(C.c_double))]
+
+
 class _Ilu(C.Structure):
     _fields_ = [("n", C.c_int64), ("rowptr", C.POINTER(C.c_int64)), ("colidx", C.POINTER(C.c_int32)),
                 ("lu", C.POINTER(C.c_double)), ("diag", C.POINTER(C.c_int64))]
@@ -241,6 +245,35 @@ class Tiles:
         return y, counts
 
 
+    def sticky_state(self):
+        """Fresh state of the sticky (P:237 literal) variant: cur_t = TilePrec_t and the working
+        copy of every stored value in tile order (c-5 "sticky variant")."""
+        return StickyState(self)
+
+    def spmv_sticky(self, state, x, level, range_guard=True):
+        """One SpMV of the sticky variant; lowers `state` in place.  Returns (y, counts)."""
+        x = _f64(x)
+        y = np.empty(self.n_rows, np.float64)
+        counts = np.zeros(5, np.int64)
+        lv = np.ascontiguousarray(level, np.uint8)
+        lib().orc_spmv_tiles(C.byref(self._s), _vp(x), _vp(y), _vp(lv), int(range_guard),
+                             C.cast(C.pointer(state._s), C.c_void_p), _vp(counts))
+        return y, counts
+
+
+class StickyState:
+    def __init__(self, A: "Tiles"):
+        arr = A.arrays()
+        self.cur = arr["TilePrec"].copy()
+        tn = arr["TileNnz"]
+        self.wv = np.empty(max(int(tn[-1]), 1), np.float64)
+        for t in range(A.tilenum):
+            for a in range(int(tn[t + 1] - tn[t])):
+                self.wv[tn[t] + a] = A.tile_value(t, a)
+        self._s = _Sticky(self.cur.ctypes.data_as(C.POINTER(C.c_uint8)),
+                          self.wv.ctypes.data_as(C.POINTER(C.c_double)))
+
+
 class OracleError(RuntimeError):
     def __init__(self, status):
         super().__init__(f"oracle status {status}")
@@ -311,8 +344,9 @@ class ILU0:
 
 # ------------------------------------------------------------------ solvers
 def _opts(tol, max_iter, mode, switch_eps, switch_absolute, sticky, range_guard):
-    # default eps = 1e-2 * tol (reading R8)
-    return _Opts(tol, max_iter, mode, 1e-2 * tol if switch_eps is None else switch_eps,
+    # default eps = tol: the convergence threshold of P:174 is the stop tolerance of P:264
+    # (reading R8)
+    return _Opts(tol, max_iter, mode, tol if switch_eps is None else switch_eps,
                  int(switch_absolute), int(sticky), int(range_guard))
 
 

@@ -518,8 +518,8 @@ double orc_dot(const double* u, const double* v, int64_t n, const orc_plan* plan
 /* ------------------------------------------------------------------------------------
  * 7. Solvers.  CG = Alg. 1 in canonical order (SURVEY c-3); BiCGSTAB = Alg. 2
  *    with the sign of s corrected (c-8 #12).  Stop on ||r||/||b|| < tol (c-8 #8),
- *    max_iter.  Switch thresholds tau = switch_eps * ||v0|| / sqrt(n) (v0 = first SpMV
- *    input; reading R8) or tau = switch_eps when switch_absolute (Alg. 1 l.3 literal).
+ *    max_iter.  Switch thresholds tau = switch_eps * ||v0||_2 (v0 = first SpMV input;
+ *    reading R8) or tau = switch_eps when switch_absolute (Alg. 1 l.3 literal).
  * ---------------------------------------------------------------------------------- */
 enum { MODE_FP64 = 0, MODE_STATIC = 1, MODE_DYNAMIC = 2 };
 
@@ -546,11 +546,13 @@ typedef struct {
     int64_t* level_counts; int64_t lc_cap; int64_t n_spmv;
 } orc_ctx;
 
-/* tau (reading R8 in DESIGN.md): eps times the RMS magnitude of the first SpMV input v0,
- * tau = (switch_eps * ||v0||_2) / sqrt(n); switch_absolute: tau = switch_eps (Alg. 1 l.3). */
+/* tau (reading R8 in DESIGN.md; SURVEY c-5): P:174 compares the entries of p_j with "the
+ * convergence threshold eps"; the stop test is relative, ||r|| < eps ||b||, so in the
+ * units of the SpMV input the threshold is eps times the norm of the first SpMV input v0
+ * (= ||b|| for CG with x0 = 0):  tau = switch_eps * ||v0||_2;  switch_absolute: tau = switch_eps
+ * (Alg. 1 l.3 literal).  Default switch_eps = tol. */
 static void ctx_set_tau(orc_ctx* c, double vnorm) {
-    double tau = c->o->switch_absolute ? c->o->switch_eps
-                                       : (c->o->switch_eps * vnorm) / sqrt((double)c->A->n_cols);
+    double tau = c->o->switch_absolute ? c->o->switch_eps : c->o->switch_eps * vnorm;
     c->th[0] = tau * 1e-3; c->th[1] = tau * 1e-2; c->th[2] = tau * 1e-1; c->th[3] = tau;
 }
 

@@ -209,7 +209,8 @@ __device__ __forceinline__ void flush_counts(const SolveArgs& a, Ctx& c, Counts&
 }
 
 __device__ __forceinline__ Thresh make_thresh(const SolveArgs& a, double v0norm) {
-    const double tau = a.switch_abs ? a.switch_eps : __ddiv_rn(__dmul_rn(a.switch_eps, v0norm), sqrt((double)a.n));
+    // reading R8: tau = eps * ||v0||_2 (P:174 threshold in the units of the SpMV input, P:264 relative stop test)
+    const double tau = a.switch_abs ? a.switch_eps : __dmul_rn(a.switch_eps, v0norm);
     return Thresh{__dmul_rn(tau, 1e-3), __dmul_rn(tau, 1e-2), __dmul_rn(tau, 1e-1), tau};
 }
 
@@ -1244,7 +1245,7 @@ mf_status run_solve(const TileMatrix& A, bool bicg, const double* b, double* x, 
     a.rh = rh; a.s = sv; a.th_g = th_g; a.lev_s = lev_s;
     a.slots = slots; a.bar = sync; a.abort_flag = reinterpret_cast<int*>(sync + 1); a.flags = sync + 2;
     a.bar_ns = bar_ns; a.phase_ns = phase_ns; a.hist = hist; a.hist_cap = hist_cap; a.lcounts = lcounts; a.lc_cap = count ? lc_cap : 0;
-    a.out = out; a.tol = o.tol; a.switch_eps = o.switch_eps < 0 ? 1e-2 * o.tol : o.switch_eps;   // reading R8
+    a.out = out; a.tol = o.tol; a.switch_eps = o.switch_eps < 0 ? o.tol : o.switch_eps;   // reading R8: eps = tol
     a.switch_abs = o.switch_absolute; a.range_guard = o.range_guard; a.max_iter = o.max_iter;
     a.mu_cap = (int)cap; a.timeout_ns = 60ull * 1000000000ull;
     double *pz = nullptr, *psh = nullptr;

@@ -215,8 +215,8 @@ class DistMatrix:
 
 
 def thresholds(switch_eps: float, v0norm: float, n: int, absolute: bool = False):
-    """Alg. 4 thresholds with reading R8: tau = eps * ||v0|| / sqrt(n)."""
-    tau = switch_eps if absolute else (switch_eps * v0norm) / math.sqrt(float(n))
+    """Alg. 4 thresholds with reading R8: tau = eps * ||v0||_2."""
+    tau = switch_eps if absolute else switch_eps * v0norm
     return np.array([tau * 1e-3, tau * 1e-2, tau * 1e-1, tau], np.float64)
 
 
@@ -238,7 +238,7 @@ def cg_solve(D: DistMatrix, b_local, tol=1e-10, max_iter=1000, mode="dynamic", s
     if nb == 0.0:
         return DistResult(x, 0, True, 0.0, np.zeros(1), row_begin=D.row_begin, row_end=D.row_end)
     p.copy_(r)
-    eps = 1e-2 * tol if switch_eps is None else switch_eps
+    eps = tol if switch_eps is None else switch_eps
     th = thresholds(eps, math.sqrt(rho), D.n) if mode == "dynamic" else None
     converged, status, j = False, "ok", 0
     while True:
