@@ -128,6 +128,8 @@ typedef struct {
     int32_t collect_stats;      /* 1: count tiles / nonzeros per effective precision in every SpMV
                                    (exact dynamic byte model; costs ALU in the SpMV loop).
                                    Implied when tile_level_counts != NULL. */
+    int32_t watchdog_ms;        /* spin watchdog of the grid barriers / ready flags / SpTRSV (0 = 60000 ms);
+                                   expiry returns MF_ERR_DEADLOCK */
 } mf_solve_opts;
 
 typedef struct {
@@ -141,6 +143,8 @@ typedef struct {
     int64_t launches;          /* kernels launched by the solve */
     double barrier_ms;         /* mean over CTAs of time spent spinning in grid barriers / ready flags */
     double phase_ms[12];       /* mean over CTAs of time per kernel phase */
+    int32_t ring_slots;        /* TMA ring depth of the SpMV (tile-synchronous layout) */
+    int32_t mu_onchip;         /* 1: the SpMV outputs stayed in shared memory across the barrier */
 } mf_solve_info;
 
 void mf_default_convert_opts(mf_convert_opts* o);

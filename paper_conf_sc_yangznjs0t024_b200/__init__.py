@@ -106,14 +106,15 @@ class SolveOpts(C.Structure):
     _fields_ = [("tol", C.c_double), ("max_iter", C.c_int64), ("mode", C.c_int32), ("switch_eps", C.c_double),
                 ("switch_absolute", C.c_int32), ("sticky", C.c_int32), ("range_guard", C.c_int32),
                 ("M", C.c_void_p), ("residual_history", C.c_void_p), ("history_cap", C.c_int64),
-                ("tile_level_counts", C.c_void_p), ("level_counts_cap", C.c_int64), ("collect_stats", C.c_int32)]
+                ("tile_level_counts", C.c_void_p), ("level_counts_cap", C.c_int64), ("collect_stats", C.c_int32),
+                ("watchdog_ms", C.c_int32)]
 
 
 class SolveInfo(C.Structure):
     _fields_ = [("iterations", C.c_int64), ("converged", C.c_int32), ("status", C.c_int32),
                 ("rel_residual", C.c_double), ("kernel_ms", C.c_double), ("model_bytes", C.c_double),
                 ("n_spmv", C.c_int64), ("launches", C.c_int64), ("barrier_ms", C.c_double),
-                ("phase_ms", C.c_double * 12)]
+                ("phase_ms", C.c_double * 12), ("ring_slots", C.c_int32), ("mu_onchip", C.c_int32)]
 
 
 _lib = None

@@ -389,13 +389,13 @@ __global__ void max2_kernel(const int64_t* __restrict__ a, const int64_t* __rest
 }
 
 // Stages of the TMA pipeline (kernels.cuh): one warp per CTA of the plan walks its tile rows and
-// cuts them greedily into stages within the caps (tile rows, slice columns, value bytes), each
-// a whole number of H-row groups when one fits, so that every half-warp gets the same number of
-// tile rows per stage.  COUNT pass: stages per CTA; FILL pass: the records.
+// cuts them greedily into stages within the caps (tile rows <= kcap, slice columns, value bytes),
+// each a whole number of H-row groups when one fits, so that every half-warp gets the same number
+// of tile rows per stage.  COUNT pass: stages per CTA; FILL pass: the records (tr0, tr1, nc).
 template <bool FILL>
-__global__ void stage_kernel(const int32_t* __restrict__ plan_tr, int G, int H, const int64_t* __restrict__ tr_slot,
+__global__ void stage_kernel(const int32_t* __restrict__ plan_tr, int G, int H, int kcap, const int64_t* __restrict__ tr_slot,
                              const int64_t* __restrict__ tr_vb, int32_t* nst, const int32_t* __restrict__ sptr,
-                             mfk::PipeStage* stg) {
+                             mfk::TsStage* stg) {
     const int g = blockIdx.x;
     const int lane = threadIdx.x & 31;
     if (g >= G) return;
@@ -405,11 +405,11 @@ __global__ void stage_kernel(const int32_t* __restrict__ plan_tr, int G, int H, 
     int32_t k = 0;
     while (S < tr1) {
         const int64_t c0 = tr_slot[S], v0 = tr_vb[S];
-        const int64_t lim = min(S + (int64_t)mfk::PIPE_KCAP, tr1);
+        const int64_t lim = min(S + (int64_t)kcap, tr1);
         int64_t emax = S;
         for (int64_t e0 = S + 1; e0 <= lim; e0 += 32) {
             const int64_t E = e0 + lane;
-            const bool fit = E <= lim && tr_slot[E] - c0 <= mfk::PIPE_CCAP && tr_vb[E] - v0 <= mfk::PIPE_VCAP;
+            const bool fit = E <= lim && tr_slot[E] - c0 <= mfk::TS_CCAP && tr_vb[E] - v0 <= mfk::TS_VCAP;
             const int nfit = __popc(__ballot_sync(0xffffffffu, fit));     // fits are a prefix (monotone)
             if (nfit > 0) emax = e0 + nfit - 1;
             if (nfit < 32) break;
@@ -418,9 +418,9 @@ __global__ void stage_kernel(const int32_t* __restrict__ plan_tr, int G, int H, 
         const int64_t grp = tr0 + ((emax - tr0) / H) * H;
         const int64_t E = grp > S ? grp : emax;
         if (FILL && lane == 0) {
-            mfk::PipeStage st{};
-            st.col0 = c0; st.col1 = tr_slot[E];
+            mfk::TsStage st{};
             st.tr0 = (int32_t)S; st.tr1 = (int32_t)E;
+            st.nc = (int32_t)(tr_slot[E] - c0);
             stg[base + k] = st;
         }
         ++k;
@@ -429,92 +429,187 @@ __global__ void stage_kernel(const int32_t* __restrict__ plan_tr, int G, int H, 
     if (!FILL && lane == 0) nst[g] = k;
 }
 
-// Blob of each stage (layout in kernels.cuh): its byte size (from the record), then, after an
-// exclusive scan of the sizes, its contents: headers, column words, local columns, the group
-// permutation and the values grouped by TilePrec.  One block of PIPE_CCAP threads per stage:
-// thread c owns column c of the stage.
-__device__ __forceinline__ void blob_layout(int K, int64_t nc, int64_t nv, int* off_cw, int* off_ss, int* off_dst, int* off_val, int* bytes) {
-    *off_cw = mfk::pipe_r16((K + 1) * 4);
-    *off_ss = *off_cw + mfk::pipe_r16((int)nc * 4);
-    *off_dst = *off_ss + (int)nc * 16;
-    *off_val = *off_dst + mfk::pipe_r16((int)nc * 2);
-    *bytes = *off_val + (int)nv;
+// Window runs of each stage: the distinct tile columns its tiles gather, sorted, cut into runs of
+// consecutive column segments (gaps of <= RUN_GAP segments are bridged: one bulk copy instead of
+// two), merged down to TS_RUNCAP runs by bridging the smallest gaps.  One block per stage.
+constexpr int RUN_GAP = 2;
+constexpr int RUNS_T = 1024;
+__global__ void __launch_bounds__(RUNS_T) runs_kernel(mfk::TsStage* stg, const int64_t* __restrict__ TileRowPtr,
+                                                      const int32_t* __restrict__ TileColidx, unsigned long long* maxw) {
+    __shared__ int32_t key[RUNS_T];
+    __shared__ int32_t rs[RUNS_T], rn[RUNS_T];
+    const int t = threadIdx.x;
+    mfk::TsStage st = stg[blockIdx.x];
+    const int64_t a = TileRowPtr[st.tr0], b = TileRowPtr[st.tr1];
+    const int nt = (int)(b - a);                          // <= TS_CCAP (a tile owns >= 1 slice column)
+    key[t] = t < nt ? TileColidx[a + t] : INT32_MAX;
+    __syncthreads();
+    for (int k = 2; k <= RUNS_T; k <<= 1)                 // bitonic sort
+        for (int j = k >> 1; j > 0; j >>= 1) {
+            const int ix = t ^ j;
+            if (ix > t) {
+                const int32_t x = key[t], y = key[ix];
+                if (((t & k) == 0) == (x > y)) { key[t] = y; key[ix] = x; }
+            }
+            __syncthreads();
+        }
+    if (t == 0) {
+        int nr = 0;
+        for (int i = 0; i < nt; ++i) {
+            const int32_t c = key[i];
+            if (nr > 0 && c <= rs[nr - 1] + rn[nr - 1] + RUN_GAP) {
+                if (c >= rs[nr - 1] + rn[nr - 1]) rn[nr - 1] = c - rs[nr - 1] + 1;
+            } else {
+                rs[nr] = c; rn[nr] = 1; ++nr;
+            }
+        }
+        while (nr > mfk::TS_RUNCAP) {                     // bridge the smallest gap
+            int best = 0;
+            int64_t bg = INT64_MAX;
+            for (int i = 0; i + 1 < nr; ++i) {
+                const int64_t gp = (int64_t)rs[i + 1] - (rs[i] + rn[i]);
+                if (gp < bg) { bg = gp; best = i; }
+            }
+            rn[best] = rs[best + 1] + rn[best + 1] - rs[best];
+            for (int i = best + 1; i + 1 < nr; ++i) { rs[i] = rs[i + 1]; rn[i] = rn[i + 1]; }
+            --nr;
+        }
+        int64_t w = 0;
+        for (int i = 0; i < mfk::TS_RUNCAP; ++i) {
+            st.run_s[i] = i < nr ? rs[i] : 0;
+            st.run_n[i] = i < nr ? rn[i] : 0;
+            st.run_w[i] = (int32_t)w;
+            if (i < nr) w += rn[i];
+        }
+        st.nrun = nr;
+        st.wseg = (int32_t)(w < (int64_t)INT32_MAX ? w : (int64_t)INT32_MAX);
+        stg[blockIdx.x] = st;
+        atomicMax(maxw, (unsigned long long)w);
+    }
 }
-__global__ void blob_size_kernel(const mfk::PipeStage* __restrict__ stg, int64_t n, const int64_t* __restrict__ tr_vb, int64_t* sz) {
+
+// Blob of each stage (layout in kernels.cuh): its byte size, then, after an exclusive scan of the
+// sizes, its contents.  One block of TS_CCAP threads per stage: thread c owns column c.
+struct BlobLayout {
+    int off_eb, off_desc, off_lc, off_wl, off_ent, off_val, bytes;
+};
+__host__ __device__ __forceinline__ BlobLayout blob_layout(int K, int64_t nc, int64_t nv, int NW) {
+    BlobLayout L;
+    L.off_eb = mfk::TS_HDR + mfk::ts_r16((K + 1) * 2);
+    L.off_desc = L.off_eb + mfk::ts_r16(K);
+    L.off_lc = L.off_desc + mfk::ts_r16(((int)nc + mfk::TS_DPAD) * 4);
+    L.off_wl = L.off_lc + ((int)nc + mfk::TS_DPAD) * 16;
+    L.off_ent = L.off_wl + mfk::ts_r16(NW * 4) + mfk::ts_r16(NW * 2);
+    L.off_val = L.off_ent + mfk::ts_r16((int)nc * 2);
+    L.bytes = L.off_val + (int)nv;
+    return L;
+}
+__global__ void blob_size_kernel(const mfk::TsStage* __restrict__ stg, int64_t n, const int64_t* __restrict__ tr_vb, int NW,
+                                 int64_t* sz) {
     const int64_t s = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
     if (s >= n) return;
-    const mfk::PipeStage st = stg[s];
-    int a, b, c, d, bytes;
-    blob_layout(st.tr1 - st.tr0, st.col1 - st.col0, tr_vb[st.tr1] - tr_vb[st.tr0], &a, &b, &c, &d, &bytes);
-    sz[s] = bytes;
+    const mfk::TsStage st = stg[s];
+    sz[s] = blob_layout(st.tr1 - st.tr0, st.nc, tr_vb[st.tr1] - tr_vb[st.tr0], NW).bytes;
 }
-__global__ void __launch_bounds__(mfk::PIPE_CCAP) blob_fill_kernel(mfk::PipeStage* stg, const int64_t* __restrict__ boff,
-                                                                     const int64_t* __restrict__ tr_slot, const int64_t* __restrict__ tr_vb,
-                                                                     const uint2* __restrict__ crec, const uint8_t* __restrict__ sslot,
-                                                                     const uint8_t* __restrict__ vstream, uint8_t* blob) {
-    __shared__ int32_t hdr[mfk::PIPE_KCAP + 1];
-    __shared__ unsigned long long wsum[mfk::PIPE_CCAP / 32];
-    __shared__ int gtot[4];
+__device__ int owner_cta(const int32_t* plan_tr, int G, int64_t TR) {
+    int lo = 0, hi = G - 1;
+    while (lo < hi) { const int mid = (lo + hi + 1) / 2; if (plan_tr[mid] <= TR) lo = mid; else hi = mid - 1; }
+    return lo;
+}
+__global__ void __launch_bounds__(mfk::TS_CCAP) blob_fill_kernel(mfk::TsStage* stg, const int64_t* __restrict__ boff,
+                                                                   const int64_t* __restrict__ tr_slot, const int64_t* __restrict__ tr_vb,
+                                                                   const uint2* __restrict__ crec, const uint8_t* __restrict__ sslot,
+                                                                   const uint8_t* __restrict__ vstream, uint8_t* blob,
+                                                                   const int32_t* __restrict__ plan_tr, int G, int H,
+                                                                   unsigned long long* maxb) {
+    __shared__ int32_t hdr[mfk::TS_KCAP + 1];
+    __shared__ int32_t ebase[mfk::TS_KCAP];       // first E slot of each tile row within its warp's buffer
+    __shared__ int32_t wcols[32], woffs[33];      // columns per warp, list offsets
     const int64_t sidx = blockIdx.x;
-    mfk::PipeStage st = stg[sidx];
+    const mfk::TsStage st = stg[sidx];
     const int K = st.tr1 - st.tr0, c = threadIdx.x;
-    const int nc = (int)(st.col1 - st.col0);
-    const int64_t nv = tr_vb[st.tr1] - tr_vb[st.tr0];
-    int off_cw, off_ss, off_dst, off_val, bytes;
-    blob_layout(K, nc, nv, &off_cw, &off_ss, &off_dst, &off_val, &bytes);
+    const int nc = st.nc, NW = H / 2 > 1 ? H / 2 : 1;   // warps = B / 32 = H / 2
+    const int64_t col0 = tr_slot[st.tr0];
+    const int64_t vb0 = tr_vb[st.tr0], nv = tr_vb[st.tr1] - vb0;
+    const BlobLayout L = blob_layout(K, nc, nv, NW);
+    const int64_t tr0c = plan_tr[owner_cta(plan_tr, G, st.tr0)];
     uint8_t* b = blob + boff[sidx];
     for (int k = c; k <= K; k += blockDim.x) {
-        hdr[k] = (int32_t)(tr_slot[st.tr0 + k] - st.col0);
-        reinterpret_cast<int32_t*>(b)[k] = hdr[k];
-    }
-    uint2 rc = make_uint2(0u, 0u);
-    int q = 0;
-    if (c < nc) {
-        rc = crec[st.col0 + c];
-        q = (int)(rc.x & 3u);
-        reinterpret_cast<uint32_t*>(b + off_cw)[c] = rc.x;
-        reinterpret_cast<uint4*>(b + off_ss)[c] = reinterpret_cast<const uint4*>(sslot)[st.col0 + c];
-    }
-    // rank of column c within its precision group: block exclusive scan of 4 packed 16-bit counters
-    const unsigned long long one = c < nc ? 1ull << (16 * q) : 0ull;
-    unsigned long long incl = one;
-    const int lane = c & 31, w = c >> 5;
-    for (int o = 1; o < 32; o <<= 1) { const unsigned long long u = __shfl_up_sync(0xffffffffu, incl, o); if (lane >= o) incl += u; }
-    if (lane == 31) wsum[w] = incl;
-    __syncthreads();
-    unsigned long long wpre = 0;
-    for (int k = 0; k < w; ++k) wpre += wsum[k];
-    const unsigned long long excl = wpre + incl - one;
-    if (c == (int)blockDim.x - 1) {
-        const unsigned long long tot = wpre + incl;
-        for (int k = 0; k < 4; ++k) gtot[k] = (int)((tot >> (16 * k)) & 0xFFFFull);
+        hdr[k] = (int32_t)(tr_slot[st.tr0 + k] - col0);
+        reinterpret_cast<int16_t*>(b + mfk::TS_HDR)[k] = (int16_t)hdr[k];
     }
     __syncthreads();
-    int gbase[4], goff[4];
-    {
-        int cols = 0, off = off_val;
-        for (int k = 0; k < 4; ++k) { gbase[k] = cols; goff[k] = off; cols += gtot[k]; off += gtot[k] * 16 * (8 >> k); }
-    }
-    if (c < nc) {
-        const int rank = (int)((excl >> (16 * q)) & 0xFFFFull);
-        reinterpret_cast<uint16_t*>(b + off_dst)[gbase[q] + rank] = (uint16_t)c;
-        // tile row of column c, then its values (16 x size(TilePrec) bytes) into its group
-        int lo = 0, hi = K - 1;
-        while (lo < hi) { const int mid = (lo + hi + 1) / 2; if (hdr[mid] <= c) lo = mid; else hi = mid - 1; }
-        const int64_t src = tr_vb[st.tr0 + lo] + rc.y;
-        const int n16 = 8 >> q;                 // 16-byte chunks per column
-        const uint4* sp = reinterpret_cast<const uint4*>(vstream + src);
-        uint4* dp = reinterpret_cast<uint4*>(b + goff[q] + (int64_t)rank * 16 * (8 >> q));
-        for (int k = 0; k < n16; ++k) dp[k] = sp[k];
-    }
     if (c == 0) {
-        stg[sidx].boff = boff[sidx];
-        stg[sidx].bbytes = bytes;
-        stg[sidx].off_cw = off_cw;
-        stg[sidx].off_ss = off_ss;
-        stg[sidx].off_dst = off_dst;
-        stg[sidx].off_val = off_val;
-        for (int k = 0; k < 4; ++k) { stg[sidx].gcnt[k] = gtot[k]; stg[sidx].goff[k] = goff[k]; }
+        // own window segment: tile column tr0 if [tr0, tr1) lies inside one run, else -1
+        int own = -1;
+        for (int i = 0; i < st.nrun; ++i)
+            if (st.run_s[i] <= st.tr0 && st.tr1 <= st.run_s[i] + st.run_n[i]) own = st.run_w[i] + (st.tr0 - st.run_s[i]);
+        int32_t* h = reinterpret_cast<int32_t*>(b);
+        h[0] = st.tr0; h[1] = st.tr1; h[2] = nc; h[3] = L.off_desc; h[4] = L.off_lc; h[5] = L.off_val; h[6] = own;
+        h[7] = (int32_t)(uint32_t)(uint64_t)col0; h[8] = (int32_t)(uint32_t)((uint64_t)col0 >> 32);
+        h[9] = L.off_wl; h[10] = L.off_ent; h[11] = L.off_eb;
+        for (int k = 12; k < 16; ++k) h[k] = 0;
+        // E slots: the columns of a warp's tile rows (half-warps 2w, 2w+1), in column order
+        for (int w = 0; w < NW; ++w) wcols[w] = 0;
+        for (int k = 0; k < K; ++k) {
+            const int w = (int)((st.tr0 + k - tr0c) % H) >> 1;
+            ebase[k] = wcols[w];
+            b[L.off_eb + k] = (uint8_t)min(wcols[w], 255);
+            wcols[w] += hdr[k + 1] - hdr[k];
+        }
+        woffs[0] = 0;
+        int mx = 0;
+        for (int w = 0; w < NW; ++w) { woffs[w + 1] = woffs[w] + wcols[w]; mx = max(mx, wcols[w]); }
+        atomicMax(maxb + 1, (unsigned long long)mx);
+    }
+    __syncthreads();
+    if (c < nc) {
+        const uint2 rc = crec[col0 + c];
+        const uint32_t tc = rc.x >> 4;
+        int lo = 0, hi = K - 1;                              // tile row of column c
+        while (lo < hi) { const int mid = (lo + hi + 1) / 2; if (hdr[mid] <= c) lo = mid; else hi = mid - 1; }
+        const int64_t voff = tr_vb[st.tr0 + lo] - vb0 + rc.y;   // column order == vstream order
+        int wseg = 0;
+        for (int i = 0; i < st.nrun; ++i)
+            if ((int64_t)tc >= st.run_s[i] && (int64_t)tc < (int64_t)st.run_s[i] + st.run_n[i]) wseg = st.run_w[i] + (int)(tc - st.run_s[i]);
+        reinterpret_cast<uint32_t*>(b + L.off_desc)[c] =
+            (rc.x & 15u) | ((uint32_t)(voff >> 4) << 4) | ((uint32_t)(wseg * mfk::PV_SEG_BYTES) << 16);
+        uint4 l16 = reinterpret_cast<const uint4*>(sslot)[col0 + c];      // local columns, stored x8 (byte offsets)
+        l16.x <<= 3; l16.y <<= 3; l16.z <<= 3; l16.w <<= 3;
+        reinterpret_cast<uint4*>(b + L.off_lc)[c] = l16;
+    }
+    if (c < mfk::TS_DPAD) {                                // padding read by short rows
+        reinterpret_cast<uint32_t*>(b + L.off_desc)[nc + c] = 0u;
+        reinterpret_cast<uint4*>(b + L.off_lc)[nc + c] = make_uint4(0u, 0u, 0u, 0u);
+    }
+    if (c < NW) {
+        // decode list of warp c: its columns grouped by TilePrec (FP64 | FP32 | FP16 | E4M3), ascending
+        const int w = c;
+        uint32_t cnt = 0;
+        uint16_t* ent = reinterpret_cast<uint16_t*>(b + L.off_ent) + woffs[w];
+        int pos = 0;
+        for (int q = 0; q < 4; ++q) {
+            int nq = 0;
+            for (int k = 0; k < K; ++k) {
+                if (((int)((st.tr0 + k - tr0c) % H) >> 1) != w) continue;
+                for (int cc = hdr[k]; cc < hdr[k + 1]; ++cc)
+                    if ((int)(crec[col0 + cc].x & 3u) == q) {
+                        ent[pos++] = (uint16_t)(cc | ((ebase[k] + cc - hdr[k]) << 9));   // column | E slot << 9
+                        ++nq;
+                    }
+            }
+            cnt |= (uint32_t)min(nq, 255) << (8 * q);
+        }
+        reinterpret_cast<uint32_t*>(b + L.off_wl)[w] = cnt;
+        reinterpret_cast<uint16_t*>(b + L.off_wl + mfk::ts_r16(NW * 4))[w] = (uint16_t)woffs[w];
+    }
+    for (int64_t k = c; k < nv / 16; k += blockDim.x)
+        reinterpret_cast<uint4*>(b + L.off_val)[k] = reinterpret_cast<const uint4*>(vstream + vb0)[k];
+    if (c == 0) {
+        stg[sidx].boff_lo = (uint32_t)(uint64_t)boff[sidx];
+        stg[sidx].boff_hi = (uint32_t)((uint64_t)boff[sidx] >> 32);
+        stg[sidx].bbytes = L.bytes;
+        atomicMax(maxb, (unsigned long long)L.bytes);
     }
 }
 
@@ -602,7 +697,7 @@ mf_status convert_csr(int64_t n_rows, int64_t n_cols, int64_t nnz, const int64_t
         MF_CUDA(cudaStreamSynchronize(s));
         dev_free(dmx, s);
     }
-    const bool ts_fits = mx[0] <= (unsigned long long)mfk::PIPE_CCAP && mx[1] <= (unsigned long long)mfk::PIPE_VCAP;
+    const bool ts_fits = mx[0] <= (unsigned long long)mfk::TS_CCAP && mx[1] <= (unsigned long long)mfk::TS_VCAP;
     if (o.layout == 1) A->ts = 0;
     else if (o.layout == 2) A->ts = ts_fits ? 1 : 0;
     else A->ts = ts_fits && (double)tot[CNT_WTS] <= 1.6 * (double)tot[CNT_WIDTH] ? 1 : 0;
@@ -695,46 +790,85 @@ mf_status convert_csr(int64_t n_rows, int64_t n_cols, int64_t nnz, const int64_t
     deps_kernel<<<G, 256, 0, s>>>(A->plan_tr, G, A->TileRowPtr, A->TileColidx, ntr, A->dep_lo, A->dep_hi, A->seg_lo,
                                   A->seg_hi);
     MF_CUDA(cudaGetLastError());
-    if (A->ts) {   // pipeline stages of every CTA (two passes: count, fill)
+    bool ts_failed = false;
+    if (A->ts) {   // pipeline stages of every CTA (two passes: count, fill), their window runs
         int32_t* nst = nullptr;
+        unsigned long long* dmax = nullptr;
         MF_TRY(alloc(&nst, G, s));
-        stage_kernel<false><<<G, 32, 0, s>>>(A->plan_tr, G, B / 16, A->tr_slot, A->tr_vb, nst, nullptr, nullptr);
-        MF_CUDA(cudaGetLastError());
+        MF_TRY(alloc(&dmax, 3, s));
         std::vector<int32_t> nst_h(G), sp_h(G + 1);
-        MF_CUDA(cudaMemcpyAsync(nst_h.data(), nst, G * sizeof(int32_t), cudaMemcpyDeviceToHost, s));
-        MF_CUDA(cudaStreamSynchronize(s));
-        sp_h[0] = 0;
-        for (int g = 0; g < G; ++g) sp_h[g + 1] = sp_h[g] + nst_h[g];
-        A->nstg = sp_h[G];
-        MF_TRY(alloc(&A->stg_ptr, G + 1, s));
-        MF_CUDA(cudaMemcpyAsync(A->stg_ptr, sp_h.data(), (G + 1) * sizeof(int32_t), cudaMemcpyHostToDevice, s));
-        mfk::PipeStage* stg = nullptr;
-        MF_TRY(alloc(&stg, std::max<int64_t>(A->nstg, 1), s));
-        A->stg = stg;
-        stage_kernel<true><<<G, 32, 0, s>>>(A->plan_tr, G, B / 16, A->tr_slot, A->tr_vb, nullptr, A->stg_ptr, stg);
-        MF_CUDA(cudaGetLastError());
-        // blobs: sizes -> offsets -> copies; the per-column source arrays are then released
-        if (A->nstg > 0) {
+        // the window of a stage grows with its tile rows: halve the stage cap until every
+        // stage's window fits TS_WCAP segments
+        // one tile row per half-warp per stage (K = H) keeps the warp-private decode buffers small
+        for (int kcap = std::min(mfk::TS_KCAP, std::max(1, B / 16));; kcap /= 2) {
+            stage_kernel<false><<<G, 32, 0, s>>>(A->plan_tr, G, B / 16, kcap, A->tr_slot, A->tr_vb, nst, nullptr, nullptr);
+            MF_CUDA(cudaGetLastError());
+            MF_CUDA(cudaMemcpyAsync(nst_h.data(), nst, G * sizeof(int32_t), cudaMemcpyDeviceToHost, s));
+            MF_CUDA(cudaStreamSynchronize(s));
+            sp_h[0] = 0;
+            for (int g = 0; g < G; ++g) sp_h[g + 1] = sp_h[g] + nst_h[g];
+            A->nstg = sp_h[G];
+            if (A->stg_ptr) dev_free(A->stg_ptr, s);
+            if (A->stg) dev_free(A->stg, s);
+            A->stg_ptr = nullptr; A->stg = nullptr;
+            MF_TRY(alloc(&A->stg_ptr, G + 1, s));
+            MF_CUDA(cudaMemcpyAsync(A->stg_ptr, sp_h.data(), (G + 1) * sizeof(int32_t), cudaMemcpyHostToDevice, s));
+            mfk::TsStage* stg = nullptr;
+            MF_TRY(alloc(&stg, std::max<int64_t>(A->nstg, 1), s));
+            A->stg = stg;
+            stage_kernel<true><<<G, 32, 0, s>>>(A->plan_tr, G, B / 16, kcap, A->tr_slot, A->tr_vb, nullptr, A->stg_ptr, stg);
+            MF_CUDA(cudaMemsetAsync(dmax, 0, 3 * sizeof(unsigned long long), s));
+            if (A->nstg > 0) runs_kernel<<<(unsigned)A->nstg, RUNS_T, 0, s>>>(stg, A->TileRowPtr, A->TileColidx, dmax);
+            MF_CUDA(cudaGetLastError());
+            unsigned long long mw = 0;
+            MF_CUDA(cudaMemcpyAsync(&mw, dmax, sizeof(mw), cudaMemcpyDeviceToHost, s));
+            MF_CUDA(cudaStreamSynchronize(s));   // sp_h (pageable) consumed
+            A->wcap = (int32_t)std::min<unsigned long long>(mw, 1ull << 30);
+            if (mw <= (unsigned long long)mfk::TS_WCAP) break;
+            if (kcap == 1) { ts_failed = true; break; }
+        }
+        // blobs: sizes -> offsets -> contents; the per-column source arrays are then released
+        if (!ts_failed && A->nstg > 0) {
             int64_t *bsz = nullptr, *boff = nullptr, *btmp = nullptr;
             MF_TRY(alloc(&bsz, A->nstg, s));
             MF_TRY(alloc(&boff, A->nstg + 1, s));
             MF_TRY(alloc(&btmp, A->nstg / 2048 + 2, s));
-            blob_size_kernel<<<(unsigned)((A->nstg + 255) / 256), 256, 0, s>>>(stg, A->nstg, A->tr_vb, bsz);
+            blob_size_kernel<<<(unsigned)((A->nstg + 255) / 256), 256, 0, s>>>(static_cast<mfk::TsStage*>(A->stg), A->nstg, A->tr_vb,
+                                                                              B / 32, bsz);
             MF_TRY(scan_excl(bsz, A->nstg, boff, btmp, s));
             MF_CUDA(cudaMemcpyAsync(&A->blob_bytes, boff + A->nstg, sizeof(int64_t), cudaMemcpyDeviceToHost, s));
             MF_CUDA(cudaStreamSynchronize(s));
             MF_TRY(alloc(&A->blob, A->blob_bytes + 64, s));
-            blob_fill_kernel<<<(unsigned)A->nstg, mfk::PIPE_CCAP, 0, s>>>(stg, boff, A->tr_slot, A->tr_vb, A->crec, A->sslot,
-                                                                         A->vstream, A->blob);
+            blob_fill_kernel<<<(unsigned)A->nstg, mfk::TS_CCAP, 0, s>>>(static_cast<mfk::TsStage*>(A->stg), boff, A->tr_slot, A->tr_vb, A->crec, A->sslot,
+                                                                       A->vstream, A->blob, A->plan_tr, G, B / 16, dmax + 1);
             MF_CUDA(cudaGetLastError());
+            unsigned long long mb[2] = {0, 0};
+            MF_CUDA(cudaMemcpyAsync(mb, dmax + 1, sizeof(mb), cudaMemcpyDeviceToHost, s));
+            MF_CUDA(cudaStreamSynchronize(s));
+            A->blob_cap = (int32_t)((mb[0] + 127) / 128 * 128);
+            A->ecap = (int32_t)mb[1];
+            // the warp-private decode buffers must leave room for the ring (TS_EBYTES of shared memory)
+            if ((int64_t)A->ecap * 128 * (B / 32) > mfk::TS_EBYTES || A->ecap > 127) ts_failed = true;
+            A->slot_bytes = (int32_t)((A->blob_cap + (int64_t)A->wcap * mfk::PV_SEG_BYTES + 127) / 128 * 128);
             dev_free(bsz, s); dev_free(boff, s); dev_free(btmp, s);
         }
-        MF_CUDA(cudaStreamSynchronize(s));   // sp_h (pageable) consumed
         dev_free(nst, s);
+        dev_free(dmax, s);
         dev_free(A->sslot, s); A->sslot = nullptr;
         dev_free(A->crec, s); A->crec = nullptr;
         dev_free(A->vstream, s); A->vstream = nullptr;
         dev_free(A->tr_vb, s); A->tr_vb = nullptr;
+    }
+    if (ts_failed) {
+        // a stage of a single tile row gathers more than TS_WCAP column segments: this pattern
+        // is not tile-synchronous enough -- convert again with the compact layout
+        cudaEventDestroy(e0);
+        cudaEventDestroy(e1);
+        dev_free(cost, s); dev_free(cnt, s); dev_free(off, s); dev_free(tmp, s); dev_free(d_err, s);
+        destroy_tiles(A);
+        mf_convert_opts o2 = o;
+        o2.layout = 1;
+        return convert_csr(n_rows, n_cols, nnz, rowptr, colidx, vals, o2, s, A);
     }
     std::vector<int32_t> ptr_h(G + 1);
     MF_CUDA(cudaMemcpyAsync(ptr_h.data(), A->plan_tr, (G + 1) * sizeof(int32_t), cudaMemcpyDeviceToHost, s));
@@ -753,7 +887,7 @@ mf_status convert_csr(int64_t n_rows, int64_t n_cols, int64_t nnz, const int64_t
     A->convert_launches = (n_rows > 0 ? 1 : 0) + (ntr > 0 ? 2 + 1 : 0) + (NCNT + 1) * (ntr > 0 ? 3 : 0) + 2;
     A->canonical_bytes = nt * (4 + 4 + 1 + 1 + 8 + 8 + 8) + 16 + (ntr + 1) * 8 + A->rownum * 2 + nnz +
                          A->nval[0] * 8 + A->nval[1] * 4 + A->nval[2] * 2 + A->nval[3];
-    A->kernel_bytes = (A->ts ? A->blob_bytes + A->nstg * (int64_t)sizeof(mfk::PipeStage) : nslot * 2) +
+    A->kernel_bytes = (A->ts ? A->blob_bytes + A->nstg * (int64_t)sizeof(mfk::TsStage) : nslot * 2) +
                       (A->plane64 ? nslot * 8 : 0) + (A->plane32 ? nslot * 4 : 0) +
                       (A->plane16 ? nslot * 2 : 0) + (A->plane8 ? nslot : 0) + nt * 4 + (ntr + 1) * 8;
     return MF_OK;

@@ -1,9 +1,9 @@
 // kernels.cuh -- device building blocks shared by the persistent solver kernels and the
 // standalone mf_spmv / mf_levels / mf_dot kernels.
 //
-//  * spmv_tile_row: Alg. 5 for one tile row, one half-warp, lane r = row 16*TR+r.
-//    Each row is ONE fma chain over its nonzeros in ascending column order (the slice layout
-//    stores them in that order), so no floating-point atomics are needed (Alg. 5 l.13's
+//  * spmv_ts / spmv_compact: Alg. 5.  A half-warp owns a tile row, lane r = row
+//    16*TR+r; each row is ONE fma chain over its nonzeros in ascending column order (the slice
+//    layouts store them in that order), so no floating-point atomics are needed (Alg. 5 l.13's
 //    atomicAdd disappears) and the result is bit-identical for any launch shape.
 //  * level_of / tile_code: Alg. 4 thresholds and the effective precision e_t.
 //  * Reductions: the fixed tree of DESIGN.md "Reduction order" (thread fma chain -> warp
@@ -14,8 +14,9 @@
 
 namespace mfk {
 
-constexpr int STAGE = 32;          // tile codes staged in smem per half-warp
 constexpr int BYP = 4;
+
+struct TsStage;
 
 struct Mat {
     int64_t n_rows, n_cols, ntr;
@@ -24,7 +25,7 @@ struct Mat {
     const uint32_t* __restrict__ tile_info;
     const uint16_t* __restrict__ sidx;    // compact layout
     const uint8_t* __restrict__ blob;     // tile-synchronous layout: per-stage blobs (the TMA source)
-    const struct PipeStage* __restrict__ stg;   // stages of every CTA
+    const TsStage* __restrict__ stg;      // stages of every CTA
     const int32_t* __restrict__ stg_ptr;  // [G+1]
     const int64_t* __restrict__ tile_nnz; // TileNnz (canonical)
     int ts;
@@ -35,7 +36,25 @@ struct Mat {
     const uint8_t* __restrict__ p8;
     uint8_t* stk;                         // sticky variant (P:237 literal): per slice column (TS layout) or
                                           // per tile (compact), bit L set = values lowered to L in place
+    int dbg;                              // diagnostics (MF_SPMV_DBG): 1 = stream the stages, skip the rows
 };
+
+// ------------------------------------------------------------------------------------------
+// SpMV input vectors ("PV" layout).  Every vector that feeds an SpMV inside the solver (p, s,
+// p^, s^) is stored as 16-element segments of 144 bytes: 16 binary64 values, then the segment's
+// level byte (Alg. 4: 0 FP64 .. 3 FP8, 4 bypass) in the low byte of element 16,
+// element 17 padding.  The producer of the vector (the CTA that owns the rows) writes the
+// level next to the values, so one bulk copy of a run of segments stages both the x values and
+// the tile-column levels of an SpMV stage (the "vis_flag" of Alg. 5 l.2) in shared memory.
+constexpr int PVS = 18;                      // doubles per segment
+constexpr int PV_SEG_BYTES = PVS * 8;        // 144
+__host__ __device__ __forceinline__ int64_t pv_idx(int64_t i) { return (i >> 4) * PVS + (i & 15); }
+__device__ __forceinline__ int pv_level(const double* pv, int64_t seg) {
+    return (int)reinterpret_cast<const uint8_t*>(pv + seg * PVS + 16)[0];
+}
+__device__ __forceinline__ void pv_set_level(double* pv, int64_t seg, int lv) {
+    reinterpret_cast<uint8_t*>(pv + seg * PVS + 16)[0] = (uint8_t)lv;
+}
 
 __device__ __forceinline__ unsigned hw_mask() { return (threadIdx.x & 16) ? 0xFFFF0000u : 0x0000FFFFu; }
 
@@ -44,11 +63,11 @@ __device__ __forceinline__ int hw_min_i(int v, unsigned m) { return (int)__reduc
 
 // (tile column << 3) | e_t.   e_t = bypass | max_prec(floor, min_prec(TilePrec, level))
 template <bool DYN>
-__device__ __forceinline__ uint32_t tile_code(uint32_t info, const uint8_t* __restrict__ level, int range_guard) {
+__device__ __forceinline__ uint32_t tile_code(uint32_t info, const double* pv, int range_guard) {
     const uint32_t tc = info >> 4;
     int e = (int)(info & 3u);
     if (DYN) {
-        const int lv = level[tc];
+        const int lv = pv_level(pv, tc);
         if (lv == BYP) return (tc << 3) | BYP;
         e = max(e, lv);
         if (range_guard) e = min(e, (int)((info >> 2) & 3u));
@@ -60,11 +79,11 @@ __device__ __forceinline__ uint32_t tile_code(uint32_t info, const uint8_t* __re
 // the tile was lowered to in place.  Code = (tile column << 3) | e_t | TilePrec << 27 | mask << 29
 // (mask bits L = 1..3 stored as mask >> 1; tile column < 2^24); `update` (the window's code staging, one thread per tile) records a new
 // lowering, the per-slot recomputation of an unstaged window only reads the updated mask.
-__device__ __forceinline__ uint32_t sticky_code(const Mat& A, int64_t tile, const uint8_t* __restrict__ level, int range_guard,
+__device__ __forceinline__ uint32_t sticky_code(const Mat& A, int64_t tile, const double* pv, int range_guard,
                                                 bool update) {
     const uint32_t info = A.tile_info[tile];
     const uint32_t tc = info >> 4, prec = info & 3u;
-    const int lv = level[tc];
+    const int lv = pv_level(pv, tc);
     if (lv == BYP) return (tc << 3) | BYP;
     unsigned mask = A.stk[tile];
     const int cur = mask ? 31 - __clz(mask) : (int)prec;
@@ -77,13 +96,6 @@ __device__ __forceinline__ uint32_t sticky_code(const Mat& A, int64_t tile, cons
     return (tc << 3) | (uint32_t)e | (prec << 27) | ((mask >> 1) << 29);   // mask bits 1..3
 }
 constexpr uint32_t CODE_TC_MASK = 0x00FFFFFFu;   // tile column field of a code (after >> 3)
-
-__device__ __forceinline__ double load_val(const Mat& A, int e, int64_t pos) {
-    if (e == 0) return A.p64[pos];
-    if (e == 1) return (double)A.p32[pos];
-    if (e == 2) return f16_to_d(A.p16[pos]);
-    return e4m3_to_d(A.p8[pos]);
-}
 
 // Per-thread tile / nonzero counters by effective precision (FP64..FP8, bypass), packed in
 // 21-bit fields so that a data-dependent index never turns into local-memory traffic.
@@ -106,177 +118,71 @@ struct Counts {
 };
 
 // ------------------------------------------------------------------------------------------
-// Compact (row-packed SELL-16) layout: windowed SpMV over the contiguous tile rows [tr0, tr1)
-// of one CTA (all B threads call it).  A window is up to WIN_TR tile rows (a multiple of
-// H = B/16 so that half-warp h always gets tile rows tr0 + h + kH, the row mapping of the
-// dot-product contract); per window the CTA stages the tile codes (tile column + e_t) of the
-// window's tiles in shared memory.  Used for matrices whose tile-synchronous slices would pad
-// too much (scattered patterns, e.g. C4); stencil matrices take the TMA pipeline below.
-constexpr int WIN_TR = 1024;
-constexpr int CODE_CAP = 8192;
-constexpr int WIN_BUF_BYTES = CODE_CAP * 4;
-
-struct WinSmem {
-    int32_t* hs;     // [WIN_TR+1] slot (slice column) offset of each tile row, relative to s0
-    int32_t* ht;     // [WIN_TR+1] tile offset, relative to t0
-    int64_t* misc;   // [4]: -, -, window end, staged
-    unsigned long long* pb;   // [4] value-plane base addresses (FP64, FP32, FP16, E4M3)
-    unsigned char* buf;   // [WIN_BUF_BYTES]: uint32 code[CODE_CAP]
-};
-constexpr size_t WIN_SMEM_BYTES = 2 * (WIN_TR + 1) * 4 + 4 * 8 + 8 + 4 * 8 + WIN_BUF_BYTES + 16;
-
-// Value fetch: ONE aligned 8-byte load from plane[e] + pos*size(e) (planes are 8-byte aligned and
-// padded), the needed bytes shifted down.  The 8-byte word lies in the same 32-byte DRAM sector
-// as the value, so this moves no extra HBM bytes; it replaces four predicated loads.
-__device__ __forceinline__ uint64_t load_raw(const unsigned long long* pbase, int e, int64_t pos) {
-    const unsigned long long a = pbase[e] + ((unsigned long long)pos << (3 - e));
-    const unsigned long long w = __ldg(reinterpret_cast<const unsigned long long*>(a & ~7ull));
-    return w >> ((a & 7ull) * 8);
-}
-// exact upcast of the stored bits at precision e (0 FP64, 1 FP32, 2 FP16, 3 E4M3) to binary64
-__device__ __forceinline__ double decode_val(int e, uint64_t raw) {
-    const uint32_t lo = (uint32_t)raw;
-    const __half_raw h8 = __nv_cvt_fp8_to_halfraw((__nv_fp8_storage_t)(lo & 0xFFu), __NV_E4M3);
-    const unsigned short hb = e == 3 ? h8.x : (unsigned short)lo;
-    const float f16 = __half2float(__ushort_as_half(hb));
-    const float f = e >= 2 ? f16 : __uint_as_float(lo);
-    const double d = (double)f;
-    return e == 0 ? __longlong_as_double((long long)raw) : d;
-}
-
-__device__ __forceinline__ void cp_async16(void* smem, const void* gmem) {
-    const unsigned sa = (unsigned)__cvta_generic_to_shared(smem);
-    asm volatile("cp.async.cg.shared.global [%0], [%1], 16;" ::"r"(sa), "l"(gmem) : "memory");
-}
-__device__ __forceinline__ void cp_async4(void* smem, const void* gmem) {
-    const unsigned sa = (unsigned)__cvta_generic_to_shared(smem);
-    asm volatile("cp.async.ca.shared.global [%0], [%1], 4;" ::"r"(sa), "l"(gmem) : "memory");
-}
-__device__ __forceinline__ void cp_async_wait_all() { asm volatile("cp.async.wait_all;" ::: "memory"); }
-
-// compact layout: process slot words s[0..cnt) of one lane; returns updated acc
-template <bool DYN, bool COUNT, int N>
-__device__ __forceinline__ double slot_block(const Mat& A, const unsigned long long* w_pb, const uint16_t (&s)[N], int cnt, int64_t pos0,
-                                             const uint32_t* code, bool staged, int64_t tb_abs,
-                                             const uint8_t* __restrict__ level, int range_guard,
-                                             const double* x, double acc, Counts* cntp) {
-    uint64_t raw[N];
-    double xv[N];
-    int ev[N];
-#pragma unroll
-    for (int q = 0; q < N; ++q) {
-        ev[q] = BYP;
-        raw[q] = 0;
-        xv[q] = 0.0;
-        if (q < cnt && s[q] != mf::SLOT_PAD) {
-            const int j = s[q] >> 4;
-            const uint32_t c = staged ? code[j]
-                               : (DYN && A.stk != nullptr) ? sticky_code(A, tb_abs + j, level, range_guard, false)
-                                                           : tile_code<DYN>(A.tile_info[tb_abs + j], level, range_guard);
-            ev[q] = (int)(c & 7u);
-            if (COUNT) cntp->nz(ev[q]);
-            if (ev[q] != BYP) {
-                // sticky: the stored value (plane TilePrec), lowered in slot_value below
-                raw[q] = load_raw(w_pb, (DYN && A.stk != nullptr) ? (int)((c >> 27) & 3u) : ev[q], pos0 + q * 16);
-                xv[q] = x[(int64_t)((c >> 3) & CODE_TC_MASK) * 16 + (s[q] & 15)];
-                if (DYN && A.stk != nullptr) ev[q] |= (int)(c >> 24) & 0xF8;   // TilePrec << 3 | (mask >> 1) << 5
-            }
-        }
-    }
-#pragma unroll
-    for (int q = 0; q < N; ++q)
-        if ((ev[q] & 7) != BYP) {
-            double v;
-            if (DYN && A.stk != nullptr) {   // successive RNE at every level the tile was lowered to
-                const int prec = (ev[q] >> 3) & 3, m1 = ev[q] >> 5;   // m1 bit L-1 = lowered to L
-                v = decode_val(prec, raw[q]);
-#pragma unroll
-                for (int L = 1; L <= 3; ++L)
-                    if (L > prec && (m1 & (1 << (L - 1)))) v = round_to(v, L);
-            } else {
-                v = decode_val(ev[q], raw[q]);
-            }
-            acc = __fma_rn(v, xv[q], acc);
-        }
-    return acc;
-}
-
-// ------------------------------------------------------------------------------------------
 // Tile-synchronous (TS) slices streamed through shared memory by the Tensor Memory Accelerator
 // (cp.async.bulk + mbarrier): the B200 form of "load the tiles on chip" and of the
-// one-time on-chip precision conversion.
+// on-chip precision conversion.
 //
-// TS layout (convert.cu): tile row TR owns slice columns [tr_slot[TR], tr_slot[TR+1]); a slice
-// column belongs to ONE tile and holds, for lane r = row 16*TR + r, the local column (0 on
-// padding) and the value stored at TilePrec (0 on padding).  The persistent CTA owns the
-// contiguous tile rows [tr0, tr1); conversion cuts them into stages (whole groups of H = B/16
-// tile rows when they fit the caps) and packs each stage into ONE contiguous blob:
-//   [header: int32 column start per tile-row boundary, K+1 entries]
-//   [column words: (tile column << 4) | Floor << 2 | TilePrec, ncol entries]
-//   [local columns: 16 bytes per column]
-//   [destination column of each group entry: u16, grouped FP64 | FP32 | FP16 | E4M3]
-//   [values, grouped by TilePrec (FP64 block, FP32 block, FP16 block, E4M3 block), 16 per column]
-// so that a stage is a single bulk copy (TMA throughput is bounded by copies per second).
+// TS layout (convert.cu): tile row TR owns slice columns; a slice column belongs to ONE tile and
+// holds, for lane r = row 16*TR + r, the local column (0 on padding) and the value stored at
+// TilePrec (0 on padding).  The persistent CTA owns the contiguous tile rows [tr0, tr1); half-warp
+// h takes the tile rows TR = tr0 + h (mod H) (lane r = row 16*TR + r: the row mapping of the
+// dot-product contract), so warp w owns the rows of half-warps 2w and 2w+1.  Conversion cuts the
+// CTA's tile rows into stages (one tile row per half-warp by default) and packs each stage into
+// ONE contiguous blob:
+//   [int32 hdr[16]: tr0, tr1, nc, off_desc, off_lc, off_val, own_w, col0 lo, col0 hi, off_wl,
+//    off_ent, off_eb]
+//   [int16 column start per tile-row boundary, K+1 entries]
+//   [u8 first decode-buffer slot of each tile row (its columns take consecutive slots)]
+//   [u32 desc per column: TilePrec | Floor << 2 | value offset (16 B units) << 4 | window byte
+//    offset of its column segment << 16; TS_DPAD zero entries after the last column]
+//   [u8 local column x 8 (byte offset within the segment) [col][lane]]
+//   [per warp: u32 column counts per TilePrec group (4 x u8); u16 offset of its decode list]
+//   [u16 decode lists: column | slot << 9, each warp's columns grouped by TilePrec]
+//   [values in column order, 16 x size(TilePrec) bytes per column]
+// The stage record (TsStage, 32 words) lists the runs of consecutive column segments the stage
+// gathers ("x windows"); the runs are bulk-copied from the PV vector next to the blob.
 //
-// Per stage: thread 0 keeps PIPE_NST stages in flight (one "full" mbarrier each).  After a stage
-// lands:
-//   1. decode pass (all threads, warp-uniform per precision group): 4 values per thread per
-//      step, exact upcast to binary64 into E[col][lane] (the on-chip conversion of P:237); the
-//      dynamic switch (Alg. 5) is applied here: bypassed columns become 0, a column with e_t
-//      below TilePrec is rounded to e_t (RNE_{e_t}(stored value));
-//   2. __syncthreads -- the slot is consumed (its column words / local columns were copied to the
-//      decoded-stage buffer too), so thread 0 refills it at once: PIPE_NST - 1 stages stay in
-//      flight during the FMA pass;
-//   3. FMA pass: half-warp h owns tile rows tr0 + h + kH, lane r = row 16*TR + r (the row mapping
-//      of the dot-product contract) and runs the row's single fma chain in ascending column
-//      order: acc = fma(E[c][r], x[16*tile column + local column], acc) -- a zero (padding or
-//      bypass) term leaves acc unchanged.  x is gathered through L1/L2 with coherent loads; the
-//      chain of a row is fully unrolled on its column count, all loads issued before the fmas.
-// Stages hold whole groups of H tile rows (two when they fit); the decoded-stage buffer is
-// single: two __syncthreads per stage order the decode and FMA passes.
-struct PipeStage {
-    int64_t col0, col1;             // slice-column range of the stage
-    int64_t boff;                   // blob offset in Mat::blob
-    int32_t tr0, tr1;               // tile rows [tr0, tr1)
-    int32_t bbytes;                 // blob bytes (multiple of 16)
-    int32_t off_cw, off_ss, off_dst, off_val;   // section offsets within the blob
-    int32_t gcnt[4];                // columns per precision group (FP64, FP32, FP16, E4M3)
-    int32_t goff[4];                // byte offset of each group's values within the blob
-    int32_t pad[3];
-};
-static_assert(sizeof(PipeStage) == 96, "PipeStage is 96 bytes");
+// Per stage, every warp independently (no CTA barrier): wait the slot's "full" mbarrier; decode
+// its columns group by group (warp-uniform precision, 4 values per lane, exact upcast) into its
+// private FP64 buffer E_w, applying the dynamic switch of Alg. 5 (bypass -> 0; e_t below TilePrec
+// -> RNE_{e_t} of the stored value: P:237's on-chip conversion); __syncwarp; each half-warp runs
+// its row's single fma chain in ascending column order with E_w and x from the staged window;
+// arrive on the slot's "empty" mbarrier.  Warp 0 refills a slot (one lane per bulk copy) once
+// every warp has arrived.
+constexpr int TS_KCAP = 64;       // tile rows per stage
+constexpr int TS_CCAP = 512;      // slice columns per stage
+constexpr int TS_VCAP = 16384;    // value bytes per stage
+constexpr int TS_WCAP = 160;      // window segments per stage
+constexpr int TS_RUNCAP = 8;      // runs per stage
+constexpr int TS_NSTMAX = 6;      // slots in the ring
+constexpr int TS_HDR = 64;        // blob header bytes
+constexpr int TS_PF = 4;          // stage records prefetched ahead by the issuing warp
+constexpr int TS_EBYTES = 65536;  // most shared memory the warp-private decode buffers may take
+constexpr int TS_DPAD = 16;       // zero column descriptors after the last column (short-row reads)
+__host__ __device__ constexpr int ts_r16(int v) { return (v + 15) & ~15; }
 
-constexpr int PIPE_NST = 3;        // stages in flight
-constexpr int PIPE_KCAP = 64;      // tile rows per stage
-constexpr int PIPE_CCAP = 576;     // slice columns per stage
-constexpr int PIPE_VCAP = 28672;   // value bytes per stage
-__host__ __device__ constexpr int pipe_r16(int v) { return (v + 15) & ~15; }
-constexpr int PIPE_BLOB_CAP = pipe_r16((PIPE_KCAP + 1) * 4) + pipe_r16(PIPE_CCAP * 4) + PIPE_CCAP * 16 +
-                              pipe_r16(PIPE_CCAP * 2 + 8) + PIPE_VCAP;
-constexpr int PS_INFO = pipe_r16(PIPE_BLOB_CAP);               // int32 tr0, tr1, off_cw, off_ss, off_dst, gcnt[4], goff[4]
-constexpr int PS_BYTES = PS_INFO + 64;
-// decoded stage (FMA side): values FP64 [col][lane], then the column words, local columns and
-// tile-row headers copied out of the slot so that the slot is refilled right after decoding
-constexpr int PIPE_E_BYTES = PIPE_CCAP * 128;
-constexpr int PIPE_F_CW = PIPE_E_BYTES;                        // u32 column words
-constexpr int PIPE_F_SS = PIPE_F_CW + PIPE_CCAP * 4;           // u8 local columns [col][lane]
-constexpr int PIPE_F_HDR = PIPE_F_SS + PIPE_CCAP * 16;         // int32 headers, then tr0, tr1
-constexpr int PIPE_D_BYTES = PIPE_F_HDR + pipe_r16((PIPE_KCAP + 1) * 4 + 8);
-constexpr int PIPE_LEV_CAP = 4096;                             // staged level bytes (column segments gathered)
-// region: [NST slots][decoded stage][full NST u64][ctr u64][pad][levels]
-constexpr size_t PIPE_SMEM_BYTES = (size_t)PIPE_NST * PS_BYTES + (size_t)PIPE_D_BYTES + 8 * PIPE_NST + 16 + PIPE_LEV_CAP;
+// stage record: 32 words, word l read by lane l of the issuing warp
+struct TsStage {
+    uint32_t boff_lo, boff_hi;      // blob offset in Mat::blob
+    int32_t bbytes;                 // blob bytes (multiple of 16)
+    int32_t nrun, wseg;             // runs, window segments (sum of run lengths)
+    int32_t tr0, tr1, nc;
+    int32_t run_s[TS_RUNCAP];       // first segment of each run
+    int32_t run_n[TS_RUNCAP];       // segments of each run
+    int32_t run_w[TS_RUNCAP];       // window offset (segments) of each run
+};
+static_assert(sizeof(TsStage) == 128, "TsStage is 32 words");
 
 struct TsSmem {
-    unsigned char* base;
-    __device__ __forceinline__ unsigned char* slot(int s) const { return base + (size_t)s * PS_BYTES; }
-    __device__ __forceinline__ unsigned char* D() const { return base + (size_t)PIPE_NST * PS_BYTES; }
-    __device__ __forceinline__ unsigned long long* full(int s) const {
-        return reinterpret_cast<unsigned long long*>(D() + PIPE_D_BYTES) + s;
-    }
-    __device__ __forceinline__ unsigned long long* ctr() const { return full(0) + PIPE_NST; }
-    __device__ __forceinline__ unsigned long long* resident() const { return full(0) + PIPE_NST + 1; }
-    __device__ __forceinline__ uint8_t* lev() const { return reinterpret_cast<uint8_t*>(full(0) + PIPE_NST + 2); }
+    unsigned char* base;            // ring of nst slots of slot_bytes
+    double* ebuf;                   // per-warp decode buffers: ecap columns x 16 doubles per warp
+    int nst, slot_bytes, blob_cap, ecap;
+    unsigned long long* full;       // [TS_NSTMAX]
+    unsigned long long* empty;      // [TS_NSTMAX]
+    unsigned long long* ctr;        // [0] stages issued so far (ring position); [1] resident SpMVs done
+    __device__ __forceinline__ unsigned char* slot(int s) const { return base + (size_t)s * slot_bytes; }
 };
+constexpr size_t TS_CTRL_BYTES = 16 * TS_NSTMAX + 32;
 
 __device__ __forceinline__ unsigned smem_u32(const void* p) { return (unsigned)__cvta_generic_to_shared(p); }
 __device__ __forceinline__ void mbar_init(unsigned long long* b, unsigned cnt) {
@@ -321,76 +227,98 @@ __device__ __forceinline__ void bulk_g2s_ef(void* dst, const void* src, unsigned
     asm volatile("cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes.L2::cache_hint [%0], [%1], %2, [%3], %4;"
                  ::"r"(smem_u32(dst)), "l"(src), "r"(bytes), "r"(smem_u32(bar)), "l"(pol) : "memory");
 }
+__device__ __forceinline__ void bulk_g2s(void* dst, const void* src, unsigned bytes, unsigned long long* bar) {
+    asm volatile("cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];"
+                 ::"r"(smem_u32(dst)), "l"(src), "r"(bytes), "r"(smem_u32(bar)) : "memory");
+}
 
 // all threads; followed by a __syncthreads of the caller before the first SpMV
-__device__ __forceinline__ void pipe_init(const TsSmem& sm) {
+__device__ __forceinline__ void ts_init(const TsSmem& sm) {
     if (threadIdx.x == 0) {
-        for (int s = 0; s < PIPE_NST; ++s) mbar_init(sm.full(s), 1);
-        *sm.ctr() = 0ull;
-        *sm.resident() = 0ull;
+        for (int s = 0; s < TS_NSTMAX; ++s) {
+            mbar_init(sm.full + s, 1);
+            mbar_init(sm.empty + s, blockDim.x >> 5);
+        }
+        sm.ctr[0] = 0ull;
+        sm.ctr[1] = 0ull;
         asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
     }
 }
 
-// thread 0: stage st -> slot (one bulk copy)
-__device__ __forceinline__ void pipe_issue(const Mat& A, const PipeStage& st, unsigned char* slot, unsigned long long* full,
-                                           unsigned long long pol) {
-    int32_t* info = reinterpret_cast<int32_t*>(slot + PS_INFO);
-    info[0] = st.tr0;
-    info[1] = st.tr1;
-    info[2] = st.off_cw;
-    info[3] = st.off_ss;
-    info[4] = st.off_dst;
-#pragma unroll
-    for (int q = 0; q < 4; ++q) { info[5 + q] = st.gcnt[q]; info[9 + q] = st.goff[q]; }
-    info[13] = (int32_t)st.col0;
-    mbar_expect_tx(full, (unsigned)st.bbytes);
-    bulk_g2s_ef(slot, A.blob + st.boff, (unsigned)st.bbytes, full, pol);
+// Warp 0: stage record word l in lane l (rec).  Lane 0 posts the transaction bytes, then lane r
+// (r < nrun) copies window run r and lane 31 the blob.
+__device__ __forceinline__ void ts_issue(const unsigned char* blob_base, uint32_t rec, unsigned char* slot, int blob_cap,
+                                         unsigned long long* full, const double* pv, bool with_blob, unsigned long long pol,
+                                         int dbg = 0) {
+    const int lane = threadIdx.x & 31;
+    const uint32_t boff_lo = __shfl_sync(0xffffffffu, rec, 0), boff_hi = __shfl_sync(0xffffffffu, rec, 1);
+    const int bbytes = (int)__shfl_sync(0xffffffffu, rec, 2), nrun = (int)__shfl_sync(0xffffffffu, rec, 3);
+    int wseg = (int)__shfl_sync(0xffffffffu, rec, 4);
+    if (dbg == 2) wseg = 0;                   // diagnostics: blobs only
+    if (dbg == 3) with_blob = false;          // diagnostics: windows only
+    const int rs = (int)__shfl_sync(0xffffffffu, rec, 8 + (lane & 7));
+    const int rn = (int)__shfl_sync(0xffffffffu, rec, 16 + (lane & 7));
+    const int rw = (int)__shfl_sync(0xffffffffu, rec, 24 + (lane & 7));
+    if (lane == 0) mbar_expect_tx(full, (unsigned)((with_blob ? bbytes : 0) + wseg * PV_SEG_BYTES));
+    __syncwarp();
+    if (lane < nrun && lane < TS_RUNCAP && dbg != 2)
+        bulk_g2s(slot + blob_cap + rw * PV_SEG_BYTES, pv + (int64_t)rs * PVS, (unsigned)(rn * PV_SEG_BYTES), full);
+    if (lane == 31 && with_blob) {
+        const uint64_t boff = ((uint64_t)boff_hi << 32) | boff_lo;
+        bulk_g2s_ef(slot, blob_base + boff, (unsigned)bbytes, full, pol);
+    }
 }
 
-// level of tile column tc for the dynamic switch
-__device__ __forceinline__ int col_level(uint32_t tc, const uint8_t* __restrict__ level, const uint8_t* lev_s, bool lev_staged,
-                                         int32_t seg_lo) {
-    return lev_staged ? (int)lev_s[tc - (uint32_t)seg_lo] : (int)level[tc];
+// exact upcast of the stored bits at precision e (0 FP64, 1 FP32, 2 FP16, 3 E4M3) to binary64
+__device__ __forceinline__ double decode_val(int e, uint64_t raw) {
+    const uint32_t lo = (uint32_t)raw;
+    const __half_raw h8 = __nv_cvt_fp8_to_halfraw((__nv_fp8_storage_t)(lo & 0xFFu), __NV_E4M3);
+    const unsigned short hb = e == 3 ? h8.x : (unsigned short)lo;
+    const float f16 = __half2float(__ushort_as_half(hb));
+    const float f = e >= 2 ? f16 : __uint_as_float(lo);
+    const double d = (double)f;
+    return e == 0 ? __longlong_as_double((long long)raw) : d;
 }
-
 __device__ __forceinline__ double e4m3_lo(uint32_t w2) {   // the E4M3 byte in bits 0..7 -> binary64 (exact)
     const __half_raw h = __nv_cvt_fp8_to_halfraw((__nv_fp8_storage_t)(w2 & 0xFFu), __NV_E4M3);
     return (double)__half2float(__half(h));
 }
 __device__ __forceinline__ double h16(uint32_t bits) { return (double)__half2float(__ushort_as_half((unsigned short)bits)); }
 
-// Shared-memory accesses of the pipeline are plain C++ (the compiler schedules them freely between
-// the barriers); the stage slot is read-only after its "full" mbarrier completes.
-struct PipeView {
-    const int32_t* info;      // PS_INFO fields
-    const int32_t* hdr;       // column start per tile-row boundary
-    const uint32_t* cw;       // column words
-    const uint8_t* ss;        // local columns [col][lane]
-    const uint16_t* dst;      // group permutation
+// view of one landed stage
+struct TsView {
     const unsigned char* blob;
+    const double* win;
+    int S0, S1, off_desc, off_lc, off_val, own_w, off_wl, off_ent, off_eb;
+    int64_t col0;
 };
-__device__ __forceinline__ PipeView pipe_view(const unsigned char* slot) {
-    PipeView v;
+__device__ __forceinline__ TsView ts_view(const unsigned char* slot, int blob_cap) {
+    TsView v;
+    const int32_t* h = reinterpret_cast<const int32_t*>(slot);
     v.blob = slot;
-    v.info = reinterpret_cast<const int32_t*>(slot + PS_INFO);
-    v.hdr = reinterpret_cast<const int32_t*>(slot);
-    v.cw = reinterpret_cast<const uint32_t*>(slot + v.info[2]);
-    v.ss = slot + v.info[3];
-    v.dst = reinterpret_cast<const uint16_t*>(slot + v.info[4]);
+    v.win = reinterpret_cast<const double*>(slot + blob_cap);
+    v.S0 = h[0]; v.S1 = h[1];
+    v.off_desc = h[3]; v.off_lc = h[4]; v.off_val = h[5]; v.own_w = h[6];
+    v.col0 = (int64_t)(((uint64_t)(uint32_t)h[8] << 32) | (uint32_t)h[7]);
+    v.off_wl = h[9]; v.off_ent = h[10]; v.off_eb = h[11];
     return v;
 }
 
-// decode pass: group Q (0 FP64 .. 3 E4M3) of the stage -> E.  Unit = 4 lanes of one column.
-template <int Q, bool DYN>
-__device__ __forceinline__ void pipe_decode_group(const PipeView& v, double* E, int ncol_q, int goff, const uint16_t* dst_q,
-                                                  const uint8_t* __restrict__ level, const uint8_t* lev_s, bool lev_staged,
-                                                  int32_t seg_lo, int range_guard, uint8_t* stk) {
-    const int units = ncol_q * 4;
-    for (int u = threadIdx.x; u < units; u += blockDim.x) {
-        const int j = u >> 2, r0 = (u & 3) * 4;
-        const unsigned d = dst_q[j];                                   // destination column in the stage
-        const unsigned char* src = v.blob + goff + ((j * 16 + r0) << (3 - Q));
+// Decode of one warp's columns into its buffer E (Q: the group's TilePrec, warp-uniform).  Unit u
+// = 4 lanes of one column.  Dynamic switch (Alg. 5 l.2-4, range guard R19): bypass -> 0, e_t below
+// TilePrec -> RNE_{e_t}(stored).  Sticky variant (P:237 literal): the column's mask of the levels
+// it was lowered to in place (Mat::stk, per slice column); the working value is RNE applied at
+// every lowered level in ascending order (successive rounding).
+template <int Q, bool DYN, bool STK>
+__device__ __forceinline__ void ts_decode_group(const TsView& v, const uint16_t* ent, int n, double* E, int range_guard,
+                                                uint8_t* stk) {
+    const int lane = threadIdx.x & 31;
+    const uint32_t* desc = reinterpret_cast<const uint32_t*>(v.blob + v.off_desc);
+    for (int u = lane; u < 4 * n; u += 32) {
+        const uint32_t en = ent[u >> 2];
+        const int c = (int)(en & 511u), r0 = (u & 3) * 4;
+        const uint32_t d = desc[c];
+        const unsigned char* src = v.blob + v.off_val + ((d >> 4) & 0xFFFu) * 16u + (r0 << (3 - Q));
         double w[4];
         if (Q == 0) {
             const double2 a = reinterpret_cast<const double2*>(src)[0], b = reinterpret_cast<const double2*>(src)[1];
@@ -405,39 +333,32 @@ __device__ __forceinline__ void pipe_decode_group(const PipeView& v, double* E, 
             const uint32_t a = *reinterpret_cast<const uint32_t*>(src);
             w[0] = e4m3_lo(a); w[1] = e4m3_lo(a >> 8); w[2] = e4m3_lo(a >> 16); w[3] = e4m3_lo(a >> 24);
         }
-        if (DYN && stk != nullptr) {
-            // sticky variant (P:237 literal; oracle spmv_tiles): e_t = max(cur, level) with the
-            // range guard; a new lower e_t lowers the tile's working values in place for good --
-            // the working value is RNE applied at every level the column has been lowered to, in
-            // ascending order (successive rounding, as the in-place copy has it)
-            const uint32_t word = v.cw[d];
-            const int lv = col_level(word >> 4, level, lev_s, lev_staged, seg_lo);
-            if (lv == BYP) { w[0] = w[1] = w[2] = w[3] = 0.0; }
-            else {
-                uint8_t* sp = stk + (v.info[13] + (int)d);
-                unsigned mask = *sp;
-                const int cur = mask ? 31 - __clz(mask) : Q;
-                int e = max(lv, cur);
-                if (range_guard) e = min(e, (int)((word >> 2) & 3u));
-                if (e > cur) {
-                    mask |= 1u << e;
-                    if (r0 == 0) *sp = (uint8_t)mask;   // every unit of the column computes the same mask
-                }
-#pragma unroll
-                for (int L = Q + 1; L <= 3; ++L)
-                    if (mask & (1u << L)) {
-#pragma unroll
-                        for (int k = 0; k < 4; ++k) w[k] = round_to(w[k], L);
+        if (DYN) {
+            const int lv = (int)(reinterpret_cast<const uint8_t*>(v.win) + (d >> 16))[128];
+            if (STK) {
+                if (lv == BYP) { w[0] = w[1] = w[2] = w[3] = 0.0; }
+                else {
+                    uint8_t* sp = stk + (v.col0 + c);
+                    unsigned mask = *sp;
+                    const int cur = mask ? 31 - __clz(mask) : Q;
+                    int e = max(lv, cur);
+                    if (range_guard) e = min(e, (int)((d >> 2) & 3u));
+                    if (e > cur) {
+                        mask |= 1u << e;
+                        if (r0 == 0) *sp = (uint8_t)mask;   // every unit of the column computes the same mask
                     }
-            }
-        } else if (DYN) {   // e_t = bypass | max(TilePrec, level), range guard e_t <= Floor (Alg. 5)
-            const uint32_t word = v.cw[d];
-            const int lv = col_level(word >> 4, level, lev_s, lev_staged, seg_lo);
-            if (lv > Q) {
+#pragma unroll
+                    for (int L = Q + 1; L <= 3; ++L)
+                        if (mask & (1u << L)) {
+#pragma unroll
+                            for (int k = 0; k < 4; ++k) w[k] = round_to(w[k], L);
+                        }
+                }
+            } else if (lv > Q) {
                 if (lv == BYP) { w[0] = w[1] = w[2] = w[3] = 0.0; }
                 else {
                     int e = lv;
-                    if (range_guard) e = min(e, (int)((word >> 2) & 3u));
+                    if (range_guard) e = min(e, (int)((d >> 2) & 3u));
                     if (e != Q) {
 #pragma unroll
                         for (int k = 0; k < 4; ++k) w[k] = round_to(w[k], e);
@@ -445,231 +366,254 @@ __device__ __forceinline__ void pipe_decode_group(const PipeView& v, double* E, 
                 }
             }
         }
-        double2* ea = reinterpret_cast<double2*>(E + d * 16 + r0);
+        double2* ea = reinterpret_cast<double2*>(E + (en >> 9) * 16 + r0);
         ea[0] = make_double2(w[0], w[1]);
         ea[1] = make_double2(w[2], w[3]);
     }
 }
 
-template <bool DYN>
-__device__ __forceinline__ void pipe_decode(const PipeView& v, unsigned char* D, const uint8_t* __restrict__ level, const uint8_t* lev_s,
-                                            bool lev_staged, int32_t seg_lo, int range_guard, uint8_t* stk) {
-    double* E = reinterpret_cast<double*>(D);
-    {   // the FMA side's copy of the column words, local columns and headers
-        const int S0 = v.info[0], S1 = v.info[1], K = S1 - S0;
-        const int ncol = v.hdr[K];
-        uint4* fss = reinterpret_cast<uint4*>(D + PIPE_F_SS);
-        const uint4* sss = reinterpret_cast<const uint4*>(v.ss);
-        for (int c = threadIdx.x; c < ncol; c += blockDim.x) fss[c] = sss[c];
-        uint32_t* fcw = reinterpret_cast<uint32_t*>(D + PIPE_F_CW);
-        for (int c = threadIdx.x; c < ncol; c += blockDim.x) fcw[c] = v.cw[c];
-        int32_t* fh = reinterpret_cast<int32_t*>(D + PIPE_F_HDR);
-        for (int k = threadIdx.x; k <= K; k += blockDim.x) fh[k] = v.hdr[k];
-        if (threadIdx.x == 0) {
-            int32_t* tail = reinterpret_cast<int32_t*>(D + PIPE_D_BYTES) - 2;
-            tail[0] = S0;
-            tail[1] = S1;
-        }
-    }
-    const uint16_t* dst = v.dst;
-    const int g0 = v.info[5], g1 = v.info[6], g2 = v.info[7], g3 = v.info[8];
-    pipe_decode_group<0, DYN>(v, E, g0, v.info[9], dst, level, lev_s, lev_staged, seg_lo, range_guard, stk);
-    dst += g0;
-    pipe_decode_group<1, DYN>(v, E, g1, v.info[10], dst, level, lev_s, lev_staged, seg_lo, range_guard, stk);
-    dst += g1;
-    pipe_decode_group<2, DYN>(v, E, g2, v.info[11], dst, level, lev_s, lev_staged, seg_lo, range_guard, stk);
-    dst += g2;
-    pipe_decode_group<3, DYN>(v, E, g3, v.info[12], dst, level, lev_s, lev_staged, seg_lo, range_guard, stk);
-}
-
-// one tile row of N columns starting at stage column c: every load first, then the fma chain.
-// x is written during the solve by other CTAs (ordered by the barriers' acquire): plain coherent
-// loads (x is not __restrict__, so never the read-only .nc path).
+// one tile row of this half-warp, N = the warp's widest row: columns beyond W read the next
+// descriptors (or the zero padding) and contribute fma(0, x, acc) == acc exactly (acc is never -0,
+// x is finite), so both half-warps run the same instruction stream.  Per column: descriptor and
+// local-column byte offset (LDS, immediate offsets), x from the window, the decoded value from
+// the warp's buffer (consecutive slots per row), one fma in ascending column order.
 template <int N>
-__device__ __forceinline__ double pipe_row(const uint32_t* cw, const uint8_t* ssl, const double* El, int c, const double* x) {
+__device__ __forceinline__ double ts_row(const TsView& v, const double* Er, int a, int W, int lane) {
+    const uint32_t* desc = reinterpret_cast<const uint32_t*>(v.blob + v.off_desc) + a;
+    const uint8_t* lcb = v.blob + v.off_lc + a * 16 + lane;
+    const unsigned char* win = reinterpret_cast<const unsigned char*>(v.win);
     double ev[N], xv[N];
 #pragma unroll
     for (int q = 0; q < N; ++q) {
-        const uint32_t word = cw[c + q];
-        const uint32_t lc = ssl[(c + q) * 16];
-        ev[q] = El[(c + q) * 16];
-        xv[q] = x[(word & ~15u) | lc];
+        const uint32_t d = desc[q];
+        ev[q] = q < W ? Er[q * 16] : 0.0;
+        xv[q] = *reinterpret_cast<const double*>(win + (d >> 16) + lcb[q * 16]);
     }
     double acc = 0.0;
 #pragma unroll
     for (int q = 0; q < N; ++q) acc = __fma_rn(ev[q], xv[q], acc);
     return acc;
 }
-// rows wider than 12 columns: chunks of 8 (the chain continues across chunks)
-__device__ __forceinline__ double pipe_row_long(const uint32_t* cw, const uint8_t* ssl, const double* El, int c, int W, const double* x) {
-    double acc = 0.0;
-    int q0 = 0;
-    for (; q0 + 8 <= W; q0 += 8) {
-        double ev[8], xv[8];
-#pragma unroll
-        for (int q = 0; q < 8; ++q) {
-            const int cc = c + q0 + q;
-            ev[q] = El[cc * 16];
-            xv[q] = x[(cw[cc] & ~15u) | ssl[cc * 16]];
+// rows wider than 12 slice columns: plain loop over the columns in order (the chain is exact)
+__device__ __forceinline__ double ts_row_long(const TsView& v, const double* Er, int a, int W, int lane) {
+    const uint32_t* desc = reinterpret_cast<const uint32_t*>(v.blob + v.off_desc) + a;
+    const uint8_t* lcb = v.blob + v.off_lc + a * 16 + lane;
+    const unsigned char* win = reinterpret_cast<const unsigned char*>(v.win);
+    double r = 0.0;
+    for (int q = 0; q < W; ++q)
+        r = __fma_rn(Er[q * 16], *reinterpret_cast<const double*>(win + (desc[q] >> 16) + lcb[q * 16]), r);
+    return r;
+}
+__device__ __forceinline__ double ts_row_any(const TsView& v, const double* Er, int a, int W, int Wmax, int lane) {
+    switch (Wmax) {
+    case 0: return 0.0;
+    case 1: return ts_row<1>(v, Er, a, W, lane);
+    case 2: return ts_row<2>(v, Er, a, W, lane);
+    case 3: return ts_row<3>(v, Er, a, W, lane);
+    case 4: return ts_row<4>(v, Er, a, W, lane);
+    case 5: return ts_row<5>(v, Er, a, W, lane);
+    case 6: return ts_row<6>(v, Er, a, W, lane);
+    case 7: return ts_row<7>(v, Er, a, W, lane);
+    case 8: return ts_row<8>(v, Er, a, W, lane);
+    case 9: return ts_row<9>(v, Er, a, W, lane);
+    case 10: return ts_row<10>(v, Er, a, W, lane);
+    case 11: return ts_row<11>(v, Er, a, W, lane);
+    case 12: return ts_row<12>(v, Er, a, W, lane);
+    default: return ts_row_long(v, Er, a, W, lane);
+    }
+}
+
+// consume one landed stage (one warp): decode its columns, then the rows of its two half-warps.
+// own_mode: 0 none; 1 the SpMV input at the row (from the window when the stage's own segments
+// are staged); 2 the normal vector `ownv`.
+template <bool DYN, bool STK, class Emit>
+__device__ __forceinline__ void ts_consume(const TsView& v, int64_t tr0c, const double* pv, int range_guard, int own_mode,
+                                           const double* ownv, int64_t n, uint8_t* stk, int dbg, double* E, Emit& emit) {
+    const int t = threadIdx.x, H = blockDim.x >> 4, h = t >> 4, lane = t & 15, w = t >> 5;
+    if (dbg >= 1) return;
+    {
+        const uint32_t cnt = reinterpret_cast<const uint32_t*>(v.blob + v.off_wl)[w];
+        const int NW = blockDim.x >> 5;
+        const uint16_t* ent = reinterpret_cast<const uint16_t*>(v.blob + v.off_ent) +
+                              reinterpret_cast<const uint16_t*>(v.blob + v.off_wl + ts_r16(NW * 4))[w];
+        const int n0 = cnt & 0xFF, n1 = (cnt >> 8) & 0xFF, n2 = (cnt >> 16) & 0xFF, n3 = cnt >> 24;
+        ts_decode_group<0, DYN, STK>(v, ent, n0, E, range_guard, stk);
+        ts_decode_group<1, DYN, STK>(v, ent + n0, n1, E, range_guard, stk);
+        ts_decode_group<2, DYN, STK>(v, ent + n0 + n1, n2, E, range_guard, stk);
+        ts_decode_group<3, DYN, STK>(v, ent + n0 + n1 + n2, n3, E, range_guard, stk);
+    }
+    __syncwarp();
+    const int16_t* cs = reinterpret_cast<const int16_t*>(v.blob + TS_HDR);
+    const int rel = v.S0 - (int)tr0c;
+    const int off0 = (H & (H - 1)) == 0 ? (rel & (H - 1)) : rel % H;
+    const int first = h >= off0 ? h - off0 : h - off0 + H;
+    // both half-warps of the warp run the same iterations (their row or nothing)
+    for (int k = first;; k += H) {
+        const bool mine = v.S0 + k < v.S1;
+        if (!__any_sync(0xffffffffu, mine)) break;
+        const int a = mine ? cs[k] : 0, W = mine ? cs[k + 1] - a : 0;
+        const int Wmax = max(W, __shfl_xor_sync(0xffffffffu, W, 16));
+        const double* Er = E + (mine ? (int)v.blob[v.off_eb + k] : 0) * 16 + lane;
+        const double acc = ts_row_any(v, Er, a, W, Wmax, lane);
+        if (mine) {
+            const int TR = v.S0 + k;
+            double ov = 0.0;
+            const int64_t i = (int64_t)TR * 16 + lane;
+            if (own_mode == 1) ov = v.own_w >= 0 ? v.win[(v.own_w + k) * PVS + lane] : pv[(int64_t)TR * PVS + lane];
+            else if (own_mode == 2 && i < n) ov = ownv[i];
+            emit((int64_t)TR, lane, acc, ov);
+        }
+    }
+    __syncwarp();
+}
+
+// The whole SpMV of one CTA (all threads), tile rows [tr0c, tr1c) = the CTA's plan range, input
+// vector pv (PV layout, levels included).  Called with every thread of the CTA; the caller
+// guarantees pv is complete (ready flags / barrier).
+template <bool DYN, bool STK, class Emit>
+__device__ __forceinline__ void spmv_ts(const Mat& A, int64_t tr0c, const double* pv, int range_guard, const TsSmem& sm,
+                                        int own_mode, const double* ownv, Emit& emit) {
+    const int t = threadIdx.x, w = t >> 5, lane = t & 31;
+    const int32_t s_begin = A.stg_ptr[blockIdx.x], ns = A.stg_ptr[blockIdx.x + 1] - s_begin;
+    const uint32_t* recs = reinterpret_cast<const uint32_t*>(A.stg + s_begin);
+    const int NST = sm.nst;
+    double* E = sm.ebuf + (size_t)w * sm.ecap * 16;
+    __syncthreads();                          // ring counters / previous phase's smem users
+    if (ns == 0 || A.dbg == 4) return;
+    unsigned long long pol = 0;
+    if (w == 0) {
+        pol = policy_evict_first();
+        asm volatile("fence.proxy.async.global;" ::: "memory");   // generic-proxy writes of pv -> bulk copies
+    }
+    if (ns <= NST) {
+        // every stage of this CTA fits the ring: the blobs stay resident across SpMVs (small
+        // matrices, e.g. C1); only the x windows are re-staged
+        const unsigned rc = (unsigned)sm.ctr[1];
+        if (w == 0)
+            for (int k = 0; k < ns; ++k) ts_issue(A.blob, recs[k * 32 + lane], sm.slot(k), sm.blob_cap, sm.full + k, pv, rc == 0, pol, A.dbg);
+        for (int k = 0; k < ns; ++k) {
+            mbar_wait(sm.full + k, rc & 1u);
+            ts_consume<DYN, STK>(ts_view(sm.slot(k), sm.blob_cap), tr0c, pv, range_guard, own_mode, ownv, A.n_rows, A.stk, A.dbg, E, emit);
+        }
+        __syncthreads();
+        if (t == 0) sm.ctr[1] = rc + 1;
+        return;
+    }
+    // streaming: ring position u0 (slot = u mod NST, phase = (u / NST) & 1), 32-bit counters
+    const unsigned u0 = (unsigned)sm.ctr[0];
+    int sl = (int)(u0 % (unsigned)NST);
+    unsigned ph = (u0 / (unsigned)NST) & 1u;
+    uint32_t pre[TS_PF];                      // warp 0: records of stages k + NST .. k + NST + TS_PF - 1
+    if (w == 0) {
+        int isl = sl;
+        unsigned iph = ph;
+        for (int k = 0; k < min(ns, NST); ++k) {
+            // the slot's previous use (previous SpMV) finished before the caller's barrier; its
+            // "empty" phase completed: wait on it to keep the parity in step
+            if (u0 + k >= (unsigned)NST) mbar_wait(sm.empty + isl, iph ^ 1u);
+            ts_issue(A.blob, recs[k * 32 + lane], sm.slot(isl), sm.blob_cap, sm.full + isl, pv, true, pol, A.dbg);
+            if (++isl == NST) { isl = 0; iph ^= 1u; }
         }
 #pragma unroll
-        for (int q = 0; q < 8; ++q) acc = __fma_rn(ev[q], xv[q], acc);
+        for (int j = 0; j < TS_PF; ++j) pre[j] = NST + j < ns ? recs[(NST + j) * 32 + lane] : 0u;
     }
-    for (; q0 < W; ++q0) {
-        const int cc = c + q0;
-        acc = __fma_rn(El[cc * 16], x[(cw[cc] & ~15u) | ssl[cc * 16]], acc);
+    for (int k = 0; k < ns; ++k) {
+        mbar_wait(sm.full + sl, ph);
+        ts_consume<DYN, STK>(ts_view(sm.slot(sl), sm.blob_cap), tr0c, pv, range_guard, own_mode, ownv, A.n_rows, A.stk, A.dbg, E, emit);
+        if (lane == 0) mbar_arrive(sm.empty + sl);
+        if (w == 0 && k + NST < ns) {
+            mbar_wait(sm.empty + sl, ph);         // every warp is done with the slot
+            ts_issue(A.blob, pre[0], sm.slot(sl), sm.blob_cap, sm.full + sl, pv, true, pol, A.dbg);
+#pragma unroll
+            for (int j = 0; j + 1 < TS_PF; ++j) pre[j] = pre[j + 1];
+            pre[TS_PF - 1] = k + NST + TS_PF < ns ? recs[(k + NST + TS_PF) * 32 + lane] : 0u;
+        }
+        if (++sl == NST) { sl = 0; ph ^= 1u; }
     }
+    __syncthreads();
+    if (t == 0) sm.ctr[0] = u0 + (unsigned)ns;
+}
+
+// ------------------------------------------------------------------------------------------
+// Compact (row-packed SELL-16) layout: windowed SpMV over the contiguous tile rows [tr0, tr1)
+// of one CTA (all B threads call it).  A window is up to WIN_TR tile rows (a multiple of
+// H = B/16 so that half-warp h always gets tile rows tr0 + h + kH, the row mapping of the
+// dot-product contract); per window the CTA stages the tile codes (tile column + e_t) of the
+// window's tiles in shared memory.  Used for matrices whose tile-synchronous slices would pad
+// too much (scattered patterns, e.g. C4); stencil-like matrices take the TMA pipeline above.
+constexpr int WIN_TR = 1024;
+constexpr int CODE_CAP = 8192;
+constexpr int WIN_BUF_BYTES = CODE_CAP * 4;
+
+struct WinSmem {
+    int32_t* hs;     // [WIN_TR+1] slot (slice column) offset of each tile row, relative to s0
+    int32_t* ht;     // [WIN_TR+1] tile offset, relative to t0
+    int64_t* misc;   // [4]: -, -, window end, staged
+    unsigned long long* pb;   // [4] value-plane base addresses (FP64, FP32, FP16, E4M3)
+    unsigned char* buf;   // [WIN_BUF_BYTES]: uint32 code[CODE_CAP]
+};
+constexpr size_t WIN_SMEM_BYTES = 2 * (WIN_TR + 1) * 4 + 4 * 8 + 8 + 4 * 8 + WIN_BUF_BYTES + 16;
+
+// Value fetch: ONE aligned 8-byte load from plane[e] + pos*size(e) (planes are 8-byte aligned and
+// padded), the needed bytes shifted down.  The 8-byte word lies in the same 32-byte DRAM sector
+// as the value, so this moves no extra HBM bytes; it replaces four predicated loads.
+__device__ __forceinline__ uint64_t load_raw(const unsigned long long* pbase, int e, int64_t pos) {
+    const unsigned long long a = pbase[e] + ((unsigned long long)pos << (3 - e));
+    const unsigned long long w = __ldg(reinterpret_cast<const unsigned long long*>(a & ~7ull));
+    return w >> ((a & 7ull) * 8);
+}
+
+// compact layout: process slot words s[0..cnt) of one lane; returns updated acc.  The code of a
+// tile is (tile column << 3) | e_t (sticky: | TilePrec << 27 | mask << 29, tile column < 2^24).
+template <bool DYN, bool STK, int N>
+__device__ __forceinline__ double slot_block(const Mat& A, const unsigned long long* w_pb, const uint16_t (&s)[N], int cnt, int64_t pos0,
+                                             const uint32_t* code, bool staged, int64_t tb_abs, const double* pv,
+                                             int range_guard, double acc) {
+    uint64_t raw[N];
+    double xv[N];
+    int ev[N];
+#pragma unroll
+    for (int q = 0; q < N; ++q) {
+        ev[q] = BYP;
+        raw[q] = 0;
+        xv[q] = 0.0;
+        if (q < cnt && s[q] != mf::SLOT_PAD) {
+            const int j = s[q] >> 4;
+            const uint32_t c = staged ? code[j]
+                               : STK ? sticky_code(A, tb_abs + j, pv, range_guard, false)
+                                     : tile_code<DYN>(A.tile_info[tb_abs + j], pv, range_guard);
+            ev[q] = (int)(c & 7u);
+            if (ev[q] != BYP) {
+                // sticky: the stored value (plane TilePrec), lowered in the loop below
+                raw[q] = load_raw(w_pb, STK ? (int)((c >> 27) & 3u) : ev[q], pos0 + q * 16);
+                const uint32_t tc = STK ? ((c >> 3) & CODE_TC_MASK) : (c >> 3);
+                xv[q] = pv[(int64_t)tc * PVS + (s[q] & 15)];
+                if (STK) ev[q] |= (int)(c >> 24) & 0xF8;   // TilePrec << 3 | (mask >> 1) << 5
+            }
+        }
+    }
+#pragma unroll
+    for (int q = 0; q < N; ++q)
+        if ((ev[q] & 7) != BYP) {
+            double v;
+            if (STK) {   // successive RNE at every level the tile was lowered to
+                const int prec = (ev[q] >> 3) & 3, m1 = ev[q] >> 5;   // m1 bit L-1 = lowered to L
+                v = decode_val(prec, raw[q]);
+#pragma unroll
+                for (int L = 1; L <= 3; ++L)
+                    if (L > prec && (m1 & (1 << (L - 1)))) v = round_to(v, L);
+            } else {
+                v = decode_val(ev[q], raw[q]);
+            }
+            acc = __fma_rn(v, xv[q], acc);
+        }
     return acc;
 }
-__device__ __forceinline__ double pipe_row_any(const uint32_t* cw, const uint8_t* ssl, const double* El, int c, int W, const double* x) {
-    switch (W) {
-    case 0: return 0.0;
-    case 1: return pipe_row<1>(cw, ssl, El, c, x);
-    case 2: return pipe_row<2>(cw, ssl, El, c, x);
-    case 3: return pipe_row<3>(cw, ssl, El, c, x);
-    case 4: return pipe_row<4>(cw, ssl, El, c, x);
-    case 5: return pipe_row<5>(cw, ssl, El, c, x);
-    case 6: return pipe_row<6>(cw, ssl, El, c, x);
-    case 7: return pipe_row<7>(cw, ssl, El, c, x);
-    case 8: return pipe_row<8>(cw, ssl, El, c, x);
-    case 9: return pipe_row<9>(cw, ssl, El, c, x);
-    case 10: return pipe_row<10>(cw, ssl, El, c, x);
-    case 11: return pipe_row<11>(cw, ssl, El, c, x);
-    case 12: return pipe_row<12>(cw, ssl, El, c, x);
-    default: return pipe_row_long(cw, ssl, El, c, W, x);
-    }
-}
 
-// FMA pass of one stage: half-warp h takes its tile rows (TR = tr0c + h (mod H)) in ascending order
-template <class Emit>
-__device__ __forceinline__ void pipe_fma(const Mat& A, const unsigned char* D, int64_t tr0c, const double* x,
-                                         const double* own, Emit& emit) {
-    const int t = threadIdx.x, H = blockDim.x >> 4, h = t >> 4, lane = t & 15;
-    const int32_t* hdr = reinterpret_cast<const int32_t*>(D + PIPE_F_HDR);
-    const uint32_t* cw = reinterpret_cast<const uint32_t*>(D + PIPE_F_CW);
-    const uint8_t* ssl = D + PIPE_F_SS + lane;
-    const double* El = reinterpret_cast<const double*>(D) + lane;
-
-    // S0, S1 follow the K+1 headers; K is recovered from them (S1 - S0)
-    int S0 = 0, S1 = 0;
-    {
-        // headers occupy [0, K]; tr0/tr1 at K+1, K+2 -- found from the fixed KCAP-sized area
-        const int32_t* tail = reinterpret_cast<const int32_t*>(D + PIPE_D_BYTES) - 2;
-        S0 = tail[0];
-        S1 = tail[1];
-    }
-    const int off0 = (int)(S0 - tr0c) % H;
-    for (int TR = S0 + (h - off0 + H) % H; TR < S1; TR += H) {
-        const int k = TR - S0;
-        const int a = hdr[k], W = hdr[k + 1] - a;
-        const int64_t i = (int64_t)TR * 16 + lane;
-        const double ov = (own != nullptr && i < A.n_rows) ? own[i] : 0.0;
-        emit((int64_t)TR, lane, pipe_row_any(cw, ssl, El, a, W, x), ov);
-    }
-}
-
-// the whole SpMV of one CTA (all threads), tile rows [tr0c, tr1c) = the CTA's plan range
-template <bool DYN, bool COUNT, class Emit>
-__device__ __forceinline__ void spmv_pipe(const Mat& A, int64_t tr0c, int64_t tr1c, const double* x,
-                                          const uint8_t* __restrict__ level, int range_guard, const TsSmem& sm, Counts* cnt,
-                                          int32_t seg_lo, int32_t seg_hi, const double* own, Emit& emit) {
-    const int t = threadIdx.x, B = blockDim.x;
-    const int32_t s_begin = A.stg_ptr[blockIdx.x], ns = A.stg_ptr[blockIdx.x + 1] - s_begin;
-    const int32_t nlev = seg_hi - seg_lo + 1;
-    const bool lev_staged = DYN && nlev > 0 && nlev <= PIPE_LEV_CAP;
-    __syncthreads();                          // smem users of the previous phase are done
-    if (ns <= PIPE_NST) {
-        // every stage of this CTA fits the ring: load once, keep the slots resident across SpMVs
-        // (small matrices, e.g. C1: no TMA round trip per SpMV)
-        const bool loaded = *sm.resident() != 0ull;
-        if (!loaded && t == 0) {
-            const unsigned long long pol = policy_evict_first();
-            for (int k = 0; k < ns; ++k) pipe_issue(A, A.stg[s_begin + k], sm.slot(k), sm.full(k), pol);
-        }
-        if (lev_staged)
-            for (int i = t; i < nlev; i += B) sm.lev()[i] = level[seg_lo + i];
-        if (COUNT)
-            for (int64_t i = A.tr_tile[tr0c] + t; i < A.tr_tile[tr1c]; i += B) {
-                const int e = (int)(tile_code<DYN>(A.tile_info[i], level, range_guard) & 7u);
-                cnt->tile(e);
-                cnt->nzn(e, (int)(A.tile_nnz[i + 1] - A.tile_nnz[i]));
-            }
-        __syncthreads();
-        unsigned char* D = sm.D();
-        for (int k = 0; k < ns; ++k) {
-            if (k > 0) __syncthreads();
-            if (!loaded) mbar_wait(sm.full(k), 0u);
-            pipe_decode<DYN>(pipe_view(sm.slot(k)), D, level, sm.lev(), lev_staged, seg_lo, range_guard, A.stk);
-            __syncthreads();
-            pipe_fma(A, D, tr0c, x, own, emit);
-        }
-        __syncthreads();
-        if (t == 0) *sm.resident() = 1ull;
-        return;
-    }
-    const unsigned u0 = (unsigned)*sm.ctr();
-    unsigned long long pol = 0;
-    if (t == 0) {
-        pol = policy_evict_first();
-        for (int k = 0; k < min(ns, PIPE_NST); ++k) {
-            const unsigned u = u0 + (unsigned)k, sl = u % PIPE_NST, mm = u / PIPE_NST;
-            pipe_issue(A, A.stg[s_begin + k], sm.slot(sl), sm.full(sl), pol);
-        }
-    }
-    if (lev_staged)
-        for (int i = t; i < nlev; i += B) sm.lev()[i] = level[seg_lo + i];
-    if (COUNT)
-        for (int64_t i = A.tr_tile[tr0c] + t; i < A.tr_tile[tr1c]; i += B) {
-            const int e = (int)(tile_code<DYN>(A.tile_info[i], level, range_guard) & 7u);
-            cnt->tile(e);
-            cnt->nzn(e, (int)(A.tile_nnz[i + 1] - A.tile_nnz[i]));
-        }
-    __syncthreads();
-    const uint8_t* lev_s = sm.lev();
-    unsigned char* D = sm.D();
-    PipeStage nxt;
-    for (int k = 0; k < ns; ++k) {
-        const unsigned u = u0 + (unsigned)k, sl = u % PIPE_NST, mm = u / PIPE_NST;
-        const bool refill = t == 0 && k + PIPE_NST < ns;
-        if (refill) nxt = A.stg[s_begin + k + PIPE_NST];
-        if (k > 0) __syncthreads();           // the decoded-stage buffer is free (previous FMA pass done)
-        mbar_wait(sm.full(sl), mm & 1u);
-        pipe_decode<DYN>(pipe_view(sm.slot(sl)), D, level, lev_s, lev_staged, seg_lo, range_guard, A.stk);
-        __syncthreads();                      // decoded stage complete; slot sl no longer read
-        if (refill) pipe_issue(A, nxt, sm.slot(sl), sm.full(sl), pol);
-        pipe_fma(A, D, tr0c, x, own, emit);
-    }
-    __syncthreads();
-    if (t == 0) *sm.ctr() = (unsigned long long)(u0 + (unsigned)ns);
-}
-
-__device__ __forceinline__ void carve_spmv(unsigned char* base, WinSmem& w, TsSmem& ts) {
-    unsigned char* p = base;
-    w.misc = reinterpret_cast<int64_t*>(p);
-    p += 4 * 8 + 8;
-    w.pb = reinterpret_cast<unsigned long long*>(p);
-    p += 4 * 8;
-    w.hs = reinterpret_cast<int32_t*>(p);
-    p += (WIN_TR + 1) * 4;
-    w.ht = reinterpret_cast<int32_t*>(p);
-    p += (WIN_TR + 1) * 4;
-    p = base + pipe_r16((int)(p - base));    // base is 16-aligned; no integer round trip of the pointer
-    w.buf = p;
-    ts.base = base;    // the two views overlap: a matrix uses one layout
-}
-constexpr size_t SPMV_SMEM_BYTES = PIPE_SMEM_BYTES > WIN_SMEM_BYTES ? PIPE_SMEM_BYTES : WIN_SMEM_BYTES;
-
-// emit(TR, lane, value, own[row]) is called by every lane for each of its tile rows, in ascending
-// TR; own (nullable) is a vector the caller's fused dot needs at the row (prefetched).
-// seg_lo/seg_hi: the column segments this CTA's tiles gather (level staging).
-template <bool DYN, bool COUNT, int PF, class Emit>
-__device__ __forceinline__ void spmv_cta(const Mat& A, int64_t tr0, int64_t tr1, const double* x, const uint8_t* __restrict__ level,
-                         int range_guard, const WinSmem& w, const TsSmem& tsm, Counts* cnt, int32_t seg_lo,
-                         int32_t seg_hi, const double* own, Emit emit) {
-    if (A.ts) {
-        spmv_pipe<DYN, COUNT>(A, tr0, tr1, x, level, range_guard, tsm, cnt, seg_lo, seg_hi, own, emit);
-        return;
-    }
+// emit(TR, lane, value, own) is called by every lane for each of its tile rows, in ascending TR.
+template <bool DYN, bool STK, int PF, class Emit>
+__device__ __forceinline__ void spmv_compact(const Mat& A, int64_t tr0, int64_t tr1, const double* pv, int range_guard,
+                                             const WinSmem& w, int own_mode, const double* ownv, Emit& emit) {
     const int t = threadIdx.x, B = blockDim.x, H = B >> 4, h = t >> 4, lane = t & 15;
     __syncthreads();
     if (t < 4) w.pb[t] = t == 0 ? (unsigned long long)A.p64 : t == 1 ? (unsigned long long)A.p32
@@ -700,10 +644,8 @@ __device__ __forceinline__ void spmv_cta(const Mat& A, int64_t tr0, int64_t tr1,
         const int nt = w.ht[nw];
         uint32_t* code = reinterpret_cast<uint32_t*>(w.buf);
         for (int i = t; i < nt; i += B) {
-            const uint32_t c = (DYN && A.stk != nullptr) ? sticky_code(A, t0 + i, level, range_guard, true)
-                                                         : tile_code<DYN>(A.tile_info[t0 + i], level, range_guard);
+            const uint32_t c = STK ? sticky_code(A, t0 + i, pv, range_guard, true) : tile_code<DYN>(A.tile_info[t0 + i], pv, range_guard);
             if (staged) code[i] = c;
-            if (COUNT) cnt->tile((int)(c & 7u));
         }
         __syncthreads();
         // half-warp h: tile rows w0 + h + kH, the next row's first PF slot words prefetched
@@ -726,24 +668,79 @@ __device__ __forceinline__ void spmv_cta(const Mat& A, int64_t tr0, int64_t tr1,
             const int64_t sb = s0 + a;
             const int64_t tb_abs = t0 + w.ht[li];
             const uint32_t* cd = code + w.ht[li];
-            const int64_t i = (w0 + li) * 16 + lane;
-            const double ov = (own != nullptr && i < A.n_rows) ? own[i] : 0.0;
+            const int64_t TR = w0 + li, i = TR * 16 + lane;
+            double ov = 0.0;
+            if (own_mode == 1) ov = pv[TR * PVS + lane];
+            else if (own_mode == 2 && i < A.n_rows) ov = ownv[i];
             double acc = 0.0;
-            acc = slot_block<DYN, COUNT, PF>(A, w.pb, cur, min(W, PF), sb * 16 + lane, cd, staged, tb_abs, level,
-                                              range_guard, x, acc, cnt);
+            acc = slot_block<DYN, STK, PF>(A, w.pb, cur, min(W, PF), sb * 16 + lane, cd, staged, tb_abs, pv, range_guard, acc);
             for (int k = PF; k < W; k += PF) {
                 uint16_t more[PF];
                 const uint16_t* sp = A.sidx + (sb + k) * 16 + lane;
 #pragma unroll
                 for (int q = 0; q < PF; ++q) more[q] = (k + q < W) ? __ldg(sp + q * 16) : mf::SLOT_PAD;
-                acc = slot_block<DYN, COUNT, PF>(A, w.pb, more, min(W - k, PF), (sb + k) * 16 + lane, cd, staged, tb_abs,
-                                                  level, range_guard, x, acc, cnt);
+                acc = slot_block<DYN, STK, PF>(A, w.pb, more, min(W - k, PF), (sb + k) * 16 + lane, cd, staged, tb_abs, pv,
+                                               range_guard, acc);
             }
-            emit(w0 + li, lane, acc, ov);
+            emit(TR, lane, acc, ov);
         }
 #undef CMP_LOAD_FIRST
         w0 += nw;
     }
+}
+
+// Per-SpMV statistics (tile_level_counts, exact dynamic byte model): tiles and nonzeros of the
+// CTA's tile rows by effective precision.  Separate pass over the tile records (stats mode only).
+template <bool DYN>
+__device__ __forceinline__ void count_levels(const Mat& A, int64_t tr0c, int64_t tr1c, const double* pv, int range_guard, Counts* cnt) {
+    for (int64_t i = A.tr_tile[tr0c] + threadIdx.x; i < A.tr_tile[tr1c]; i += blockDim.x) {
+        const int e = (int)(tile_code<DYN>(A.tile_info[i], pv, range_guard) & 7u);
+        cnt->tile(e);
+        cnt->nzn(e, (int)(A.tile_nnz[i + 1] - A.tile_nnz[i]));
+    }
+}
+
+struct SpmvSmem {
+    WinSmem win;
+    TsSmem ts;
+};
+
+// carve the SpMV region: TS ring (nst slots of slot_bytes, 128-aligned) or the compact window
+// buffers (the two views overlap: a matrix uses one layout)
+__device__ __forceinline__ void carve_spmv(unsigned char* base, int nst, int slot_bytes, int blob_cap, int ecap, SpmvSmem& s) {
+    unsigned char* p = base;
+    s.ts.full = reinterpret_cast<unsigned long long*>(p);
+    s.ts.empty = s.ts.full + TS_NSTMAX;
+    s.ts.ctr = s.ts.empty + TS_NSTMAX;
+    p += TS_CTRL_BYTES;
+    p = base + ((int)(p - base) + 127) / 128 * 128;
+    s.ts.base = p;
+    s.ts.nst = nst;
+    s.ts.slot_bytes = slot_bytes;
+    s.ts.blob_cap = blob_cap;
+    s.ts.ecap = ecap;
+    s.ts.ebuf = reinterpret_cast<double*>(p + (size_t)nst * slot_bytes);
+    s.win.misc = reinterpret_cast<int64_t*>(p);
+    unsigned char* q = p + 4 * 8 + 8;
+    s.win.pb = reinterpret_cast<unsigned long long*>(q);
+    q += 4 * 8;
+    s.win.hs = reinterpret_cast<int32_t*>(q);
+    q += (WIN_TR + 1) * 4;
+    s.win.ht = reinterpret_cast<int32_t*>(q);
+    q += (WIN_TR + 1) * 4;
+    s.win.buf = p + ts_r16((int)(q - p));
+}
+// bytes of the SpMV region for a matrix (host): control words + max(ring + decode buffers, compact buffers)
+__host__ __device__ constexpr size_t spmv_smem_bytes(int ts, int nst, int slot_bytes, int ecap, int nwarps) {
+    return 128 + TS_CTRL_BYTES + (ts ? (size_t)nst * slot_bytes + (size_t)nwarps * ecap * 128 : WIN_SMEM_BYTES + 16);
+}
+
+// One SpMV of the CTA's tile rows [tr0, tr1): mu = A~_j v with v in PV layout (levels included).
+template <bool DYN, bool STK, int PF, class Emit>
+__device__ __forceinline__ void spmv_cta(const Mat& A, int64_t tr0, int64_t tr1, const double* pv, int range_guard,
+                                         const SpmvSmem& sm, int own_mode, const double* ownv, Emit emit) {
+    if (A.ts) spmv_ts<DYN, STK>(A, tr0, pv, range_guard, sm.ts, own_mode, ownv, emit);
+    else spmv_compact<DYN, STK, PF>(A, tr0, tr1, pv, range_guard, sm.win, own_mode, ownv, emit);
 }
 
 // Alg. 4 with the P:174 intervals (reading R5) on |v| (R7); NaN -> FP64.

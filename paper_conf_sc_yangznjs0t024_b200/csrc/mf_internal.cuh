@@ -82,9 +82,13 @@ struct TileMatrix {
     int64_t vbytes = 0;              // bytes of vstream
     uint8_t* blob = nullptr;         // tile-synchronous: per-stage blobs streamed by the TMA pipeline
     int64_t blob_bytes = 0;
-    void* stg = nullptr;             // tile-synchronous: mfk::PipeStage per stage of every CTA
+    void* stg = nullptr;             // tile-synchronous: mfk::TsStage per stage of every CTA
     int32_t* stg_ptr = nullptr;      // device [G+1]
     int64_t nstg = 0;
+    int32_t blob_cap = 0;            // tile-synchronous: largest stage blob (bytes, 128-aligned)
+    int32_t wcap = 0;                // tile-synchronous: largest stage window (column segments)
+    int32_t slot_bytes = 0;          // tile-synchronous: ring slot = blob_cap + wcap * 144 (128-aligned)
+    int32_t ecap = 0;                // tile-synchronous: most columns one warp decodes per stage
     // compact layout only: value planes RNE_q(stored value) per slot
     double* plane64 = nullptr;       // [16*slots] value at FP64 (tiles with TilePrec == FP64)
     float* plane32 = nullptr;        // value rounded to FP32 (tiles with TilePrec <= FP32)

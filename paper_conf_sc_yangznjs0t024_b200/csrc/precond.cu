@@ -143,11 +143,12 @@ mf_status ilu0(HostCSR& M, std::vector<int64_t>& diag) {
 template <bool FWD>
 __global__ void __launch_bounds__(256) sptrsv_kernel(TriCSR T, const double* __restrict__ diag, int64_t n,
                                                      const double* in, double* out, unsigned* flags, unsigned flag_val,
-                                                     unsigned wait_val, unsigned long long* ctr) {
+                                                     unsigned wait_val, unsigned long long* ctr, int* abort_flag) {
     __shared__ double ys[256];
     __shared__ int ready[256];
     __shared__ long long chunk;
-    mfk::sptrsv_chunked<FWD>(T.rp, T.ci, T.v, diag, n, in, out, flags, flag_val, wait_val, ctr, 0ull, ys, ready, &chunk);
+    mfk::sptrsv_chunked<FWD, false>(T.rp, T.ci, T.v, diag, n, in, out, flags, flag_val, wait_val, ctr, 0ull, ys, ready, &chunk,
+                                    abort_flag, 20ull * 1000000000ull);
 }
 
 template <class T>
@@ -170,10 +171,15 @@ mf_status run_precond_apply(Precond& P, const double* r, double* z, cudaStream_t
     }
     const unsigned e = ++P.epoch;
     const int blocks = (int)std::min<int64_t>((P.n + 255) / 256, (int64_t)sms * 8);
-    MF_CUDA(cudaMemsetAsync(P.ctr, 0, 2 * sizeof(unsigned long long), s));
-    sptrsv_kernel<true><<<blocks, 256, 0, s>>>(P.L, nullptr, P.n, r, P.y, P.flags, 2 * e + 1, 0u, P.ctr);
-    sptrsv_kernel<false><<<blocks, 256, 0, s>>>(P.U, P.udiag, P.n, P.y, z, P.flags, 2 * e + 2, 2 * e + 1, P.ctr + 1);
+    MF_CUDA(cudaMemsetAsync(P.ctr, 0, 3 * sizeof(unsigned long long), s));
+    int* abort_flag = reinterpret_cast<int*>(P.ctr + 2);
+    sptrsv_kernel<true><<<blocks, 256, 0, s>>>(P.L, nullptr, P.n, r, P.y, P.flags, 2 * e + 1, 0u, P.ctr, abort_flag);
+    sptrsv_kernel<false><<<blocks, 256, 0, s>>>(P.U, P.udiag, P.n, P.y, z, P.flags, 2 * e + 2, 2 * e + 1, P.ctr + 1, abort_flag);
     MF_CUDA(cudaGetLastError());
+    int ab = 0;
+    MF_CUDA(cudaMemcpyAsync(&ab, abort_flag, sizeof(int), cudaMemcpyDeviceToHost, s));
+    MF_CUDA(cudaStreamSynchronize(s));
+    if (ab) return fail(MF_ERR_DEADLOCK, "triangular-solve watchdog expired");
     return MF_OK;
 }
 

@@ -51,18 +51,44 @@ __device__ __forceinline__ void st_release_u32(unsigned* p, unsigned v) {
 // Chunks of blockDim.x consecutive rows (in solve order) are grabbed with one atomicAdd on
 // *ctr (values base, base+1, ...), so a chunk only waits on chunks grabbed earlier or on
 // earlier rows of its own chunk: deadlock-free without co-residency.  Inside a chunk a row
-// waits on a shared-memory flag; across chunks on the global row flag (== flag_val).
-// wait_val != 0: row i additionally waits for flags[i] == wait_val before reading in_i (the
-// backward solve waits for the forward solve of the same row).  Every CTA performs exactly one
-// failing grab, so one solve consumes ceil(n/B) + (number of CTAs) counter values.
-template <bool FWD>
+// waits on a shared-memory flag; across chunks on the global row flag.
+// Flag values are epochs that only grow (forward 2e+1 < backward 2e+2 < next forward ...), so
+// every wait is ">=": a row whose flag already moved on to a later solve of the same apply (the
+// backward solve of a nonsymmetric pattern can finish row k before a forward row that reads it)
+// never blocks a reader.  wait_val != 0: row i additionally waits for flags[i] >= wait_val
+// before reading in_i (the backward solve waits for the forward solve of the same row).
+// OUTPV: out is in the PV layout (kernels.cuh) -- the SpMV input of the preconditioned solvers.
+// Every spin has a watchdog: after timeout_ns (or when another CTA raised *abort_flag) the
+// thread stops waiting, raises *abort_flag and the caller reports MF_ERR_DEADLOCK.
+// Every CTA performs exactly one failing grab, so one solve consumes ceil(n/B) + (number of
+// CTAs) counter values.
+__device__ __forceinline__ unsigned long long sp_timer() {
+    unsigned long long t;
+    asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
+    return t;
+}
+// spin until *f >= v; false on watchdog / abort
+__device__ __forceinline__ bool sp_wait_flag(const unsigned* f, unsigned v, int* abort_flag, unsigned long long t0,
+                                             unsigned long long timeout_ns) {
+    if (ld_acquire_u32(f) >= v) return true;
+    for (unsigned k = 0;; ++k) {
+        if (ld_acquire_u32(f) >= v) return true;
+        if ((k & 63u) == 63u) {
+            if (*(volatile int*)abort_flag) return false;
+            if (sp_timer() - t0 > timeout_ns) { atomicExch(abort_flag, 1); return false; }
+        }
+    }
+}
+template <bool FWD, bool OUTPV>
 __device__ void sptrsv_chunked(const int64_t* __restrict__ rp, const int32_t* __restrict__ ci,
                                const double* __restrict__ val, const double* __restrict__ diag, int64_t n,
                                const double* in, double* out, unsigned* flags, unsigned flag_val, unsigned wait_val,
                                unsigned long long* ctr, unsigned long long base, double* ys, volatile int* ready,
-                               long long* s_chunk) {
+                               long long* s_chunk, int* abort_flag, unsigned long long timeout_ns) {
     const int B = blockDim.x, t = threadIdx.x;
     const int64_t nchunks = (n + B - 1) / B;
+    const unsigned long long t0 = sp_timer();
+    auto oidx = [](int64_t i) -> int64_t { return OUTPV ? ((i >> 4) * 18 + (i & 15)) : i; };
     while (true) {
         __syncthreads();
         if (t == 0) *s_chunk = (long long)(atomicAdd(ctr, 1ull) - base);
@@ -73,8 +99,7 @@ __device__ void sptrsv_chunked(const int64_t* __restrict__ rp, const int32_t* __
         const int64_t pos = c * B + t;                 // position in solve order
         if (pos < n) {
             const int64_t i = FWD ? pos : n - 1 - pos;
-            if (wait_val)
-                while (ld_acquire_u32(&flags[i]) != wait_val) { }
+            if (wait_val) sp_wait_flag(&flags[i], wait_val, abort_flag, t0, timeout_ns);
             double acc = __ldcg(in + i);
             const int64_t lo = rp[i], hi = rp[i + 1];
             for (int64_t q = lo; q < hi; ++q) {
@@ -83,17 +108,21 @@ __device__ void sptrsv_chunked(const int64_t* __restrict__ rp, const int32_t* __
                 double xk;
                 if (pk >= c * B) {
                     const int lk = (int)(pk - c * B);
-                    while (ready[lk] == 0) { }
+                    for (unsigned sp = 0; ready[lk] == 0; ++sp)
+                        if ((sp & 255u) == 255u && (*(volatile int*)abort_flag || sp_timer() - t0 > timeout_ns)) {
+                            atomicExch(abort_flag, 1);
+                            break;
+                        }
                     xk = ((volatile double*)ys)[lk];
                 } else {
-                    while (ld_acquire_u32(&flags[k]) != flag_val) { }
-                    xk = __ldcg(out + k);
+                    sp_wait_flag(&flags[k], flag_val, abort_flag, t0, timeout_ns);
+                    xk = __ldcg(out + oidx(k));
                 }
                 acc = __fma_rn(-val[q], xk, acc);
             }
             if (!FWD) acc = __ddiv_rn(acc, diag[i]);
             ys[t] = acc;
-            out[i] = acc;
+            out[oidx(i)] = acc;
             __threadfence();
             ready[t] = 1;
             st_release_u32(&flags[i], flag_val);
