@@ -155,7 +155,14 @@ __global__ void __launch_bounds__(THREADS) tile_row_kernel(int64_t n_rows, int64
         const int minrc = hw_min<int>(rc, m);
         const int floor_t = minrc > best ? minrc : best;
         const int tile_nz = hw_sum<int>(cnt_r, m);
-        const int w_j = hw_max<int>(cnt_r, m);              // slice columns of this tile (TS layout)
+        // tile-synchronous layout: one slice column per diagonal (local column - local row) that
+        // holds an entry of the tile, diagonals ascending (so each row's entries stay in ascending
+        // column order); compact layout: the row-packed width
+        unsigned dmask = 0;
+        if (mine)
+            for (int64_t k = ptr; k < q; ++k) dmask |= 1u << ((colidx[k] & 15) - lane + 15);
+        dmask = __reduce_or_sync(m, dmask);
+        const int w_j = __popc(dmask);                      // slice columns of this tile (TS layout)
         const unsigned bal = __ballot_sync(m, mine) >> (threadIdx.x & 16);
         const int rows_in_tile = __popc(bal);
         if (FILL) {
@@ -192,12 +199,12 @@ __global__ void __launch_bounds__(THREADS) tile_row_kernel(int64_t n_rows, int64
                     }
                     // kernel layout: compact slot (k - rstart) of this row, or tile-synchronous column
                     // colbase + (k - ptr); value planes RNE_q(stored) for q at or below TilePrec
-                    const int64_t pos = o.ts ? (slot0 + colbase + (k - ptr)) * TS + lane
+                    const int di = __popc(dmask & ((1u << (lc - lane + 15)) - 1u));   // diagonal slice of the entry
+                    const int64_t pos = o.ts ? (slot0 + colbase + di) * TS + lane
                                              : (slot0 + (k - rstart)) * TS + lane;
                     if (o.ts) {
-                        o.sslot[pos] = (uint8_t)lc;
-                        // value stream: column (colbase + k - ptr) of the tile row, 16 * size(TilePrec) bytes
-                        const int64_t vb = vb0 + vb_run + ((k - ptr) * 16 + lane) * (8 >> best);
+                        // value stream: slice column (colbase + di) of the tile row, 16 * size(TilePrec) bytes
+                        const int64_t vb = vb0 + vb_run + ((int64_t)di * 16 + lane) * (8 >> best);
                         switch (best) {
                         case 0: *reinterpret_cast<double*>(o.vstream + vb) = sv; break;
                         case 1: *reinterpret_cast<float*>(o.vstream + vb) = (float)sv; break;
@@ -215,9 +222,14 @@ __global__ void __launch_bounds__(THREADS) tile_row_kernel(int64_t n_rows, int64
             }
         }
         // static column record: word, value offset within the tile row (stage_kernel rebases it)
-        if (FILL && o.ts && lane < w_j)
+        if (FILL && o.ts && lane < w_j) {
+            // slice `lane` of the tile: its diagonal (the lane-th set bit of dmask) in bits 24..28
+            unsigned mm = dmask;
+            for (int z = 0; z < lane; ++z) mm &= mm - 1u;
+            const uint32_t dg = (uint32_t)(__ffs(mm) - 1);    // diagonal + 15
             o.crec[slot0 + colbase + lane] = make_uint2(((uint32_t)tc << 4) | ((uint32_t)floor_t << 2) | (uint32_t)best,
-                                                        (uint32_t)(vb_run + (int64_t)lane * 16 * (8 >> best)));
+                                                        (uint32_t)(vb_run + (int64_t)lane * 16 * (8 >> best)) | (dg << 24));
+        }
         if (mine) { ptr = q; cur = ptr < rend ? (colidx[ptr] >> 4) : INT32_MAX; }
         ++j;
         colbase += w_j;
@@ -491,16 +503,14 @@ __global__ void __launch_bounds__(RUNS_T) runs_kernel(mfk::TsStage* stg, const i
 // Blob of each stage (layout in kernels.cuh): its byte size, then, after an exclusive scan of the
 // sizes, its contents.  One block of TS_CCAP threads per stage: thread c owns column c.
 struct BlobLayout {
-    int off_eb, off_desc, off_lc, off_wl, off_ent, off_val, bytes;
+    int off_desc, off_wl, off_gd, off_val, bytes;
 };
 __host__ __device__ __forceinline__ BlobLayout blob_layout(int K, int64_t nc, int64_t nv, int NW) {
     BlobLayout L;
-    L.off_eb = mfk::TS_HDR + mfk::ts_r16((K + 1) * 2);
-    L.off_desc = L.off_eb + mfk::ts_r16(K);
-    L.off_lc = L.off_desc + mfk::ts_r16(((int)nc + mfk::TS_DPAD) * 4);
-    L.off_wl = L.off_lc + ((int)nc + mfk::TS_DPAD) * 16;
-    L.off_ent = L.off_wl + mfk::ts_r16(NW * 4) + mfk::ts_r16(NW * 2);
-    L.off_val = L.off_ent + mfk::ts_r16((int)nc * 2);
+    L.off_desc = mfk::TS_HDR + mfk::ts_r16((K + 1) * 2);
+    L.off_wl = L.off_desc + mfk::ts_r16(((int)nc + mfk::TS_DPAD) * 4);
+    L.off_gd = L.off_wl + NW * 16;
+    L.off_val = L.off_gd + mfk::ts_r16((int)nc * 4);
     L.bytes = L.off_val + (int)nv;
     return L;
 }
@@ -518,13 +528,16 @@ __device__ int owner_cta(const int32_t* plan_tr, int G, int64_t TR) {
 }
 __global__ void __launch_bounds__(mfk::TS_CCAP) blob_fill_kernel(mfk::TsStage* stg, const int64_t* __restrict__ boff,
                                                                    const int64_t* __restrict__ tr_slot, const int64_t* __restrict__ tr_vb,
-                                                                   const uint2* __restrict__ crec, const uint8_t* __restrict__ sslot,
+                                                                   const uint2* __restrict__ crec,
                                                                    const uint8_t* __restrict__ vstream, uint8_t* blob,
                                                                    const int32_t* __restrict__ plan_tr, int G, int H,
                                                                    unsigned long long* maxb) {
     __shared__ int32_t hdr[mfk::TS_KCAP + 1];
-    __shared__ int32_t ebase[mfk::TS_KCAP];       // first E slot of each tile row within its warp's buffer
-    __shared__ int32_t wcols[32], woffs[33];      // columns per warp, list offsets
+    __shared__ int16_t cw[mfk::TS_KCAP];                 // warp of each tile row
+    __shared__ uint8_t cq[mfk::TS_CCAP];                 // TilePrec of each column
+    __shared__ int32_t cdst[mfk::TS_CCAP];               // value byte offset of each column (grouped order)
+    __shared__ uint8_t cslot[mfk::TS_CCAP];              // decode-buffer slot of each column
+    __shared__ int32_t wcol[33], wval[33];               // columns / value bytes per warp, exclusive prefixes
     const int64_t sidx = blockIdx.x;
     const mfk::TsStage st = stg[sidx];
     const int K = st.tr1 - st.tr0, c = threadIdx.x;
@@ -537,6 +550,12 @@ __global__ void __launch_bounds__(mfk::TS_CCAP) blob_fill_kernel(mfk::TsStage* s
     for (int k = c; k <= K; k += blockDim.x) {
         hdr[k] = (int32_t)(tr_slot[st.tr0 + k] - col0);
         reinterpret_cast<int16_t*>(b + mfk::TS_HDR)[k] = (int16_t)hdr[k];
+        if (k < K) cw[k] = (int16_t)((int)((st.tr0 + k - tr0c) % H) >> 1);
+    }
+    uint2 rc = make_uint2(0u, 0u);
+    if (c < nc) {
+        rc = crec[col0 + c];
+        cq[c] = (uint8_t)(rc.x & 3u);
     }
     __syncthreads();
     if (c == 0) {
@@ -545,66 +564,70 @@ __global__ void __launch_bounds__(mfk::TS_CCAP) blob_fill_kernel(mfk::TsStage* s
         for (int i = 0; i < st.nrun; ++i)
             if (st.run_s[i] <= st.tr0 && st.tr1 <= st.run_s[i] + st.run_n[i]) own = st.run_w[i] + (st.tr0 - st.run_s[i]);
         int32_t* h = reinterpret_cast<int32_t*>(b);
-        h[0] = st.tr0; h[1] = st.tr1; h[2] = nc; h[3] = L.off_desc; h[4] = L.off_lc; h[5] = L.off_val; h[6] = own;
+        h[0] = st.tr0; h[1] = st.tr1; h[2] = nc; h[3] = L.off_desc; h[4] = 0; h[5] = L.off_val; h[6] = own;
         h[7] = (int32_t)(uint32_t)(uint64_t)col0; h[8] = (int32_t)(uint32_t)((uint64_t)col0 >> 32);
-        h[9] = L.off_wl; h[10] = L.off_ent; h[11] = L.off_eb;
+        h[9] = L.off_wl; h[10] = L.off_gd; h[11] = (int32_t)((st.tr0 - tr0c) % H);   // off0: half-warp of tile row tr0
         for (int k = 12; k < 16; ++k) h[k] = 0;
-        // E slots: the columns of a warp's tile rows (half-warps 2w, 2w+1), in column order
-        for (int w = 0; w < NW; ++w) wcols[w] = 0;
-        for (int k = 0; k < K; ++k) {
-            const int w = (int)((st.tr0 + k - tr0c) % H) >> 1;
-            ebase[k] = wcols[w];
-            b[L.off_eb + k] = (uint8_t)min(wcols[w], 255);
-            wcols[w] += hdr[k + 1] - hdr[k];
+        wcol[0] = 0; wval[0] = 0;
+        for (int w = 0; w < NW; ++w) {
+            int nw = 0, vw = 0;
+            for (int k = 0; k < K; ++k)
+                if (cw[k] == w)
+                    for (int cc = hdr[k]; cc < hdr[k + 1]; ++cc) { ++nw; vw += 16 * (8 >> cq[cc]); }
+            wcol[w + 1] = wcol[w] + nw;
+            wval[w + 1] = wval[w] + vw;
         }
-        woffs[0] = 0;
-        int mx = 0;
-        for (int w = 0; w < NW; ++w) { woffs[w + 1] = woffs[w] + wcols[w]; mx = max(mx, wcols[w]); }
-        atomicMax(maxb + 1, (unsigned long long)mx);
     }
     __syncthreads();
-    if (c < nc) {
-        const uint2 rc = crec[col0 + c];
-        const uint32_t tc = rc.x >> 4;
-        int lo = 0, hi = K - 1;                              // tile row of column c
-        while (lo < hi) { const int mid = (lo + hi + 1) / 2; if (hdr[mid] <= c) lo = mid; else hi = mid - 1; }
-        const int64_t voff = tr_vb[st.tr0 + lo] - vb0 + rc.y;   // column order == vstream order
-        int wseg = 0;
-        for (int i = 0; i < st.nrun; ++i)
-            if ((int64_t)tc >= st.run_s[i] && (int64_t)tc < (int64_t)st.run_s[i] + st.run_n[i]) wseg = st.run_w[i] + (int)(tc - st.run_s[i]);
-        reinterpret_cast<uint32_t*>(b + L.off_desc)[c] =
-            (rc.x & 15u) | ((uint32_t)(voff >> 4) << 4) | ((uint32_t)(wseg * mfk::PV_SEG_BYTES) << 16);
-        uint4 l16 = reinterpret_cast<const uint4*>(sslot)[col0 + c];      // local columns, stored x8 (byte offsets)
-        l16.x <<= 3; l16.y <<= 3; l16.z <<= 3; l16.w <<= 3;
-        reinterpret_cast<uint4*>(b + L.off_lc)[c] = l16;
-    }
-    if (c < mfk::TS_DPAD) {                                // padding read by short rows
-        reinterpret_cast<uint32_t*>(b + L.off_desc)[nc + c] = 0u;
-        reinterpret_cast<uint4*>(b + L.off_lc)[nc + c] = make_uint4(0u, 0u, 0u, 0u);
-    }
     if (c < NW) {
-        // decode list of warp c: its columns grouped by TilePrec (FP64 | FP32 | FP16 | E4M3), ascending
+        // warp c: its columns grouped by TilePrec (FP64 | FP32 | FP16 | E4M3), ascending within a
+        // group; the group order gives each column its decode-buffer slot and its value position
         const int w = c;
         uint32_t cnt = 0;
-        uint16_t* ent = reinterpret_cast<uint16_t*>(b + L.off_ent) + woffs[w];
-        int pos = 0;
+        int slot = 0, voff = wval[w];
+        uint32_t* gd = reinterpret_cast<uint32_t*>(b + L.off_gd) + wcol[w];
         for (int q = 0; q < 4; ++q) {
             int nq = 0;
             for (int k = 0; k < K; ++k) {
-                if (((int)((st.tr0 + k - tr0c) % H) >> 1) != w) continue;
+                if (cw[k] != w) continue;
                 for (int cc = hdr[k]; cc < hdr[k + 1]; ++cc)
-                    if ((int)(crec[col0 + cc].x & 3u) == q) {
-                        ent[pos++] = (uint16_t)(cc | ((ebase[k] + cc - hdr[k]) << 9));   // column | E slot << 9
-                        ++nq;
+                    if (cq[cc] == q) {
+                        const uint2 r2 = crec[col0 + cc];
+                        cslot[cc] = (uint8_t)slot;      // decode-buffer slot: rank in the warp's grouped order
+                        cdst[cc] = voff;
+                        gd[slot] = ((uint32_t)((r2.x >> 2) & 3u) << 16) | ((uint32_t)cc << 20);   // + window offset below
+                        ++slot; ++nq;
+                        voff += 16 * (8 >> q);
                     }
             }
             cnt |= (uint32_t)min(nq, 255) << (8 * q);
         }
-        reinterpret_cast<uint32_t*>(b + L.off_wl)[w] = cnt;
-        reinterpret_cast<uint16_t*>(b + L.off_wl + mfk::ts_r16(NW * 4))[w] = (uint16_t)woffs[w];
+        reinterpret_cast<uint4*>(b + L.off_wl)[w] = make_uint4(cnt, (uint32_t)wval[w], (uint32_t)wcol[w], 0u);
+        atomicMax(maxb + 1, (unsigned long long)slot);
     }
-    for (int64_t k = c; k < nv / 16; k += blockDim.x)
-        reinterpret_cast<uint4*>(b + L.off_val)[k] = reinterpret_cast<const uint4*>(vstream + vb0)[k];
+    __syncthreads();
+    if (c < nc) {
+        const uint32_t tc = rc.x >> 4;
+        int lo = 0, hi = K - 1;                              // tile row of column c
+        while (lo < hi) { const int mid = (lo + hi + 1) / 2; if (hdr[mid] <= c) lo = mid; else hi = mid - 1; }
+        int wseg = 0;
+        for (int i = 0; i < st.nrun; ++i)
+            if ((int64_t)tc >= st.run_s[i] && (int64_t)tc < (int64_t)st.run_s[i] + st.run_n[i]) wseg = st.run_w[i] + (int)(tc - st.run_s[i]);
+        const uint32_t woff = (uint32_t)(wseg * mfk::PV_SEG_BYTES);
+        const int dg = (int)((rc.y >> 24) & 31u) - 15;      // diagonal of the slice column
+        // x of lane r is window element 16 * wseg + r + dg: byte offset from the window guard
+        const uint32_t xoff = (uint32_t)(mfk::TS_GUARD + (int)woff + 8 * dg);
+        reinterpret_cast<uint32_t*>(b + L.off_desc)[c] = xoff | ((uint32_t)cslot[c] << 16);
+        reinterpret_cast<uint32_t*>(b + L.off_gd)[wcol[cw[lo]] + cslot[c]] |= woff;
+        // values of column c (16 x size(TilePrec) bytes, column order in vstream) -> grouped position
+        const int64_t src = tr_vb[st.tr0 + lo] + (rc.y & 0xFFFFFFu);
+        const int n16 = 8 >> cq[c];
+        const uint4* sp = reinterpret_cast<const uint4*>(vstream + src);
+        uint4* dp = reinterpret_cast<uint4*>(b + L.off_val + cdst[c]);
+        for (int k = 0; k < n16; ++k) dp[k] = sp[k];
+    }
+    if (c < mfk::TS_DPAD)                                  // padding read by short rows: x = guard, slot 0
+        reinterpret_cast<uint32_t*>(b + L.off_desc)[nc + c] = (uint32_t)mfk::TS_GUARD;
     if (c == 0) {
         stg[sidx].boff_lo = (uint32_t)(uint64_t)boff[sidx];
         stg[sidx].boff_hi = (uint32_t)((uint64_t)boff[sidx] >> 32);
@@ -718,11 +741,9 @@ mf_status convert_csr(int64_t n_rows, int64_t n_cols, int64_t nnz, const int64_t
     A->vbytes = A->ts ? tot[CNT_VB] : 0;
     if (A->ts) {
         // padded so that the pipeline's 16-byte aligned bulk copies stay inside the arrays
-        MF_TRY(alloc(&A->sslot, nslot + 16, s));
         MF_TRY(alloc(&A->crec, A->slots + 8, s));
         MF_TRY(alloc(&A->vstream, A->vbytes + 64, s));
         MF_TRY(alloc(&A->tr_vb, ntr + 4, s));
-        MF_CUDA(cudaMemsetAsync(A->sslot, 0, nslot + 16, s));
         MF_CUDA(cudaMemsetAsync(A->crec, 0, (A->slots + 8) * sizeof(uint2), s));
         MF_CUDA(cudaMemsetAsync(A->vstream, 0, A->vbytes + 64, s));
         MF_CUDA(cudaMemsetAsync(A->tr_vb, 0, (ntr + 4) * sizeof(int64_t), s));
@@ -799,8 +820,9 @@ mf_status convert_csr(int64_t n_rows, int64_t n_cols, int64_t nnz, const int64_t
         std::vector<int32_t> nst_h(G), sp_h(G + 1);
         // the window of a stage grows with its tile rows: halve the stage cap until every
         // stage's window fits TS_WCAP segments
-        // one tile row per half-warp per stage (K = H) keeps the warp-private decode buffers small
-        for (int kcap = std::min(mfk::TS_KCAP, std::max(1, B / 16));; kcap /= 2) {
+        // two tile rows per half-warp per stage (K = 2H: two independent fma chains per lane), halved
+        // until every stage window fits
+        for (int kcap = std::min(mfk::TS_KCAP, std::max(1, B / 8));; kcap /= 2) {
             stage_kernel<false><<<G, 32, 0, s>>>(A->plan_tr, G, B / 16, kcap, A->tr_slot, A->tr_vb, nst, nullptr, nullptr);
             MF_CUDA(cudaGetLastError());
             MF_CUDA(cudaMemcpyAsync(nst_h.data(), nst, G * sizeof(int32_t), cudaMemcpyDeviceToHost, s));
@@ -839,7 +861,7 @@ mf_status convert_csr(int64_t n_rows, int64_t n_cols, int64_t nnz, const int64_t
             MF_CUDA(cudaMemcpyAsync(&A->blob_bytes, boff + A->nstg, sizeof(int64_t), cudaMemcpyDeviceToHost, s));
             MF_CUDA(cudaStreamSynchronize(s));
             MF_TRY(alloc(&A->blob, A->blob_bytes + 64, s));
-            blob_fill_kernel<<<(unsigned)A->nstg, mfk::TS_CCAP, 0, s>>>(static_cast<mfk::TsStage*>(A->stg), boff, A->tr_slot, A->tr_vb, A->crec, A->sslot,
+            blob_fill_kernel<<<(unsigned)A->nstg, mfk::TS_CCAP, 0, s>>>(static_cast<mfk::TsStage*>(A->stg), boff, A->tr_slot, A->tr_vb, A->crec,
                                                                        A->vstream, A->blob, A->plan_tr, G, B / 16, dmax + 1);
             MF_CUDA(cudaGetLastError());
             unsigned long long mb[2] = {0, 0};
@@ -848,8 +870,8 @@ mf_status convert_csr(int64_t n_rows, int64_t n_cols, int64_t nnz, const int64_t
             A->blob_cap = (int32_t)((mb[0] + 127) / 128 * 128);
             A->ecap = (int32_t)mb[1];
             // the warp-private decode buffers must leave room for the ring (TS_EBYTES of shared memory)
-            if ((int64_t)A->ecap * 128 * (B / 32) > mfk::TS_EBYTES || A->ecap > 127) ts_failed = true;
-            A->slot_bytes = (int32_t)((A->blob_cap + (int64_t)A->wcap * mfk::PV_SEG_BYTES + 127) / 128 * 128);
+            if ((int64_t)A->ecap * 128 * (B / 32) > mfk::TS_EBYTES || A->ecap > 255) ts_failed = true;
+            A->slot_bytes = (int32_t)((A->blob_cap + mfk::TS_GUARD + (int64_t)A->wcap * mfk::PV_SEG_BYTES + 127) / 128 * 128);
             dev_free(bsz, s); dev_free(boff, s); dev_free(btmp, s);
         }
         dev_free(nst, s);

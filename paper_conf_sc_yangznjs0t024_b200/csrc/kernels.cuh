@@ -36,7 +36,6 @@ struct Mat {
     const uint8_t* __restrict__ p8;
     uint8_t* stk;                         // sticky variant (P:237 literal): per slice column (TS layout) or
                                           // per tile (compact), bit L set = values lowered to L in place
-    int dbg;                              // diagnostics (MF_SPMV_DBG): 1 = stream the stages, skip the rows
 };
 
 // ------------------------------------------------------------------------------------------
@@ -129,16 +128,17 @@ struct Counts {
 // dot-product contract), so warp w owns the rows of half-warps 2w and 2w+1.  Conversion cuts the
 // CTA's tile rows into stages (one tile row per half-warp by default) and packs each stage into
 // ONE contiguous blob:
-//   [int32 hdr[16]: tr0, tr1, nc, off_desc, off_lc, off_val, own_w, col0 lo, col0 hi, off_wl,
-//    off_ent, off_eb]
+//   [int32 hdr[16]: tr0, tr1, nc, off_desc, -, off_val, own_w, col0 lo, col0 hi, off_wl, off_gd]
 //   [int16 column start per tile-row boundary, K+1 entries]
-//   [u8 first decode-buffer slot of each tile row (its columns take consecutive slots)]
-//   [u32 desc per column: TilePrec | Floor << 2 | value offset (16 B units) << 4 | window byte
-//    offset of its column segment << 16; TS_DPAD zero entries after the last column]
-//   [u8 local column x 8 (byte offset within the segment) [col][lane]]
-//   [per warp: u32 column counts per TilePrec group (4 x u8); u16 offset of its decode list]
-//   [u16 decode lists: column | slot << 9, each warp's columns grouped by TilePrec]
-//   [values in column order, 16 x size(TilePrec) bytes per column]
+//   [u32 desc per column: x offset | slot << 16; TS_DPAD padding entries]
+//   [per warp uint4: column counts per TilePrec group (4 x u8), value offset, gd offset]
+//   [u32 gd per column in each warp's grouped order: window byte offset | Floor << 16 | column << 20]
+//   [values: per warp, its columns grouped by TilePrec (FP64 | FP32 | FP16 | E4M3), 16 x size each]
+// A slice column holds ONE diagonal of its tile (local column - local row = d, diagonals in
+// ascending order), so lane r's x is window element 16 w + r + d: the descriptor carries the byte
+// offset of element 16 w + d from the slot's zero guard (padding lanes read finite values).  The
+// decode-buffer slot of a column is its rank in the warp's grouped order, so the decode is a
+// linear stream per group (no per-value indirection).
 // The stage record (TsStage, 32 words) lists the runs of consecutive column segments the stage
 // gathers ("x windows"); the runs are bulk-copied from the PV vector next to the blob.
 //
@@ -152,13 +152,14 @@ struct Counts {
 constexpr int TS_KCAP = 64;       // tile rows per stage
 constexpr int TS_CCAP = 512;      // slice columns per stage
 constexpr int TS_VCAP = 16384;    // value bytes per stage
-constexpr int TS_WCAP = 160;      // window segments per stage
+constexpr int TS_WCAP = 224;      // window segments per stage
 constexpr int TS_RUNCAP = 8;      // runs per stage
 constexpr int TS_NSTMAX = 6;      // slots in the ring
 constexpr int TS_HDR = 64;        // blob header bytes
 constexpr int TS_PF = 4;          // stage records prefetched ahead by the issuing warp
-constexpr int TS_EBYTES = 65536;  // most shared memory the warp-private decode buffers may take
-constexpr int TS_DPAD = 16;       // zero column descriptors after the last column (short-row reads)
+constexpr int TS_EBYTES = 98304;  // most shared memory the warp-private decode buffers may take
+constexpr int TS_DPAD = 16;       // padding column descriptors after the last column (short-row reads)
+constexpr int TS_GUARD = 128;     // zero bytes before each slot's x window (reads of padding lanes)
 __host__ __device__ constexpr int ts_r16(int v) { return (v + 15) & ~15; }
 
 // stage record: 32 words, word l read by lane l of the issuing warp
@@ -201,12 +202,18 @@ __device__ __forceinline__ bool mbar_try(unsigned long long* b, unsigned parity)
     return ok != 0;
 }
 // bounded wait: a pipeline that cannot complete traps (kernel error) instead of hanging the GPU
+__device__ __forceinline__ bool mbar_try_suspend(unsigned long long* b, unsigned parity) {
+    unsigned ok;
+    asm volatile("{\n\t.reg .pred p;\n\tmbarrier.try_wait.parity.shared::cta.b64 p, [%1], %2, %3;\n\tselp.u32 %0, 1, 0, p;\n\t}"
+                 : "=r"(ok) : "r"(smem_u32(b)), "r"(parity), "r"(2000u) : "memory");
+    return ok != 0;
+}
 static __device__ __noinline__ void mbar_wait_slow(unsigned long long* b, unsigned parity) {
     unsigned long long t0;
     asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t0));
     for (unsigned k = 1;; ++k) {
-        if (mbar_try(b, parity)) return;
-        if ((k & 1023u) == 0) {
+        if (mbar_try_suspend(b, parity)) return;   // the warp sleeps (<= 2 us) until the phase completes
+        if ((k & 63u) == 0) {
             unsigned long long t1;
             asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t1));
             if (t1 - t0 > 20ull * 1000000000ull) __trap();
@@ -234,6 +241,9 @@ __device__ __forceinline__ void bulk_g2s(void* dst, const void* src, unsigned by
 
 // all threads; followed by a __syncthreads of the caller before the first SpMV
 __device__ __forceinline__ void ts_init(const TsSmem& sm) {
+    for (int s = 0; s < sm.nst; ++s)      // the zero guard before each slot's window (never a TMA target)
+        for (int i = threadIdx.x; i < TS_GUARD / 8; i += blockDim.x)
+            reinterpret_cast<double*>(sm.slot(s) + sm.blob_cap)[i] = 0.0;
     if (threadIdx.x == 0) {
         for (int s = 0; s < TS_NSTMAX; ++s) {
             mbar_init(sm.full + s, 1);
@@ -248,21 +258,18 @@ __device__ __forceinline__ void ts_init(const TsSmem& sm) {
 // Warp 0: stage record word l in lane l (rec).  Lane 0 posts the transaction bytes, then lane r
 // (r < nrun) copies window run r and lane 31 the blob.
 __device__ __forceinline__ void ts_issue(const unsigned char* blob_base, uint32_t rec, unsigned char* slot, int blob_cap,
-                                         unsigned long long* full, const double* pv, bool with_blob, unsigned long long pol,
-                                         int dbg = 0) {
+                                         unsigned long long* full, const double* pv, bool with_blob, unsigned long long pol) {
     const int lane = threadIdx.x & 31;
     const uint32_t boff_lo = __shfl_sync(0xffffffffu, rec, 0), boff_hi = __shfl_sync(0xffffffffu, rec, 1);
     const int bbytes = (int)__shfl_sync(0xffffffffu, rec, 2), nrun = (int)__shfl_sync(0xffffffffu, rec, 3);
-    int wseg = (int)__shfl_sync(0xffffffffu, rec, 4);
-    if (dbg == 2) wseg = 0;                   // diagnostics: blobs only
-    if (dbg == 3) with_blob = false;          // diagnostics: windows only
+    const int wseg = (int)__shfl_sync(0xffffffffu, rec, 4);
     const int rs = (int)__shfl_sync(0xffffffffu, rec, 8 + (lane & 7));
     const int rn = (int)__shfl_sync(0xffffffffu, rec, 16 + (lane & 7));
     const int rw = (int)__shfl_sync(0xffffffffu, rec, 24 + (lane & 7));
     if (lane == 0) mbar_expect_tx(full, (unsigned)((with_blob ? bbytes : 0) + wseg * PV_SEG_BYTES));
     __syncwarp();
-    if (lane < nrun && lane < TS_RUNCAP && dbg != 2)
-        bulk_g2s(slot + blob_cap + rw * PV_SEG_BYTES, pv + (int64_t)rs * PVS, (unsigned)(rn * PV_SEG_BYTES), full);
+    if (lane < nrun && lane < TS_RUNCAP)
+        bulk_g2s(slot + blob_cap + TS_GUARD + rw * PV_SEG_BYTES, pv + (int64_t)rs * PVS, (unsigned)(rn * PV_SEG_BYTES), full);
     if (lane == 31 && with_blob) {
         const uint64_t boff = ((uint64_t)boff_hi << 32) | boff_lo;
         bulk_g2s_ef(slot, blob_base + boff, (unsigned)bbytes, full, pol);
@@ -284,41 +291,44 @@ __device__ __forceinline__ double e4m3_lo(uint32_t w2) {   // the E4M3 byte in b
     return (double)__half2float(__half(h));
 }
 __device__ __forceinline__ double h16(uint32_t bits) { return (double)__half2float(__ushort_as_half((unsigned short)bits)); }
+__device__ __forceinline__ float f16f(uint32_t bits) { return __half2float(__ushort_as_half((unsigned short)bits)); }
+__device__ __forceinline__ float e4m3f(uint32_t w2) {      // the E4M3 byte in bits 0..7 -> binary32 (exact)
+    const __half_raw h = __nv_cvt_fp8_to_halfraw((__nv_fp8_storage_t)(w2 & 0xFFu), __NV_E4M3);
+    return __half2float(__half(h));
+}
 
-// view of one landed stage
+// view of one landed stage (header: three 16-byte loads)
 struct TsView {
     const unsigned char* blob;
     const double* win;
-    int S0, S1, off_desc, off_lc, off_val, own_w, off_wl, off_ent, off_eb;
+    int S0, S1, off_desc, off_val, own_w, off_wl, off_gd, off0;
     int64_t col0;
 };
 __device__ __forceinline__ TsView ts_view(const unsigned char* slot, int blob_cap) {
     TsView v;
-    const int32_t* h = reinterpret_cast<const int32_t*>(slot);
+    const int4 h0 = reinterpret_cast<const int4*>(slot)[0];
+    const int4 h1 = reinterpret_cast<const int4*>(slot)[1];
+    const int4 h2 = reinterpret_cast<const int4*>(slot)[2];
     v.blob = slot;
-    v.win = reinterpret_cast<const double*>(slot + blob_cap);
-    v.S0 = h[0]; v.S1 = h[1];
-    v.off_desc = h[3]; v.off_lc = h[4]; v.off_val = h[5]; v.own_w = h[6];
-    v.col0 = (int64_t)(((uint64_t)(uint32_t)h[8] << 32) | (uint32_t)h[7]);
-    v.off_wl = h[9]; v.off_ent = h[10]; v.off_eb = h[11];
+    v.win = reinterpret_cast<const double*>(slot + blob_cap + TS_GUARD);
+    v.S0 = h0.x; v.S1 = h0.y; v.off_desc = h0.w;
+    v.off_val = h1.y; v.own_w = h1.z;
+    v.col0 = (int64_t)(((uint64_t)(uint32_t)h2.x << 32) | (uint32_t)h1.w);
+    v.off_wl = h2.y; v.off_gd = h2.z; v.off0 = h2.w;
     return v;
 }
 
-// Decode of one warp's columns into its buffer E (Q: the group's TilePrec, warp-uniform).  Unit u
-// = 4 lanes of one column.  Dynamic switch (Alg. 5 l.2-4, range guard R19): bypass -> 0, e_t below
-// TilePrec -> RNE_{e_t}(stored).  Sticky variant (P:237 literal): the column's mask of the levels
-// it was lowered to in place (Mat::stk, per slice column); the working value is RNE applied at
-// every lowered level in ascending order (successive rounding).
+// Decode of one warp's group of n columns at TilePrec Q (warp-uniform) into its buffer E: values
+// vb[0 .. 16n) -> E[slot0*16 ..), 4 values per lane per step, exact upcast.  Dynamic switch (Alg. 5
+// l.2-4, range guard R19): bypass -> 0, e_t below TilePrec -> RNE_{e_t}(stored).  Sticky variant
+// (P:237 literal): the column's mask of the levels it was lowered to in place (Mat::stk, per slice
+// column); the working value is RNE applied at every lowered level in ascending order.
 template <int Q, bool DYN, bool STK>
-__device__ __forceinline__ void ts_decode_group(const TsView& v, const uint16_t* ent, int n, double* E, int range_guard,
-                                                uint8_t* stk) {
+__device__ __forceinline__ void ts_decode_group(const TsView& v, const unsigned char* vb, const uint32_t* gd, int n, double* E,
+                                                int range_guard, uint8_t* stk) {
     const int lane = threadIdx.x & 31;
-    const uint32_t* desc = reinterpret_cast<const uint32_t*>(v.blob + v.off_desc);
     for (int u = lane; u < 4 * n; u += 32) {
-        const uint32_t en = ent[u >> 2];
-        const int c = (int)(en & 511u), r0 = (u & 3) * 4;
-        const uint32_t d = desc[c];
-        const unsigned char* src = v.blob + v.off_val + ((d >> 4) & 0xFFFu) * 16u + (r0 << (3 - Q));
+        const unsigned char* src = vb + (u << (5 - Q));
         double w[4];
         if (Q == 0) {
             const double2 a = reinterpret_cast<const double2*>(src)[0], b = reinterpret_cast<const double2*>(src)[1];
@@ -334,18 +344,19 @@ __device__ __forceinline__ void ts_decode_group(const TsView& v, const uint16_t*
             w[0] = e4m3_lo(a); w[1] = e4m3_lo(a >> 8); w[2] = e4m3_lo(a >> 16); w[3] = e4m3_lo(a >> 24);
         }
         if (DYN) {
-            const int lv = (int)(reinterpret_cast<const uint8_t*>(v.win) + (d >> 16))[128];
+            const uint32_t g = gd[u >> 2];
+            const int lv = (int)(reinterpret_cast<const uint8_t*>(v.win) + (g & 0xFFFFu))[128];
             if (STK) {
                 if (lv == BYP) { w[0] = w[1] = w[2] = w[3] = 0.0; }
                 else {
-                    uint8_t* sp = stk + (v.col0 + c);
+                    uint8_t* sp = stk + (v.col0 + (int)(g >> 20));
                     unsigned mask = *sp;
                     const int cur = mask ? 31 - __clz(mask) : Q;
                     int e = max(lv, cur);
-                    if (range_guard) e = min(e, (int)((d >> 2) & 3u));
+                    if (range_guard) e = min(e, (int)((g >> 16) & 3u));
                     if (e > cur) {
                         mask |= 1u << e;
-                        if (r0 == 0) *sp = (uint8_t)mask;   // every unit of the column computes the same mask
+                        if ((u & 3) == 0) *sp = (uint8_t)mask;   // every unit of the column computes the same mask
                     }
 #pragma unroll
                     for (int L = Q + 1; L <= 3; ++L)
@@ -358,7 +369,7 @@ __device__ __forceinline__ void ts_decode_group(const TsView& v, const uint16_t*
                 if (lv == BYP) { w[0] = w[1] = w[2] = w[3] = 0.0; }
                 else {
                     int e = lv;
-                    if (range_guard) e = min(e, (int)((d >> 2) & 3u));
+                    if (range_guard) e = min(e, (int)((g >> 16) & 3u));
                     if (e != Q) {
 #pragma unroll
                         for (int k = 0; k < 4; ++k) w[k] = round_to(w[k], e);
@@ -366,60 +377,105 @@ __device__ __forceinline__ void ts_decode_group(const TsView& v, const uint16_t*
                 }
             }
         }
-        double2* ea = reinterpret_cast<double2*>(E + (en >> 9) * 16 + r0);
-        ea[0] = make_double2(w[0], w[1]);
-        ea[1] = make_double2(w[2], w[3]);
+        // the two 16-byte halves in a lane-rotated order: conflict-free shared stores
+        double2* ea = reinterpret_cast<double2*>(E + u * 4);
+        if ((u >> 2) & 1) {
+            ea[1] = make_double2(w[2], w[3]);
+            ea[0] = make_double2(w[0], w[1]);
+        } else {
+            ea[0] = make_double2(w[0], w[1]);
+            ea[1] = make_double2(w[2], w[3]);
+        }
     }
 }
 
-// one tile row of this half-warp, N = the warp's widest row: columns beyond W read the next
-// descriptors (or the zero padding) and contribute fma(0, x, acc) == acc exactly (acc is never -0,
-// x is finite), so both half-warps run the same instruction stream.  Per column: descriptor and
-// local-column byte offset (LDS, immediate offsets), x from the window, the decoded value from
-// the warp's buffer (consecutive slots per row), one fma in ascending column order.
+// One tile row of this half-warp, N = the warp's widest row: columns beyond W read the next
+// descriptors (or the padding ones) and contribute fma(0, x, acc) == acc exactly (acc is never -0,
+// x is finite), so both half-warps run the same instruction stream.  Per column: the descriptor
+// (LDS, immediate offset), x of the lane's diagonal from the window, the decoded value from the
+// warp's buffer, one fma in ascending column order.
+struct TsRowCtx {
+    const uint32_t* desc;
+    const unsigned char* xw;        // slot's window guard + lane * 8
+    const double* el;               // warp's decode buffer + lane
+};
 template <int N>
-__device__ __forceinline__ double ts_row(const TsView& v, const double* Er, int a, int W, int lane) {
-    const uint32_t* desc = reinterpret_cast<const uint32_t*>(v.blob + v.off_desc) + a;
-    const uint8_t* lcb = v.blob + v.off_lc + a * 16 + lane;
-    const unsigned char* win = reinterpret_cast<const unsigned char*>(v.win);
+__device__ __forceinline__ double ts_row(const TsRowCtx& r, int a, int W) {
     double ev[N], xv[N];
 #pragma unroll
     for (int q = 0; q < N; ++q) {
-        const uint32_t d = desc[q];
-        ev[q] = q < W ? Er[q * 16] : 0.0;
-        xv[q] = *reinterpret_cast<const double*>(win + (d >> 16) + lcb[q * 16]);
+        const uint32_t d = r.desc[a + q];
+        ev[q] = q < W ? r.el[(d >> 16) * 16] : 0.0;
+        xv[q] = *reinterpret_cast<const double*>(r.xw + (d & 0xFFFFu));
     }
     double acc = 0.0;
 #pragma unroll
     for (int q = 0; q < N; ++q) acc = __fma_rn(ev[q], xv[q], acc);
     return acc;
 }
-// rows wider than 12 slice columns: plain loop over the columns in order (the chain is exact)
-__device__ __forceinline__ double ts_row_long(const TsView& v, const double* Er, int a, int W, int lane) {
-    const uint32_t* desc = reinterpret_cast<const uint32_t*>(v.blob + v.off_desc) + a;
-    const uint8_t* lcb = v.blob + v.off_lc + a * 16 + lane;
-    const unsigned char* win = reinterpret_cast<const unsigned char*>(v.win);
-    double r = 0.0;
-    for (int q = 0; q < W; ++q)
-        r = __fma_rn(Er[q * 16], *reinterpret_cast<const double*>(win + (desc[q] >> 16) + lcb[q * 16]), r);
-    return r;
+__device__ __forceinline__ double ts_row_long(const TsRowCtx& r, int a, int W) {
+    double acc = 0.0;
+    for (int q = 0; q < W; ++q) {
+        const uint32_t d = r.desc[a + q];
+        acc = __fma_rn(r.el[(d >> 16) * 16], *reinterpret_cast<const double*>(r.xw + (d & 0xFFFFu)), acc);
+    }
+    return acc;
 }
-__device__ __forceinline__ double ts_row_any(const TsView& v, const double* Er, int a, int W, int Wmax, int lane) {
+__device__ __forceinline__ double ts_row_any(const TsRowCtx& r, int a, int W, int Wmax) {
     switch (Wmax) {
     case 0: return 0.0;
-    case 1: return ts_row<1>(v, Er, a, W, lane);
-    case 2: return ts_row<2>(v, Er, a, W, lane);
-    case 3: return ts_row<3>(v, Er, a, W, lane);
-    case 4: return ts_row<4>(v, Er, a, W, lane);
-    case 5: return ts_row<5>(v, Er, a, W, lane);
-    case 6: return ts_row<6>(v, Er, a, W, lane);
-    case 7: return ts_row<7>(v, Er, a, W, lane);
-    case 8: return ts_row<8>(v, Er, a, W, lane);
-    case 9: return ts_row<9>(v, Er, a, W, lane);
-    case 10: return ts_row<10>(v, Er, a, W, lane);
-    case 11: return ts_row<11>(v, Er, a, W, lane);
-    case 12: return ts_row<12>(v, Er, a, W, lane);
-    default: return ts_row_long(v, Er, a, W, lane);
+    case 1: return ts_row<1>(r, a, W);
+    case 2: return ts_row<2>(r, a, W);
+    case 3: return ts_row<3>(r, a, W);
+    case 4: return ts_row<4>(r, a, W);
+    case 5: return ts_row<5>(r, a, W);
+    case 6: return ts_row<6>(r, a, W);
+    case 7: return ts_row<7>(r, a, W);
+    case 8: return ts_row<8>(r, a, W);
+    case 9: return ts_row<9>(r, a, W);
+    case 10: return ts_row<10>(r, a, W);
+    case 11: return ts_row<11>(r, a, W);
+    case 12: return ts_row<12>(r, a, W);
+    default: return ts_row_long(r, a, W);
+    }
+}
+// two tile rows of this half-warp at once (independent fma chains: ILP 2)
+template <int N>
+__device__ __forceinline__ void ts_row2(const TsRowCtx& r, int a1, int W1, int a2, int W2, double& acc1, double& acc2) {
+    double e1[N], x1[N], e2[N], x2[N];
+#pragma unroll
+    for (int q = 0; q < N; ++q) {
+        const uint32_t d1 = r.desc[a1 + q], d2 = r.desc[a2 + q];
+        e1[q] = q < W1 ? r.el[(d1 >> 16) * 16] : 0.0;
+        e2[q] = q < W2 ? r.el[(d2 >> 16) * 16] : 0.0;
+        x1[q] = *reinterpret_cast<const double*>(r.xw + (d1 & 0xFFFFu));
+        x2[q] = *reinterpret_cast<const double*>(r.xw + (d2 & 0xFFFFu));
+    }
+    double s1 = 0.0, s2 = 0.0;
+#pragma unroll
+    for (int q = 0; q < N; ++q) {
+        s1 = __fma_rn(e1[q], x1[q], s1);
+        s2 = __fma_rn(e2[q], x2[q], s2);
+    }
+    acc1 = s1;
+    acc2 = s2;
+}
+__device__ __forceinline__ void ts_row2_any(const TsRowCtx& r, int a1, int W1, int a2, int W2, int Wmax, double& acc1, double& acc2) {
+    switch (Wmax) {
+    case 0: acc1 = acc2 = 0.0; return;
+    case 1: ts_row2<1>(r, a1, W1, a2, W2, acc1, acc2); return;
+    case 2: ts_row2<2>(r, a1, W1, a2, W2, acc1, acc2); return;
+    case 3: ts_row2<3>(r, a1, W1, a2, W2, acc1, acc2); return;
+    case 4: ts_row2<4>(r, a1, W1, a2, W2, acc1, acc2); return;
+    case 5: ts_row2<5>(r, a1, W1, a2, W2, acc1, acc2); return;
+    case 6: ts_row2<6>(r, a1, W1, a2, W2, acc1, acc2); return;
+    case 7: ts_row2<7>(r, a1, W1, a2, W2, acc1, acc2); return;
+    case 8: ts_row2<8>(r, a1, W1, a2, W2, acc1, acc2); return;
+    case 9: ts_row2<9>(r, a1, W1, a2, W2, acc1, acc2); return;
+    default:
+        acc1 = ts_row_long(r, a1, W1);
+        acc2 = ts_row_long(r, a2, W2);
+        return;
     }
 }
 
@@ -427,41 +483,56 @@ __device__ __forceinline__ double ts_row_any(const TsView& v, const double* Er, 
 // own_mode: 0 none; 1 the SpMV input at the row (from the window when the stage's own segments
 // are staged); 2 the normal vector `ownv`.
 template <bool DYN, bool STK, class Emit>
-__device__ __forceinline__ void ts_consume(const TsView& v, int64_t tr0c, const double* pv, int range_guard, int own_mode,
-                                           const double* ownv, int64_t n, uint8_t* stk, int dbg, double* E, Emit& emit) {
+__device__ __forceinline__ void ts_consume(const TsView& v, const double* pv, int range_guard, int own_mode, const double* ownv,
+                                           int64_t n, uint8_t* stk, double* E, Emit& emit) {
     const int t = threadIdx.x, H = blockDim.x >> 4, h = t >> 4, lane = t & 15, w = t >> 5;
-    if (dbg >= 1) return;
     {
-        const uint32_t cnt = reinterpret_cast<const uint32_t*>(v.blob + v.off_wl)[w];
-        const int NW = blockDim.x >> 5;
-        const uint16_t* ent = reinterpret_cast<const uint16_t*>(v.blob + v.off_ent) +
-                              reinterpret_cast<const uint16_t*>(v.blob + v.off_wl + ts_r16(NW * 4))[w];
-        const int n0 = cnt & 0xFF, n1 = (cnt >> 8) & 0xFF, n2 = (cnt >> 16) & 0xFF, n3 = cnt >> 24;
-        ts_decode_group<0, DYN, STK>(v, ent, n0, E, range_guard, stk);
-        ts_decode_group<1, DYN, STK>(v, ent + n0, n1, E, range_guard, stk);
-        ts_decode_group<2, DYN, STK>(v, ent + n0 + n1, n2, E, range_guard, stk);
-        ts_decode_group<3, DYN, STK>(v, ent + n0 + n1 + n2, n3, E, range_guard, stk);
+        const uint4 wl = reinterpret_cast<const uint4*>(v.blob + v.off_wl)[w];
+        const int n0 = wl.x & 0xFF, n1 = (wl.x >> 8) & 0xFF, n2 = (wl.x >> 16) & 0xFF, n3 = wl.x >> 24;
+        const unsigned char* vb = v.blob + v.off_val + wl.y;
+        const uint32_t* gd = reinterpret_cast<const uint32_t*>(v.blob + v.off_gd) + wl.z;
+        ts_decode_group<0, DYN, STK>(v, vb, gd, n0, E, range_guard, stk);
+        vb += n0 * 128; gd += n0;
+        ts_decode_group<1, DYN, STK>(v, vb, gd, n1, E + n0 * 16, range_guard, stk);
+        vb += n1 * 64; gd += n1;
+        ts_decode_group<2, DYN, STK>(v, vb, gd, n2, E + (n0 + n1) * 16, range_guard, stk);
+        vb += n2 * 32; gd += n2;
+        ts_decode_group<3, DYN, STK>(v, vb, gd, n3, E + (n0 + n1 + n2) * 16, range_guard, stk);
     }
     __syncwarp();
     const int16_t* cs = reinterpret_cast<const int16_t*>(v.blob + TS_HDR);
-    const int rel = v.S0 - (int)tr0c;
-    const int off0 = (H & (H - 1)) == 0 ? (rel & (H - 1)) : rel % H;
-    const int first = h >= off0 ? h - off0 : h - off0 + H;
-    // both half-warps of the warp run the same iterations (their row or nothing)
-    for (int k = first;; k += H) {
-        const bool mine = v.S0 + k < v.S1;
-        if (!__any_sync(0xffffffffu, mine)) break;
-        const int a = mine ? cs[k] : 0, W = mine ? cs[k + 1] - a : 0;
-        const int Wmax = max(W, __shfl_xor_sync(0xffffffffu, W, 16));
-        const double* Er = E + (mine ? (int)v.blob[v.off_eb + k] : 0) * 16 + lane;
-        const double acc = ts_row_any(v, Er, a, W, Wmax, lane);
-        if (mine) {
-            const int TR = v.S0 + k;
-            double ov = 0.0;
+    TsRowCtx rc;
+    rc.desc = reinterpret_cast<const uint32_t*>(v.blob + v.off_desc);
+    rc.xw = reinterpret_cast<const unsigned char*>(v.win) - TS_GUARD + lane * 8;
+    rc.el = E + lane;
+    auto emit_row = [&](int k, double acc) {
+        const int TR = v.S0 + k;
+        double ov = 0.0;
+        if (own_mode == 1) ov = v.own_w >= 0 ? v.win[(v.own_w + k) * PVS + lane] : pv[(int64_t)TR * PVS + lane];
+        else if (own_mode == 2) {
             const int64_t i = (int64_t)TR * 16 + lane;
-            if (own_mode == 1) ov = v.own_w >= 0 ? v.win[(v.own_w + k) * PVS + lane] : pv[(int64_t)TR * PVS + lane];
-            else if (own_mode == 2 && i < n) ov = ownv[i];
-            emit((int64_t)TR, lane, acc, ov);
+            if (i < n) ov = ownv[i];
+        }
+        emit((int64_t)TR, lane, acc, ov);
+    };
+    // rows k and k + H of this half-warp together (two chains); both half-warps of the warp run the
+    // same iterations (their rows or nothing).  off0 = (S0 - tr0c) mod H (conversion).
+    const int nrow = v.S1 - v.S0;
+    for (int k = h >= v.off0 ? h - v.off0 : h - v.off0 + H;; k += 2 * H) {
+        const bool m1 = k < nrow, m2 = k + H < nrow;
+        if (!__any_sync(0xffffffffu, m1)) break;
+        const int a1 = m1 ? cs[k] : 0, W1 = m1 ? cs[k + 1] - a1 : 0;
+        const int a2 = m2 ? cs[k + H] : 0, W2 = m2 ? cs[k + H + 1] - a2 : 0;
+        int Wm = max(W1, W2);
+        Wm = max(Wm, __shfl_xor_sync(0xffffffffu, Wm, 16));
+        if (__any_sync(0xffffffffu, m2)) {
+            double acc1, acc2;
+            ts_row2_any(rc, a1, W1, a2, W2, Wm, acc1, acc2);
+            if (m1) emit_row(k, acc1);
+            if (m2) emit_row(k + H, acc2);
+        } else {
+            const double acc1 = ts_row_any(rc, a1, W1, Wm);
+            if (m1) emit_row(k, acc1);
         }
     }
     __syncwarp();
@@ -477,9 +548,9 @@ __device__ __forceinline__ void spmv_ts(const Mat& A, int64_t tr0c, const double
     const int32_t s_begin = A.stg_ptr[blockIdx.x], ns = A.stg_ptr[blockIdx.x + 1] - s_begin;
     const uint32_t* recs = reinterpret_cast<const uint32_t*>(A.stg + s_begin);
     const int NST = sm.nst;
-    double* E = sm.ebuf + (size_t)w * sm.ecap * 16;
+    double* E = sm.ebuf + (size_t)w * sm.ecap * 16;     // decode buffer: ecap columns x 16 doubles
     __syncthreads();                          // ring counters / previous phase's smem users
-    if (ns == 0 || A.dbg == 4) return;
+    if (ns == 0) return;
     unsigned long long pol = 0;
     if (w == 0) {
         pol = policy_evict_first();
@@ -490,10 +561,10 @@ __device__ __forceinline__ void spmv_ts(const Mat& A, int64_t tr0c, const double
         // matrices, e.g. C1); only the x windows are re-staged
         const unsigned rc = (unsigned)sm.ctr[1];
         if (w == 0)
-            for (int k = 0; k < ns; ++k) ts_issue(A.blob, recs[k * 32 + lane], sm.slot(k), sm.blob_cap, sm.full + k, pv, rc == 0, pol, A.dbg);
+            for (int k = 0; k < ns; ++k) ts_issue(A.blob, recs[k * 32 + lane], sm.slot(k), sm.blob_cap, sm.full + k, pv, rc == 0, pol);
         for (int k = 0; k < ns; ++k) {
             mbar_wait(sm.full + k, rc & 1u);
-            ts_consume<DYN, STK>(ts_view(sm.slot(k), sm.blob_cap), tr0c, pv, range_guard, own_mode, ownv, A.n_rows, A.stk, A.dbg, E, emit);
+            ts_consume<DYN, STK>(ts_view(sm.slot(k), sm.blob_cap), pv, range_guard, own_mode, ownv, A.n_rows, A.stk, E, emit);
         }
         __syncthreads();
         if (t == 0) sm.ctr[1] = rc + 1;
@@ -511,7 +582,7 @@ __device__ __forceinline__ void spmv_ts(const Mat& A, int64_t tr0c, const double
             // the slot's previous use (previous SpMV) finished before the caller's barrier; its
             // "empty" phase completed: wait on it to keep the parity in step
             if (u0 + k >= (unsigned)NST) mbar_wait(sm.empty + isl, iph ^ 1u);
-            ts_issue(A.blob, recs[k * 32 + lane], sm.slot(isl), sm.blob_cap, sm.full + isl, pv, true, pol, A.dbg);
+            ts_issue(A.blob, recs[k * 32 + lane], sm.slot(isl), sm.blob_cap, sm.full + isl, pv, true, pol);
             if (++isl == NST) { isl = 0; iph ^= 1u; }
         }
 #pragma unroll
@@ -519,11 +590,11 @@ __device__ __forceinline__ void spmv_ts(const Mat& A, int64_t tr0c, const double
     }
     for (int k = 0; k < ns; ++k) {
         mbar_wait(sm.full + sl, ph);
-        ts_consume<DYN, STK>(ts_view(sm.slot(sl), sm.blob_cap), tr0c, pv, range_guard, own_mode, ownv, A.n_rows, A.stk, A.dbg, E, emit);
+        ts_consume<DYN, STK>(ts_view(sm.slot(sl), sm.blob_cap), pv, range_guard, own_mode, ownv, A.n_rows, A.stk, E, emit);
         if (lane == 0) mbar_arrive(sm.empty + sl);
         if (w == 0 && k + NST < ns) {
             mbar_wait(sm.empty + sl, ph);         // every warp is done with the slot
-            ts_issue(A.blob, pre[0], sm.slot(sl), sm.blob_cap, sm.full + sl, pv, true, pol, A.dbg);
+            ts_issue(A.blob, pre[0], sm.slot(sl), sm.blob_cap, sm.full + sl, pv, true, pol);
 #pragma unroll
             for (int j = 0; j + 1 < TS_PF; ++j) pre[j] = pre[j + 1];
             pre[TS_PF - 1] = k + NST + TS_PF < ns ? recs[(k + NST + TS_PF) * 32 + lane] : 0u;

@@ -35,8 +35,8 @@ __global__ void pack_pv_kernel(const double* __restrict__ x, int64_t n, const ui
 }
 
 // mf_spmv: the same staged SpMV as the solver, one block per CTA of the launch plan
-template <bool DYN, bool COUNT>
-__global__ void __launch_bounds__(1024) spmv_kernel(Mat A, const int32_t* __restrict__ plan_tr, const double* pv,
+template <bool DYN, bool COUNT, int MAXT>
+__global__ void __launch_bounds__(MAXT, 1) spmv_kernel(Mat A, const int32_t* __restrict__ plan_tr, const double* pv,
                                                     double* __restrict__ y, int range_guard, unsigned long long* counts,
                                                     int nst, int slot_bytes, int blob_cap, int ecap) {
     extern __shared__ __align__(128) unsigned char smem_raw[];
@@ -139,7 +139,7 @@ void* pick_kernel(int maxt, bool bicg, bool dyn, bool count, bool sticky, bool p
 Mat mat_view(const TileMatrix& A) {
     return Mat{A.n_rows, A.n_cols, A.ntr, A.tr_slot, A.TileRowPtr, A.tile_info, A.sidx, A.blob,
                reinterpret_cast<const mfk::TsStage*>(A.stg), A.stg_ptr, A.TileNnz, A.ts, (int)A.max_w,
-               A.plane64, A.plane32, A.plane16, A.plane8, nullptr, getenv("MF_SPMV_DBG") ? atoi(getenv("MF_SPMV_DBG")) : 0};
+               A.plane64, A.plane32, A.plane16, A.plane8, nullptr};
 }
 
 // Ring depth of the TMA pipeline for a shared-memory budget (bytes available to the ring)
@@ -201,13 +201,36 @@ mf_status run_spmv(const TileMatrix& A, const double* x, double* y, const uint8_
     const int nst = std::max(1, ring_depth(A, (int64_t)smem_optin - 128 - 256 - (int64_t)mfk::TS_CTRL_BYTES - ebytes));
     const size_t smem = 128 + mfk::spmv_smem_bytes(A.ts, nst, A.slot_bytes, A.ecap, A.B / 32);
     void* fn;
-    if (level) fn = counts_host ? (void*)spmv_kernel<true, true> : (void*)spmv_kernel<true, false>;
-    else fn = counts_host ? (void*)spmv_kernel<false, true> : (void*)spmv_kernel<false, false>;
+    if (A.B > 512) {
+        if (level) fn = counts_host ? (void*)spmv_kernel<true, true, 1024> : (void*)spmv_kernel<true, false, 1024>;
+        else fn = counts_host ? (void*)spmv_kernel<false, true, 1024> : (void*)spmv_kernel<false, false, 1024>;
+    } else {
+        if (level) fn = counts_host ? (void*)spmv_kernel<true, true, 512> : (void*)spmv_kernel<true, false, 512>;
+        else fn = counts_host ? (void*)spmv_kernel<false, true, 512> : (void*)spmv_kernel<false, false, 512>;
+    }
     MF_CUDA(cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
     const int32_t* plan = A.plan_tr;
     int slot_bytes = A.slot_bytes, blob_cap = A.blob_cap, nst_a = nst, ecap = A.ecap;
     void* args[] = {&M, (void*)&plan, (void*)&pv, (void*)&y, &range_guard, &dcnt, &nst_a, &slot_bytes, &blob_cap, &ecap};
-    MF_CUDA(cudaLaunchKernel(fn, dim3(A.G), dim3(A.B), args, smem, s));
+    // diagnostics: MF_SPMV_REPS = launches of the SpMV kernel alone (timed with CUDA events,
+    // reported on stderr with the warp-1 breakdown when MF_PHASE_DUMP is set)
+    const int reps = getenv("MF_SPMV_REPS") ? std::max(1, atoi(getenv("MF_SPMV_REPS"))) : 1;
+    Events ev;
+    if (reps > 1) {
+        MF_CUDA(cudaEventCreate(&ev.e0));
+        MF_CUDA(cudaEventCreate(&ev.e1));
+        MF_CUDA(cudaLaunchKernel(fn, dim3(A.G), dim3(A.B), args, smem, s));   // warm-up
+        MF_CUDA(cudaEventRecord(ev.e0, s));
+    }
+    for (int k = 0; k < reps; ++k) MF_CUDA(cudaLaunchKernel(fn, dim3(A.G), dim3(A.B), args, smem, s));
+    if (reps > 1) {
+        MF_CUDA(cudaEventRecord(ev.e1, s));
+        MF_CUDA(cudaEventSynchronize(ev.e1));
+        float ms = 0;
+        MF_CUDA(cudaEventElapsedTime(&ms, ev.e0, ev.e1));
+        fprintf(stderr, "mf_spmv kernel: %.2f us per launch (%d launches, ring %d x %d B, decode %d cols/warp)\n",
+                ms * 1e3 / reps, reps, nst, A.slot_bytes, A.ecap);
+    }
     if (counts_host) {
         unsigned long long h[10];
         MF_CUDA(cudaMemcpyAsync(h, dcnt, sizeof(h), cudaMemcpyDeviceToHost, s));
