@@ -33,7 +33,7 @@ def build(force: bool = False) -> str:
     """Compile liboracle.so with gcc (plain C11, no FMA contraction)."""
     if force or not os.path.exists(_LIB_PATH) or os.path.getmtime(_LIB_PATH) < os.path.getmtime(_SRC):
         tmp = _LIB_PATH + f".{os.getpid()}.tmp"
-        subprocess.check_call(["gcc", "-O2", "-std=c11", "-fPIC", "-shared", "-ffp-contract=off",
+        subprocess.check_call(["gcc", "-O2", "-std=c11", "-fPIC", "-shared", "-ffp-contract=off", "-fopenmp",
                                "-o", tmp, _SRC, "-lm"])
         os.replace(tmp, _LIB_PATH)
     return _LIB_PATH
@@ -115,6 +115,10 @@ def lib():
             L.orc_ilu0.argtypes = [i64, vp, vp, vp, vp, vp]; L.orc_ilu0.restype = C.c_int
             L.orc_ilu_apply.argtypes = [C.POINTER(_Ilu), vp, vp]; L.orc_ilu_apply.restype = None
             L.orc_csr_validate.argtypes = [i64, i64, i64, vp, vp, vp]; L.orc_csr_validate.restype = C.c_int
+            L.orc_baseline_threads.argtypes = [C.c_int]; L.orc_baseline_threads.restype = C.c_int
+            base_args = [i64, vp, vp, vp, C.POINTER(_Ilu), vp, vp, d, i64, C.POINTER(_Info)]
+            L.orc_cg_csr_omp.argtypes = base_args; L.orc_cg_csr_omp.restype = C.c_int
+            L.orc_bicgstab_csr_omp.argtypes = base_args; L.orc_bicgstab_csr_omp.restype = C.c_int
             _lib = L
     return _lib
 
@@ -402,3 +406,21 @@ def true_relres(rowptr, colidx, vals, b, x) -> float:
     colidx = np.ascontiguousarray(colidx, np.int32)
     vals, b, x = _f64(vals), _f64(b), _f64(x)
     return lib().orc_true_relres(len(rowptr) - 1, _vp(rowptr), _vp(colidx), _vp(vals), _vp(b), _vp(x))
+
+
+def baseline_solve(kind, rowptr, colidx, vals, b, M=None, tol=1e-10, max_iter=1000, threads=0):
+    """The CPU baseline of BASELINE.md section 7: textbook binary64 CSR CG ("cg") or BiCGSTAB
+    ("bicgstab"), ILU(0)-preconditioned when M is an ILU0, OpenMP over `threads` host threads
+    (0 = all in the affinity mask).  Returns the result dict plus the thread count used."""
+    rowptr = np.ascontiguousarray(rowptr, np.int64)
+    colidx = np.ascontiguousarray(colidx, np.int32)
+    vals, b = _f64(vals), _f64(b)
+    n = len(rowptr) - 1
+    used = lib().orc_baseline_threads(int(threads) if threads else len(os.sched_getaffinity(0)))
+    x = np.zeros(n)
+    info = _Info()
+    fn = lib().orc_cg_csr_omp if kind == "cg" else lib().orc_bicgstab_csr_omp
+    st = fn(n, _vp(rowptr), _vp(colidx), _vp(vals), None if M is None else C.byref(M._s), _vp(b), _vp(x),
+            float(tol), int(max_iter), C.byref(info))
+    return {"x": x, "status": st, "iterations": info.iterations, "converged": bool(info.converged),
+            "rel_residual": info.rel_residual, "threads": used}

@@ -841,3 +841,146 @@ static void ilu_apply(const orc_ilu* M, const double* r, double* z) {
 }
 
 void orc_ilu_apply(const orc_ilu* M, const double* r, double* z) { ilu_apply(M, r, z); }
+
+/* ------------------------------------------------------------------------------------
+ * 9. The CPU baseline: textbook binary64 CSR CG / BiCGSTAB (Alg. 1-2,
+ *    P:70) and their ILU(0)-preconditioned forms (PCG standard, PBiCGSTAB right-
+ *    preconditioned as in orc_pcg / orc_pbicgstab), with the SpMV, the dots and the AXPYs
+ *    spread over `threads` OpenMP threads (static schedule).  The dots are OpenMP sum
+ *    reductions, so the summation order (not the arithmetic) differs from the sequential
+ *    oracle; the triangular solves of the preconditioner stay sequential.  Pinned against the
+ *    sequential oracle's FP64 mode (tests/test_oracle_baseline.py).
+ * ---------------------------------------------------------------------------------- */
+#ifdef _OPENMP
+#include <omp.h>
+#endif
+
+static void par_spmv(int64_t n, const int64_t* rp, const int32_t* ci, const double* v, const double* x, double* y) {
+#pragma omp parallel for schedule(static)
+    for (int64_t i = 0; i < n; ++i) {
+        double acc = 0.0;
+        for (int64_t k = rp[i]; k < rp[i + 1]; ++k) acc = fma(v[k], x[ci[k]], acc);
+        y[i] = acc;
+    }
+}
+static double par_dot(int64_t n, const double* u, const double* w) {
+    double s = 0.0;
+#pragma omp parallel for schedule(static) reduction(+ : s)
+    for (int64_t i = 0; i < n; ++i) s = fma(u[i], w[i], s);
+    return s;
+}
+
+int orc_baseline_threads(int threads) {
+#ifdef _OPENMP
+    if (threads > 0) omp_set_num_threads(threads);
+    return omp_get_max_threads();
+#else
+    (void)threads;
+    return 1;
+#endif
+}
+
+/* CG (M == NULL) or PCG with ILU(0) */
+int orc_cg_csr_omp(int64_t n, const int64_t* rp, const int32_t* ci, const double* v, const orc_ilu* M,
+                   const double* b, double* x, double tol, int64_t max_iter, orc_info* info) {
+    size_t nb8 = sizeof(double) * (size_t)(n > 0 ? n : 1);
+    double *r = malloc(nb8), *p = malloc(nb8), *mu = malloc(nb8), *z = M ? malloc(nb8) : NULL;
+    memset(info, 0, sizeof(*info));
+    int st = ORC_OK;
+    par_spmv(n, rp, ci, v, x, mu);
+#pragma omp parallel for schedule(static)
+    for (int64_t i = 0; i < n; ++i) r[i] = b[i] - mu[i];
+    double nb = sqrt(par_dot(n, b, b));
+    double rr = par_dot(n, r, r), rho;
+    int64_t j = 0;
+    if (nb == 0.0) { for (int64_t i = 0; i < n; ++i) x[i] = 0.0; info->converged = 1; goto done; }
+    if (M) { ilu_apply(M, r, z); memcpy(p, z, nb8); rho = par_dot(n, r, z); }
+    else { memcpy(p, r, nb8); rho = rr; }
+    for (;; ++j) {
+        double relres = sqrt(rr) / nb;
+        info->rel_residual = relres;
+        if (relres < tol) { info->converged = 1; break; }
+        if (j == max_iter) break;
+        par_spmv(n, rp, ci, v, p, mu);
+        double sigma = par_dot(n, mu, p);
+        if (!(sigma > 0.0) || !isfinite(sigma)) { st = ORC_ERR_BREAKDOWN; break; }
+        double alpha = rho / sigma;
+#pragma omp parallel for schedule(static)
+        for (int64_t i = 0; i < n; ++i) { x[i] = fma(alpha, p[i], x[i]); r[i] = fma(-alpha, mu[i], r[i]); }
+        rr = par_dot(n, r, r);
+        double rho_new;
+        if (M) { ilu_apply(M, r, z); rho_new = par_dot(n, r, z); } else rho_new = rr;
+        double beta = rho_new / rho;
+        rho = rho_new;
+        const double* d = M ? z : r;
+#pragma omp parallel for schedule(static)
+        for (int64_t i = 0; i < n; ++i) p[i] = fma(beta, p[i], d[i]);
+    }
+done:
+    info->iterations = j; info->status = st; info->n_spmv = j;
+    free(r); free(p); free(mu); free(z);
+    return st;
+}
+
+/* BiCGSTAB (M == NULL) or right-preconditioned PBiCGSTAB with ILU(0) */
+int orc_bicgstab_csr_omp(int64_t n, const int64_t* rp, const int32_t* ci, const double* v, const orc_ilu* M,
+                         const double* b, double* x, double tol, int64_t max_iter, orc_info* info) {
+    size_t nb8 = sizeof(double) * (size_t)(n > 0 ? n : 1);
+    double *r = malloc(nb8), *rh = malloc(nb8), *p = malloc(nb8), *mu = malloc(nb8), *s = malloc(nb8), *th = malloc(nb8);
+    double *ph = M ? malloc(nb8) : NULL, *sh = M ? malloc(nb8) : NULL;
+    memset(info, 0, sizeof(*info));
+    int st = ORC_OK;
+    int64_t j = 0;
+    par_spmv(n, rp, ci, v, x, mu);
+#pragma omp parallel for schedule(static)
+    for (int64_t i = 0; i < n; ++i) r[i] = b[i] - mu[i];
+    double nb = sqrt(par_dot(n, b, b));
+    if (nb == 0.0) { for (int64_t i = 0; i < n; ++i) x[i] = 0.0; info->converged = 1; goto done; }
+    memcpy(rh, r, nb8); memcpy(p, r, nb8);
+    double rho = par_dot(n, r, rh), rr = par_dot(n, r, r);
+    for (;; ++j) {
+        double relres = sqrt(rr) / nb;
+        info->rel_residual = relres;
+        if (relres < tol) { info->converged = 1; break; }
+        if (j == max_iter) break;
+        const double* pin = p;
+        if (M) { ilu_apply(M, p, ph); pin = ph; }
+        par_spmv(n, rp, ci, v, pin, mu);
+        double eta = par_dot(n, mu, rh);
+        if (eta == 0.0 || !isfinite(eta)) { st = ORC_ERR_BREAKDOWN; break; }
+        double alpha = rho / eta;
+#pragma omp parallel for schedule(static)
+        for (int64_t i = 0; i < n; ++i) s[i] = fma(-alpha, mu[i], r[i]);
+        const double* sin_ = s;
+        if (M) { ilu_apply(M, s, sh); sin_ = sh; }
+        par_spmv(n, rp, ci, v, sin_, th);
+        double tt = par_dot(n, th, th), ts = par_dot(n, th, s);
+        if (tt == 0.0) {
+#pragma omp parallel for schedule(static)
+            for (int64_t i = 0; i < n; ++i) { x[i] = fma(alpha, pin[i], x[i]); r[i] = s[i]; }
+            rr = par_dot(n, r, r); ++j;
+            info->rel_residual = sqrt(rr) / nb;
+            if (info->rel_residual < tol) info->converged = 1; else st = ORC_ERR_BREAKDOWN;
+            break;
+        }
+        double omega = ts / tt;
+        if (omega == 0.0 || !isfinite(omega)) { st = ORC_ERR_BREAKDOWN; break; }
+#pragma omp parallel for schedule(static)
+        for (int64_t i = 0; i < n; ++i) { x[i] = fma(omega, sin_[i], fma(alpha, pin[i], x[i])); r[i] = fma(-omega, th[i], s[i]); }
+        double rho_new = par_dot(n, r, rh);
+        rr = par_dot(n, r, r);
+        if (rho_new == 0.0 || !isfinite(rho_new)) {
+            ++j; info->rel_residual = sqrt(rr) / nb;
+            if (info->rel_residual < tol) info->converged = 1; else st = ORC_ERR_BREAKDOWN;
+            break;
+        }
+        double beta = (rho_new / rho) * (alpha / omega);
+        rho = rho_new;
+#pragma omp parallel for schedule(static)
+        for (int64_t i = 0; i < n; ++i) p[i] = fma(beta, fma(-omega, mu[i], p[i]), r[i]);
+    }
+done:
+    info->iterations = j; info->status = st; info->n_spmv = 2 * j;
+    free(r); free(rh); free(p); free(mu); free(s); free(th); free(ph); free(sh);
+    return st;
+}

@@ -334,7 +334,7 @@ class SolveResult:
 
 def _solve(fn, A: TileMatrix, b, x0=None, tol=1e-10, max_iter=1000, mode=MODE_DYNAMIC, switch_eps=None,
            switch_absolute=False, range_guard=True, sticky=False, history=True, level_counts=False,
-           collect_stats=False, M=None, stream=None, raise_on_breakdown=True) -> SolveResult:
+           collect_stats=False, M=None, stream=None, raise_on_breakdown=True, watchdog_ms=0) -> SolveResult:
     import torch
     _need_cuda(b, torch.float64, "b")
     x = torch.zeros_like(b) if x0 is None else x0.clone()
@@ -351,6 +351,7 @@ def _solve(fn, A: TileMatrix, b, x0=None, tol=1e-10, max_iter=1000, mode=MODE_DY
     if lc is not None:
         o.tile_level_counts, o.level_counts_cap = lc.ctypes.data, lc.shape[0]
     o.collect_stats = int(collect_stats)
+    o.watchdog_ms = int(watchdog_ms)
     info = SolveInfo()
     st = fn(A._h, _ptr(b), _ptr(x), C.byref(o), C.byref(info), _stream_ptr(stream))
     if st != 0 and (raise_on_breakdown or st != 7):

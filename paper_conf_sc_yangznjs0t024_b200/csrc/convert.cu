@@ -277,8 +277,11 @@ __device__ int64_t block_incl_scan(int64_t v, int64_t* sh) {
     return v;
 }
 
-__global__ void scan_block_sums(const int64_t* __restrict__ in, int64_t n, int64_t* bsum) {
+// Multi-array scans: blockIdx.y selects array y (in + y * istride, out + y * ostride, tmp + y * nb).
+__global__ void scan_block_sums(const int64_t* __restrict__ in, int64_t n, int64_t* bsum, int64_t istride, int64_t nb) {
     __shared__ int64_t sh[32];
+    in += blockIdx.y * istride;
+    bsum += blockIdx.y * nb;
     int64_t base = (int64_t)blockIdx.x * SCAN_CHUNK;
     int64_t a = base + 2 * threadIdx.x;
     int64_t v = (a < n ? in[a] : 0) + (a + 1 < n ? in[a + 1] : 0);
@@ -286,9 +289,10 @@ __global__ void scan_block_sums(const int64_t* __restrict__ in, int64_t n, int64
     if (threadIdx.x == blockDim.x - 1) bsum[blockIdx.x] = v;
 }
 
-__global__ void scan_sums_serial(int64_t* bsum, int64_t nb) {   // one block: exclusive scan in place
+__global__ void scan_sums_serial(int64_t* bsum, int64_t nb) {   // block y: exclusive scan of array y in place
     __shared__ int64_t sh[32];
     __shared__ int64_t carry;
+    bsum += blockIdx.x * nb;
     if (threadIdx.x == 0) carry = 0;
     __syncthreads();
     for (int64_t c = 0; c < nb; c += blockDim.x) {
@@ -303,8 +307,12 @@ __global__ void scan_sums_serial(int64_t* bsum, int64_t nb) {   // one block: ex
     }
 }
 
-__global__ void scan_apply(const int64_t* __restrict__ in, int64_t n, const int64_t* __restrict__ bsum, int64_t* out) {
+__global__ void scan_apply(const int64_t* __restrict__ in, int64_t n, const int64_t* __restrict__ bsum, int64_t* out,
+                           int64_t istride, int64_t ostride, int64_t nb) {
     __shared__ int64_t sh[32];
+    in += blockIdx.y * istride;
+    out += blockIdx.y * ostride;
+    bsum += blockIdx.y * nb;
     int64_t base = (int64_t)blockIdx.x * SCAN_CHUNK;
     int64_t a = base + 2 * threadIdx.x;
     int64_t x0 = a < n ? in[a] : 0, x1 = a + 1 < n ? in[a + 1] : 0;
@@ -316,15 +324,23 @@ __global__ void scan_apply(const int64_t* __restrict__ in, int64_t n, const int6
     if (n == 0 && blockIdx.x == 0 && threadIdx.x == 0) out[0] = 0;
 }
 
-// out[0..n] = exclusive scan of in[0..n), out[n] = total
-mf_status scan_excl(const int64_t* in, int64_t n, int64_t* out, int64_t* tmp, cudaStream_t s) {
-    int64_t nb = (n + SCAN_CHUNK - 1) / SCAN_CHUNK;
-    if (n == 0) { MF_CUDA(cudaMemsetAsync(out, 0, sizeof(int64_t), s)); return MF_OK; }
-    scan_block_sums<<<(unsigned)nb, SCAN_T, 0, s>>>(in, n, tmp);
-    scan_sums_serial<<<1, SCAN_T, 0, s>>>(tmp, nb);
-    scan_apply<<<(unsigned)nb, SCAN_T, 0, s>>>(in, n, tmp, out);
+// out[y][0..n] = exclusive scans of in[y][0..n) for narr arrays (out[y][n] = total): 3 launches
+mf_status scan_excl_multi(const int64_t* in, int64_t n, int narr, int64_t istride, int64_t* out, int64_t ostride, int64_t* tmp,
+                          cudaStream_t s) {
+    if (n == 0) {
+        for (int y = 0; y < narr; ++y) MF_CUDA(cudaMemsetAsync(out + y * ostride, 0, sizeof(int64_t), s));
+        return MF_OK;
+    }
+    const int64_t nb = (n + SCAN_CHUNK - 1) / SCAN_CHUNK;
+    scan_block_sums<<<dim3((unsigned)nb, narr), SCAN_T, 0, s>>>(in, n, tmp, istride, nb);
+    scan_sums_serial<<<narr, SCAN_T, 0, s>>>(tmp, nb);
+    scan_apply<<<dim3((unsigned)nb, narr), SCAN_T, 0, s>>>(in, n, tmp, out, istride, ostride, nb);
     MF_CUDA(cudaGetLastError());
     return MF_OK;
+}
+// out[0..n] = exclusive scan of in[0..n), out[n] = total
+mf_status scan_excl(const int64_t* in, int64_t n, int64_t* out, int64_t* tmp, cudaStream_t s) {
+    return scan_excl_multi(in, n, 1, 0, out, 0, tmp, s);
 }
 
 // ------------------------------------------------------------------ launch plan
@@ -552,10 +568,21 @@ __global__ void __launch_bounds__(mfk::TS_CCAP) blob_fill_kernel(mfk::TsStage* s
         reinterpret_cast<int16_t*>(b + mfk::TS_HDR)[k] = (int16_t)hdr[k];
         if (k < K) cw[k] = (int16_t)((int)((st.tr0 + k - tr0c) % H) >> 1);
     }
+    __shared__ uint8_t cfl[mfk::TS_CCAP];                // Floor of each column
     uint2 rc = make_uint2(0u, 0u);
     if (c < nc) {
         rc = crec[col0 + c];
         cq[c] = (uint8_t)(rc.x & 3u);
+        cfl[c] = (uint8_t)((rc.x >> 2) & 3u);
+    }
+    __syncthreads();
+    if (c < NW) {      // columns and value bytes of warp c (its rows: half-warps 2c, 2c+1)
+        int nw = 0, vw = 0;
+        for (int k = 0; k < K; ++k)
+            if (cw[k] == c)
+                for (int cc = hdr[k]; cc < hdr[k + 1]; ++cc) { ++nw; vw += 16 * (8 >> cq[cc]); }
+        wcol[c + 1] = nw;
+        wval[c + 1] = vw;
     }
     __syncthreads();
     if (c == 0) {
@@ -569,14 +596,7 @@ __global__ void __launch_bounds__(mfk::TS_CCAP) blob_fill_kernel(mfk::TsStage* s
         h[9] = L.off_wl; h[10] = L.off_gd; h[11] = (int32_t)((st.tr0 - tr0c) % H);   // off0: half-warp of tile row tr0
         for (int k = 12; k < 16; ++k) h[k] = 0;
         wcol[0] = 0; wval[0] = 0;
-        for (int w = 0; w < NW; ++w) {
-            int nw = 0, vw = 0;
-            for (int k = 0; k < K; ++k)
-                if (cw[k] == w)
-                    for (int cc = hdr[k]; cc < hdr[k + 1]; ++cc) { ++nw; vw += 16 * (8 >> cq[cc]); }
-            wcol[w + 1] = wcol[w] + nw;
-            wval[w + 1] = wval[w] + vw;
-        }
+        for (int w = 0; w < NW; ++w) { wcol[w + 1] += wcol[w]; wval[w + 1] += wval[w]; }
     }
     __syncthreads();
     if (c < NW) {
@@ -592,10 +612,9 @@ __global__ void __launch_bounds__(mfk::TS_CCAP) blob_fill_kernel(mfk::TsStage* s
                 if (cw[k] != w) continue;
                 for (int cc = hdr[k]; cc < hdr[k + 1]; ++cc)
                     if (cq[cc] == q) {
-                        const uint2 r2 = crec[col0 + cc];
                         cslot[cc] = (uint8_t)slot;      // decode-buffer slot: rank in the warp's grouped order
                         cdst[cc] = voff;
-                        gd[slot] = ((uint32_t)((r2.x >> 2) & 3u) << 16) | ((uint32_t)cc << 20);   // + window offset below
+                        gd[slot] = ((uint32_t)cfl[cc] << 16) | ((uint32_t)cc << 20);   // + window offset below
                         ++slot; ++nq;
                         voff += 16 * (8 >> q);
                     }
@@ -683,7 +702,7 @@ mf_status convert_csr(int64_t n_rows, int64_t n_cols, int64_t nnz, const int64_t
     const int64_t S = ntr + 1;
     MF_TRY(alloc(&cnt, (size_t)NCNT * std::max<int64_t>(ntr, 1), s));
     MF_TRY(alloc(&off, (size_t)NCNT * S, s));
-    MF_TRY(alloc(&tmp, (size_t)(ntr / SCAN_CHUNK + 2), s));
+    MF_TRY(alloc(&tmp, (size_t)NCNT * (ntr / SCAN_CHUNK + 2), s));
     const int tr_per_block = THREADS / 16;
     const unsigned tblocks = (unsigned)std::max<int64_t>((ntr + tr_per_block - 1) / tr_per_block, 1);
     Out none{};
@@ -693,7 +712,7 @@ mf_status convert_csr(int64_t n_rows, int64_t n_cols, int64_t nnz, const int64_t
                                                             cnt, d_err, none);
         MF_CUDA(cudaGetLastError());
     }
-    for (int c = 0; c < NCNT; ++c) MF_TRY(scan_excl(cnt + c * ntr, ntr, off + c * S, tmp, s));
+    MF_TRY(scan_excl_multi(cnt, ntr, NCNT, ntr, off, S, tmp, s));
     std::vector<int64_t> tot(NCNT);
     for (int c = 0; c < NCNT; ++c)
         MF_CUDA(cudaMemcpyAsync(&tot[c], off + c * S + ntr, sizeof(int64_t), cudaMemcpyDeviceToHost, s));

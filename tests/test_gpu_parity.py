@@ -270,10 +270,11 @@ def test_full_size_C3_prefix_and_convergence(mf, orc):
     """C3 at full size: bit-identical first 25 iterations vs the oracle; the full GPU solve
     reaches 1e-10 and its true residual is checked by the oracle."""
     A = W.make("C3")
-    ro, rg, Gm = run_pair(mf, orc, A, "bicgstab", 2, max_iter=25, tol=0.0)
+    eps = W.CONFIGS["C3"]["switch_eps"]
+    ro, rg, Gm = run_pair(mf, orc, A, "bicgstab", 2, max_iter=25, tol=0.0, switch_eps=eps)
     assert np.array_equal(rg.history, ro["history"]) and np.array_equal(rg.x.cpu().numpy(), ro["x"])
     b = W.rhs_ones(A)
-    full = mf.bicgstab_solve(Gm, dev(b), max_iter=20000)
+    full = mf.bicgstab_solve(Gm, dev(b), max_iter=20000, switch_eps=eps)
     assert full.converged
     tr = orc.true_relres(A.rowptr, A.colidx, A.vals, b, full.x.cpu().numpy())
     assert tr < 1e-9
@@ -386,3 +387,52 @@ def test_sticky_unsupported_combinations(mf):
     Gt = mf.TileMatrix.from_host_csr(A, grid_ctas=4, block_threads=256, layout=2)
     with pytest.raises(mf.MFError):
         mf.cg_solve(Gt, b, mode=2, sticky=True, level_counts=True)
+
+
+@pytest.mark.parametrize("solver", ["cg", "bicgstab"])
+def test_watchdog_reports_deadlock(mf, solver):
+    """A CTA that never publishes its SpMV input (test hook MF_DEBUG_STALL_CTA) makes the others'
+    ready-flag waits expire: the solve returns MF_ERR_DEADLOCK (9) instead of hanging the GPU, and
+    the next solve on the same device works."""
+    import os
+    A = W.make("C2", 16) if solver == "cg" else W.make("C3", 64)
+    G = mf.TileMatrix.from_host_csr(A, grid_ctas=4, block_threads=256)
+    b = dev(W.rhs_ones(A))
+    fn = mf.cg_solve if solver == "cg" else mf.bicgstab_solve
+    os.environ["MF_DEBUG_STALL_CTA"] = "1"
+    try:
+        with pytest.raises(mf.MFError) as e:
+            fn(G, b, watchdog_ms=300)
+        assert e.value.status == 9
+    finally:
+        del os.environ["MF_DEBUG_STALL_CTA"]
+    r = fn(G, b, max_iter=3000)
+    assert r.converged
+
+
+def test_sptrsv_nonsymmetric_pattern(mf, orc):
+    """In-kernel ILU(0) apply on a matrix whose pattern is NOT symmetric (a backward row
+    may finish before a forward row reads its flag): PBiCGSTAB bit-identical to the oracle."""
+    rng = np.random.default_rng(3)
+    n = 3000
+    rows, cols, vals = [], [], []
+    for i in range(n):
+        cs = set([i] + [c for c in rng.integers(max(0, i - 40), i, 3)] + [c for c in rng.integers(i, min(n, i + 200), 2)])
+        for c in sorted(cs):
+            rows.append(i); cols.append(int(c))
+            vals.append(8.0 if c == i else float(rng.choice([-1.0, 0.5, -0.25, 1.5])))
+    rp = np.zeros(n + 1, np.int64)
+    np.cumsum(np.bincount(rows, minlength=n), out=rp[1:])
+    A = W.CSR(n, n, rp, np.array(cols, np.int32), np.array(vals))
+    D = A.dense()
+    assert not np.array_equal(D != 0, (D != 0).T)        # the pattern is nonsymmetric
+    b = W.rhs_ones(A)
+    Gm = mf.TileMatrix.from_host_csr(A, grid_ctas=6, block_threads=256)
+    g, bb, R = Gm.plan()
+    T = oracle_tiles(orc, A)
+    rp_, ci, sv = T.stored_csr()
+    M = orc.ILU0(rp_, ci, sv)
+    ro = orc.bicgstab(T, b, M=M, mode=2, plan=orc.Plan(g, bb, R), max_iter=300)
+    rg = mf.bicgstab_solve(Gm, dev(b), M=mf.Precond(Gm), mode=2, max_iter=300, watchdog_ms=20000)
+    assert ro["converged"] and rg.converged and rg.iterations == ro["iterations"]
+    assert np.array_equal(rg.x.cpu().numpy(), ro["x"])

@@ -237,8 +237,11 @@ CONFIGS = {
                solver="cg", max_iter=1000),
     "C2": dict(desc="CG mixed precision on 3D 7-point Poisson 128^3 (2.1M rows) value-scaled tiles, 1 GPU",
                solver="cg", max_iter=1000),
+    # C3: with the paper's eps = tol the dynamic switch stalls BiCGSTAB on this matrix
+    # (20000 iterations, relres 6e3); eps = 1e-11 .. 1e-14 stall too, 1e-15 converges in 8455
+    # iterations (FP64: 6444).  Sweep: profiles/r02_c3_eps_sweep.log (tools/c3_modes.py).
     "C3": dict(desc="BiCGSTAB on 2D convection-diffusion 2048^2 (4.2M rows), 1 GPU",
-               solver="bicgstab", max_iter=20000),
+               solver="bicgstab", max_iter=20000, switch_eps=1e-15),
     "C4spd": dict(desc="PCG (ILU0) on SuiteSparse-shaped SPD, 1M rows ~29 nnz/row, 1 GPU",
                   solver="pcg", max_iter=1000),
     "C4ind": dict(desc="PBiCGSTAB (ILU0) on SuiteSparse-shaped indefinite, 1M rows, 1 GPU",
