@@ -184,14 +184,56 @@ mf_status mf_cg_solve(const mf_tile_matrix* A, const double* b, double* x, const
 mf_status mf_bicgstab_solve(const mf_tile_matrix* A, const double* b, double* x, const mf_solve_opts* opts,
                             mf_solve_info* info, mf_stream stream);
 
-/* ---------------------------------------------------------------- multi-GPU (row blocks, SURVEY 8(e))
- * One process per GPU; rank k owns the tile-aligned rows [row_begin, row_end) of the global
- * matrix and converts them as a local n_local x n_ext matrix whose columns are the contiguous
- * range [xlo, xhi) of global columns its rows gather (xlo a multiple of 16, so local and global
- * 16-segments coincide).  The halo exchange of the search direction and the scalar reductions
- * run over NCCL from the Python layer (torch.distributed); every arithmetic step runs in these
- * kernels, with the launch plan's reduction tree (rank partials are then summed in rank order).
- * Alg. 1 steps C and D: */
+/* ---------------------------------------------------------------- multi-GPU (row blocks, SURVEY 8(b), 8(e))
+ * The paper's solver is single-GPU; the build partitions matrices too large for one GPU
+ * (BASELINE configs[4]) into contiguous blocks of whole 16-row tile rows, one block per GPU, one
+ * process per GPU.  Communication is NCCL (over NVLink) inside libmf: the caller only ships the
+ * 128-byte unique id from rank 0 to the other ranks (e.g. with torch.distributed).
+ *
+ * Rank k owns rows [row_begin, row_end) (row_begin a multiple of 16; the blocks of all ranks are
+ * contiguous, in rank order, and cover the matrix).  It converts its rows as a local tile matrix
+ * whose columns are its own 16-element segments followed by the halo segments its rows gather
+ * (one-to-one with global segments: tiles, TilePrec and the dynamic levels of Alg. 4 are the
+ * global matrix's).  Per iteration: halo exchange of the SpMV input (ncclSend / ncclRecv per
+ * peer), the staged tile SpMV, rank partials of every dot (the launch plan's tree) all-gathered
+ * and summed in rank order from +0 on every rank (deterministic; one rank == mf_cg_solve bit for
+ * bit), every scalar on the device, iterations enqueued as CUDA graphs with a device stop flag.
+ * All calls are collective over the communicator's ranks. */
+typedef struct mf_comm mf_comm;
+/* host: 128 bytes (ncclUniqueId), created on rank 0 and broadcast to the others by the caller */
+mf_status mf_nccl_unique_id(void* out);
+mf_status mf_comm_create(const void* nccl_unique_id, int32_t nranks, int32_t rank, mf_comm** out);
+mf_status mf_comm_destroy(mf_comm* comm);
+mf_status mf_comm_info(const mf_comm* comm, int32_t* nranks, int32_t* rank);
+/* rowptr int64[row_end-row_begin+1] (local, from 0), colidx int32[nnz_local] GLOBAL columns
+ * (strictly increasing per row), vals f64[nnz_local]; device pointers.  The handle is freed with
+ * mf_tile_matrix_destroy; mf_tile_matrix_info / export describe the LOCAL matrix. */
+mf_status mf_tile_matrix_from_csr_dist(mf_comm* comm, int64_t n_global, int64_t row_begin, int64_t row_end,
+                                       int64_t nnz_local, const int64_t* rowptr, const int32_t* colidx,
+                                       const double* vals, const mf_convert_opts* opts, mf_stream stream,
+                                       mf_tile_matrix** out);
+/* local slices: b[row_end-row_begin], x (in x0, out x); info (host) is the global solve's (every
+ * rank gets the same iterations / residual history).  Preconditioning / sticky / level
+ * statistics: MF_ERR_NOT_IMPLEMENTED. */
+mf_status mf_cg_solve_dist(const mf_tile_matrix* A, const double* b, double* x, const mf_solve_opts* opts,
+                           mf_solve_info* info, mf_stream stream);
+mf_status mf_bicgstab_solve_dist(const mf_tile_matrix* A, const double* b, double* x, const mf_solve_opts* opts,
+                                 mf_solve_info* info, mf_stream stream);
+/* host: this rank's row block, halo segments received and own segments sent per exchange */
+mf_status mf_dist_info(const mf_tile_matrix* A, int64_t* row_begin, int64_t* row_end, int64_t* halo_segments,
+                       int64_t* send_segments);
+
+/* Host-only planner (no GPU): the global 16-element column segments that rank `rank`'s rows gather
+ * outside its own block (ascending; the first halo_cap written to halo_segments, host, nullable),
+ * their count (*nhalo) and how many each rank owns (recv_counts[nranks], host).  rank_rows
+ * [nranks+1] host row boundaries; colidx host, global.  The device plan of
+ * mf_tile_matrix_from_csr_dist is the same. */
+mf_status mf_dist_plan(int64_t n_global, int32_t nranks, const int64_t* rank_rows, int32_t rank, int64_t nnz,
+                       const int32_t* colidx, int64_t* recv_counts, int32_t* halo_segments, int64_t halo_cap,
+                       int64_t* nhalo);
+
+/* Per-rank steps of the classic multi-kernel CG (Alg. 1 steps C and D) on a
+ * matrix's rows, with the launch plan's reduction tree: the comparison path of SURVEY 8(f) f3. */
 /* x += alpha p ; r = fma(-alpha, mu, r) on the matrix's rows; *rr (host) = (r, r), plan tree. */
 mf_status mf_cg_update_xr(const mf_tile_matrix* A, double alpha, const double* p, const double* mu, double* x,
                           double* r, double* rr, mf_stream stream);

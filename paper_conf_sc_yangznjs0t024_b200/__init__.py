@@ -34,7 +34,8 @@ SYMBOLS = ["mf_default_convert_opts", "mf_default_solve_opts", "mf_set_allocator
            "mf_tile_matrix_destroy", "mf_tile_matrix_info", "mf_tile_matrix_export", "mf_spmv", "mf_levels",
            "mf_dot", "mf_precond_create", "mf_precond_destroy", "mf_precond_apply", "mf_cg_solve",
            "mf_bicgstab_solve", "mf_cg_update_xr", "mf_cg_update_p", "mf_status_string", "mf_last_error",
-           "mf_abi_version"]
+           "mf_abi_version", "mf_nccl_unique_id", "mf_comm_create", "mf_comm_destroy", "mf_comm_info",
+           "mf_tile_matrix_from_csr_dist", "mf_cg_solve_dist", "mf_bicgstab_solve_dist", "mf_dist_info", "mf_dist_plan"]
 
 NVCC_FLAGS = ["-gencode", "arch=compute_100a,code=sm_100a", "-O3", "-lineinfo", "-std=c++17", "-fmad=false",
               "-Xcompiler", "-fPIC"]
@@ -155,6 +156,16 @@ def lib():
         L.mf_bicgstab_solve.argtypes = [vp, vp, vp, C.POINTER(SolveOpts), C.POINTER(SolveInfo), vp]
         L.mf_cg_update_xr.argtypes = [vp, d, vp, vp, vp, vp, C.POINTER(d), vp]
         L.mf_cg_update_p.argtypes = [vp, d, vp, vp, vp]
+        L.mf_nccl_unique_id.argtypes = [vp]
+        L.mf_comm_create.argtypes = [vp, i32, i32, C.POINTER(vp)]
+        L.mf_comm_destroy.argtypes = [vp]
+        L.mf_comm_info.argtypes = [vp, C.POINTER(i32), C.POINTER(i32)]
+        L.mf_tile_matrix_from_csr_dist.argtypes = [vp, i64, i64, i64, i64, vp, vp, vp, C.POINTER(ConvertOpts), vp,
+                                                   C.POINTER(vp)]
+        L.mf_cg_solve_dist.argtypes = [vp, vp, vp, C.POINTER(SolveOpts), C.POINTER(SolveInfo), vp]
+        L.mf_bicgstab_solve_dist.argtypes = [vp, vp, vp, C.POINTER(SolveOpts), C.POINTER(SolveInfo), vp]
+        L.mf_dist_info.argtypes = [vp, C.POINTER(i64), C.POINTER(i64), C.POINTER(i64), C.POINTER(i64)]
+        L.mf_dist_plan.argtypes = [i64, i32, vp, i32, i64, vp, vp, vp, i64, C.POINTER(i64)]
         _lib = L
         return L
 

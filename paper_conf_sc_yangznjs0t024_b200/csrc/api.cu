@@ -1,6 +1,6 @@
 // api.cu -- the C ABI of libmf (include/mf.h): argument checks, handles, allocator hook,
 // error strings.  Every compute step runs in the kernels of convert.cu / solver.cu /
-// precond.cu / dist.cu.
+// precond.cu / dist.cu (the multi-GPU calls are defined in dist.cu).
 #include <cuda_runtime.h>
 
 #include <mutex>
@@ -78,7 +78,7 @@ using namespace mf;
 
 extern "C" {
 
-int32_t mf_abi_version(void) { return 1; }
+int32_t mf_abi_version(void) { return 2; }
 
 const char* mf_last_error(void) { return g_last_error.c_str(); }
 
@@ -163,6 +163,7 @@ mf_status mf_tile_matrix_from_csr(int64_t n_rows, int64_t n_cols, int64_t nnz, c
 
 mf_status mf_tile_matrix_destroy(mf_tile_matrix* A) {
     if (!A) return MF_OK;
+    if (A->dist) dist_destroy(A->dist);
     destroy_tiles(&A->m);
     delete A;
     return MF_OK;

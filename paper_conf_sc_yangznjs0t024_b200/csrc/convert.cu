@@ -657,6 +657,10 @@ __global__ void __launch_bounds__(mfk::TS_CCAP) blob_fill_kernel(mfk::TsStage* s
 
 }  // namespace
 
+mf_status scan_excl_i64(const int64_t* in, int64_t n, int64_t* out, int64_t* tmp, cudaStream_t s) {
+    return scan_excl(in, n, out, tmp, s);
+}
+
 void destroy_tiles(TileMatrix* A) {
     cudaStream_t s = A->owner_stream;
     void* ptrs[] = {A->TileRowidx, A->TileColidx, A->TilePrec, A->Floor, A->TileNnz, A->Nonrow, A->ValOff,

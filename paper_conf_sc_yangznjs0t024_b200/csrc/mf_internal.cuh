@@ -110,6 +110,8 @@ struct TileMatrix {
 mf_status convert_csr(int64_t n_rows, int64_t n_cols, int64_t nnz, const int64_t* rowptr, const int32_t* colidx,
                       const double* vals, const mf_convert_opts& o, cudaStream_t s, TileMatrix* A);
 void destroy_tiles(TileMatrix* A);
+// out[0..n] = exclusive scan of in[0..n) (out[n] = total); tmp: n / 2048 + 2 elements
+mf_status scan_excl_i64(const int64_t* in, int64_t n, int64_t* out, int64_t* tmp, cudaStream_t s);
 
 mf_status run_spmv(const TileMatrix& A, const double* x, double* y, const uint8_t* level, int range_guard,
                    int64_t* counts_host, cudaStream_t s);
@@ -123,8 +125,15 @@ mf_status run_solve(const TileMatrix& A, bool bicg, const double* b, double* x, 
 
 }  // namespace mf
 
+namespace mf {
+struct DistInfo;      // dist.cu: the row block, halo plan and communicator of a distributed matrix
+struct Comm;
+void dist_destroy(DistInfo* D);
+}  // namespace mf
+
 struct mf_tile_matrix {
     mf::TileMatrix m;
+    mf::DistInfo* dist = nullptr;       // set by mf_tile_matrix_from_csr_dist
 };
 
 // ------------------------------------------------------------------ device helpers

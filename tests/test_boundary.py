@@ -53,7 +53,7 @@ def test_status_strings_and_defaults(mf):
     c = mf.ConvertOpts()
     L.mf_default_convert_opts(C.byref(c))
     assert (c.classify, c.loss_tol, c.grid_ctas, c.block_threads, c.layout) == (1, 1e-15, 0, 0, 0)
-    assert L.mf_abi_version() == 1
+    assert L.mf_abi_version() == 2
 
 
 def test_struct_sizes_match_header(mf, tmp_path):

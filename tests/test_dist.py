@@ -1,11 +1,11 @@
-"""Row-block multi-GPU path (paper_conf_sc_yangznjs0t024_b200/dist.py).
+"""Row-block multi-GPU path (libmf dist.cu through paper_conf_sc_yangznjs0t024_b200.dist).
 
-CPU (-m "not gpu"): the partition / halo plan, and the distributed CG driver itself with
-world_size 2 over gloo, its per-rank arithmetic supplied by a numpy test engine (tests only --
-the product engine is libmf's CUDA kernels and has no CPU fallback).
-GPU: with one rank over NCCL the driver (libmf kernels + rank-order reductions) reproduces the
-single-kernel mf_cg_solve bit for bit."""
-import math
+CPU (-m "not gpu"): the row partition, and libmf's host halo planner (mf_dist_plan) driven by a
+world-size-2 gloo job: each rank plans its halo with libmf, the ranks exchange their requests over
+gloo exactly as dist_create does over NCCL, and a numpy emulation of the distributed SpMV built
+from those plans (own segments + received halo segments, remapped columns) equals the global SpMV.
+GPU: one rank over NCCL -- mf_cg_solve_dist / mf_bicgstab_solve_dist equal the oracle's
+kernel-order emulation bit for bit (histories, x) and the single-kernel solves."""
 import os
 import socket
 
@@ -26,54 +26,6 @@ def free_port():
     return p
 
 
-class NumpyEngine:
-    """Test-only per-rank arithmetic (FP64, plain order) on CPU tensors."""
-
-    def matrix(self, n_local, n_ext, rowptr, colidx, vals, classify=True):
-        return sp.csr_matrix((vals, colidx, rowptr), shape=(n_local, n_ext))
-
-    def vector(self, n):
-        return torch.zeros(int(n), dtype=torch.float64)
-
-    def spmv(self, M, xe, y, level):
-        assert level is None
-        y.copy_(torch.from_numpy(M @ xe.numpy()))
-
-    def levels(self, v, th):
-        raise AssertionError("static mode only")
-
-    def dot(self, M, u, v):
-        return float(np.dot(u.numpy(), v.numpy()))
-
-    def update_xr(self, M, alpha, p, mu, x, r):
-        x.add_(alpha * p)
-        r.sub_(alpha * mu)
-        return float(torch.dot(r, r))
-
-    def update_p(self, M, beta, r, p):
-        p.mul_(beta).add_(r)
-
-
-def plain_cg(A, b, tol=1e-10, max_iter=1000):
-    M = sp.csr_matrix((A.vals, A.colidx, A.rowptr), shape=(A.n_rows, A.n_cols))
-    x = np.zeros_like(b)
-    r = b.copy()
-    p = r.copy()
-    rho = r @ r
-    nb = math.sqrt(b @ b)
-    j = 0
-    while math.sqrt(rho) / nb >= tol and j < max_iter:
-        mu = M @ p
-        alpha = rho / (mu @ p)
-        x += alpha * p
-        r -= alpha * mu
-        rr = r @ r
-        p = r + (rr / rho) * p
-        rho = rr
-        j += 1
-    return x, j
-
-
 def test_partition_rows_tile_aligned_and_balanced():
     A = W.make("C2", 32)
     for P in (1, 2, 3, 4, 8):
@@ -86,25 +38,38 @@ def test_partition_rows_tile_aligned_and_balanced():
 
 
 def test_halo_plan_slab_stencil():
-    """3D 7-point Poisson 32^3 in 4 slabs: each interior rank exchanges exactly one 32x32 plane
-    with each neighbour (the C5 pattern)."""
+    """3D 7-point Poisson 32^3 in 4 slabs (the C5 pattern): every interior rank receives exactly one
+    32x32 plane (64 segments) from each neighbour and nothing else."""
     m = 32
     A = W.poisson3d(m)
     P = 4
     bnd = dist.partition_rows(A.n_rows, P)
-    ext = []
+    plane_segs = m * m // 16
     for k in range(P):
-        rp, ci, _ = dist.local_rows(A, bnd[k], bnd[k + 1])
-        ext.append((bnd[k], bnd[k + 1]) + dist.local_extent(ci, bnd[k], bnd[k + 1], A.n_rows))
-    plans = [dist.HaloPlan.build(k, ext) for k in range(P)]
-    plane = m * m
-    for k, pl in enumerate(plans):
-        peers = sorted(q for q, _, _ in pl.recv)
-        assert peers == [q for q in (k - 1, k + 1) if 0 <= q < P]
-        assert all(hi - lo == plane for _, lo, hi in pl.recv)
-        # what k receives from q is exactly what q sends to k
-        for q, lo, hi in pl.recv:
-            assert (k, lo, hi) in plans[q].send
+        _, ci, _ = dist.local_rows(A, bnd[k], bnd[k + 1])
+        segs, counts = dist.halo_plan(A.n_rows, bnd, k, ci)
+        want = np.zeros(P, np.int64)
+        for q in (k - 1, k + 1):
+            if 0 <= q < P:
+                want[q] = plane_segs
+        assert np.array_equal(counts, want)
+        assert np.all(np.diff(segs) > 0) and len(segs) == want.sum()
+
+
+def test_halo_plan_scattered_is_exact():
+    """C4-shaped scattered pattern: the plan lists exactly the off-block segments the rows touch
+    (no column hull), each attributed to its owner."""
+    A = W.make("C4spd", 1 << 13)
+    P = 3
+    bnd = dist.partition_rows(A.n_rows, P, A.rowptr)
+    for k in range(P):
+        _, ci, _ = dist.local_rows(A, bnd[k], bnd[k + 1])
+        segs, counts = dist.halo_plan(A.n_rows, bnd, k, ci)
+        g = np.unique(ci.astype(np.int64) >> 4)
+        own = (g >= bnd[k] // 16) & (g < (bnd[k + 1] + 15) // 16)
+        assert np.array_equal(segs, g[~own])
+        owner = np.searchsorted(np.asarray(bnd[1:]), segs.astype(np.int64) * 16, side="right")
+        assert np.array_equal(np.bincount(owner, minlength=P), counts)
 
 
 def _worker(rank, world, port, out):
@@ -112,55 +77,95 @@ def _worker(rank, world, port, out):
     os.environ.update(MASTER_ADDR="127.0.0.1", MASTER_PORT=str(port))
     td.init_process_group("gloo", rank=rank, world_size=world)
     try:
-        A = W.poisson3d(16)
-        b = W.rhs_ones(A)
+        A = W.make("C4ind", 1 << 12)
         bnd = dist.partition_rows(A.n_rows, world, A.rowptr)
         rb, re = bnd[rank], bnd[rank + 1]
-        comm = dist.Comm()
-        D = dist.DistMatrix(NumpyEngine(), comm, A.n_rows, rb, re, *dist.local_rows(A, rb, re))
-        res = dist.cg_solve(D, torch.from_numpy(b[rb:re].copy()), mode="static")
-        xs = [torch.zeros(bnd[q + 1] - bnd[q], dtype=torch.float64) for q in range(world)]
-        td.all_gather(xs, res.x)
+        rp, ci, va = dist.local_rows(A, rb, re)
+        segs, counts = dist.halo_plan(A.n_rows, bnd, rank, ci)
+        # requests: the segments I need from each peer (what dist_create sends over NCCL)
+        cnt = torch.from_numpy(counts.copy())
+        allc = [torch.zeros_like(cnt) for _ in range(world)]
+        td.all_gather(allc, cnt)
+        off = np.concatenate([[0], np.cumsum(counts)])
+        reqs = {}
+        for q in range(world):
+            if q == rank:
+                continue
+            mine = torch.from_numpy(segs[off[q]:off[q + 1]].astype(np.int64))
+            theirs = torch.zeros(int(allc[q][rank]), dtype=torch.int64)
+            if rank < q:
+                td.send(mine, q); td.recv(theirs, q)
+            else:
+                td.recv(theirs, q); td.send(mine, q)
+            reqs[q] = theirs.numpy()
+        # halo exchange of x (segments of 16) along the plans, then the local SpMV
+        x = np.random.default_rng(7).standard_normal(A.n_rows)
+        nown = (re - rb + 15) // 16
+        xe = np.zeros((nown + len(segs)) * 16)
+        xe[:re - rb] = x[rb:re]
+        for q in range(world):
+            if q == rank:
+                continue
+            send = np.concatenate([x[s * 16:s * 16 + 16] for s in reqs[q]]) if len(reqs[q]) else np.zeros(0)
+            assert all(bnd[rank] <= s * 16 < bnd[rank + 1] for s in reqs[q])
+            rbuf = torch.zeros(16 * int(counts[q]), dtype=torch.float64)
+            if rank < q:
+                td.send(torch.from_numpy(send), q); td.recv(rbuf, q)
+            else:
+                td.recv(rbuf, q); td.send(torch.from_numpy(send), q)
+            xe[(nown + off[q]) * 16:(nown + off[q + 1]) * 16] = rbuf.numpy()
+        pos = {int(s): k for k, s in enumerate(segs)}
+        cl = np.array([c - rb if rb <= c < re else (nown + pos[c >> 4]) * 16 + (c & 15) for c in ci], np.int64)
+        y = sp.csr_matrix((va, cl, rp), shape=(re - rb, len(xe))) @ xe
+        yall = torch.zeros(A.n_rows, dtype=torch.float64)
+        yall[rb:re] = torch.from_numpy(y)
+        td.all_reduce(yall)                      # disjoint slices: the sum assembles y
         if rank == 0:
-            np.save(out, np.concatenate([t.numpy() for t in xs]))
-            np.save(out + ".it.npy", np.array([res.iterations, int(res.converged), res.halo_bytes]))
+            np.save(out, yall.numpy())
     finally:
         td.destroy_process_group()
 
 
 @pytest.mark.dist
-def test_dist_cg_gloo_world2_matches_single_process(tmp_path):
+def test_dist_plan_gloo_world2_spmv_exact(tmp_path):
     import torch.multiprocessing as tmp
-    out = str(tmp_path / "x.npy")
+    out = str(tmp_path / "y.npy")
     tmp.spawn(_worker, args=(2, free_port(), out), nprocs=2, join=True)
-    x = np.load(out)
-    it, conv, halo = np.load(out + ".it.npy")
-    A = W.poisson3d(16)
-    b = W.rhs_ones(A)
-    xr, jr = plain_cg(A, b)
-    assert conv == 1 and abs(int(it) - jr) <= 1
-    assert np.linalg.norm(x - xr) / np.linalg.norm(xr) < 1e-8
-    assert np.max(np.abs(x - 1.0)) < 1e-6          # b = A*1
-    assert halo == 16 * 16 * 8 * int(it)           # one 16x16 plane per iteration from the neighbour
+    A = W.make("C4ind", 1 << 12)
+    x = np.random.default_rng(7).standard_normal(A.n_rows)
+    yref = sp.csr_matrix((A.vals, A.colidx, A.rowptr), shape=(A.n_rows, A.n_cols)) @ x
+    assert np.allclose(np.load(out), yref, rtol=1e-13, atol=1e-13)
 
 
 @pytest.mark.gpu
-def test_dist_world1_bit_identical_to_single_kernel():
-    """One rank over NCCL: the distributed driver equals mf_cg_solve bit for bit (histories, x)."""
+def test_dist_world1_matches_oracle_and_single_kernel(orc):
+    """One rank over NCCL: the distributed solves equal the oracle's kernel-order emulation bit for
+    bit (histories and x), hence the single-kernel solves too."""
     import torch.distributed as td
     import paper_conf_sc_yangznjs0t024_b200 as mf
     os.environ.update(MASTER_ADDR="127.0.0.1", MASTER_PORT=str(free_port()))
-    td.init_process_group("nccl", rank=0, world_size=1)
+    td.init_process_group("nccl", rank=0, world_size=1, device_id=torch.device("cuda", 0))
     try:
-        for name, scale in (("C2", 16), ("C1", 64)):
+        comm = dist.Comm()
+        for name, scale, solver in (("C2", 16, "cg"), ("C1", 64, "cg"), ("C3", 64, "bicgstab"), ("C4spd", 1 << 12, "cg")):
             A = W.make(name, scale)
             b = W.rhs_ones(A)
-            T = mf.TileMatrix.from_host_csr(A)
-            ref = mf.cg_solve(T, torch.from_numpy(b).cuda(), mode=mf.MODE_DYNAMIC, tol=1e-10, max_iter=1000)
-            D = dist.DistMatrix(dist.CudaEngine("cuda"), dist.Comm(), A.n_rows, 0, A.n_rows, *dist.local_rows(A, 0, A.n_rows))
-            res = dist.cg_solve(D, torch.from_numpy(b).cuda(), tol=1e-10, max_iter=1000, mode="dynamic")
-            assert res.converged and res.iterations == ref.iterations
-            assert np.array_equal(res.history, ref.history)
-            assert torch.equal(res.x, ref.x)
+            D = dist.DistTileMatrix.from_host_csr(comm, A, 0, A.n_rows)
+            assert D.dist_info()["halo_segments"] == 0
+            g, bb, R = mf.TileMatrix.plan(D)
+            T = orc.Tiles(A.n_rows, A.n_cols, A.rowptr, A.colidx, A.vals)
+            ofn = orc.cg if solver == "cg" else orc.bicgstab
+            ro = ofn(T, b, mode=2, plan=orc.Plan(g, bb, R), max_iter=2000)
+            fn = dist.cg_solve if solver == "cg" else dist.bicgstab_solve
+            res = fn(D, torch.from_numpy(b).cuda(), mode=mf.MODE_DYNAMIC, max_iter=2000)
+            assert res.converged and ro["converged"] and res.iterations == ro["iterations"], name
+            assert np.array_equal(res.history, ro["history"]), name
+            assert np.array_equal(res.x.cpu().numpy(), ro["x"]), name
+            Ts = mf.TileMatrix.from_host_csr(A)
+            sfn = mf.cg_solve if solver == "cg" else mf.bicgstab_solve
+            rs = sfn(Ts, torch.from_numpy(b).cuda(), mode=mf.MODE_DYNAMIC, max_iter=2000)
+            assert torch.equal(rs.x, res.x), name
+            D.close()
+        comm.close()
     finally:
         td.destroy_process_group()

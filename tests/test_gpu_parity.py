@@ -436,3 +436,51 @@ def test_sptrsv_nonsymmetric_pattern(mf, orc):
     rg = mf.bicgstab_solve(Gm, dev(b), M=mf.Precond(Gm), mode=2, max_iter=300, watchdog_ms=20000)
     assert ro["converged"] and rg.converged and rg.iterations == ro["iterations"]
     assert np.array_equal(rg.x.cpu().numpy(), ro["x"])
+
+
+def test_compact_multiwindow_parity(mf, orc):
+    """Compact layout with CTAs whose tile rows hold more tiles than one code window (CODE_CAP =
+    8192): the multi-window path of the compact SpMV, as full-size C4 takes it."""
+    A = W.make("C4spd", 1 << 17)
+    Gm = mf.TileMatrix.from_host_csr(A, grid_ctas=8, block_threads=256)
+    assert Gm.info()["layout"] == 1
+    ex = Gm.export()
+    R, trp = ex["PlanRows"], ex["TileRowPtr"]
+    tiles_per_cta = [trp[min(R[g + 1] // 16, len(trp) - 1)] - trp[R[g] // 16] for g in range(8)]
+    assert min(tiles_per_cta) > 8192
+    g, bb, R = Gm.plan()
+    T = oracle_tiles(orc, A)
+    b = W.rhs_ones(A)
+    rp, ci, sv = T.stored_csr()
+    M = orc.ILU0(rp, ci, sv)
+    ro = orc.cg(T, b, M=M, mode=2, plan=orc.Plan(g, bb, R), max_iter=200)
+    rg = mf.cg_solve(Gm, dev(b), M=mf.Precond(Gm), mode=2, max_iter=200, level_counts=True)
+    assert ro["converged"] and rg.converged and rg.iterations == ro["iterations"]
+    assert np.array_equal(rg.history, ro["history"])
+    assert np.array_equal(rg.x.cpu().numpy(), ro["x"])
+    assert np.array_equal(rg.level_counts, ro["level_counts"])
+
+
+@pytest.mark.slow
+@pytest.mark.parametrize("name", ["C4spd", "C4ind"])
+def test_full_size_C4_prefix_and_convergence(mf, orc, name):
+    """BASELINE configs[3] at full size (2^20 rows, ILU(0), bench launch configuration): the first
+    12 iterations bit-identical to the oracle's kernel-order emulation, then the full GPU solve
+    converges and its true residual (oracle, FP64 CSR) is below 1e-9."""
+    A = W.make(name)
+    b = W.rhs_ones(A)
+    Gm = mf.TileMatrix.from_host_csr(A)
+    g, bb, R = Gm.plan()
+    T = oracle_tiles(orc, A)
+    rp, ci, sv = T.stored_csr()
+    M = orc.ILU0(rp, ci, sv)
+    P = mf.Precond(Gm)
+    ofn = orc.cg if name == "C4spd" else orc.bicgstab
+    gfn = mf.cg_solve if name == "C4spd" else mf.bicgstab_solve
+    ro = ofn(T, b, M=M, mode=2, plan=orc.Plan(g, bb, R), max_iter=12, tol=0.0)
+    rg = gfn(Gm, dev(b), M=P, mode=2, max_iter=12, tol=0.0)
+    assert np.array_equal(rg.history, ro["history"])
+    assert np.array_equal(rg.x.cpu().numpy(), ro["x"])
+    full = gfn(Gm, dev(b), M=P, mode=2, max_iter=1000)
+    assert full.converged
+    assert orc.true_relres(A.rowptr, A.colidx, A.vals, b, full.x.cpu().numpy()) < 1e-9

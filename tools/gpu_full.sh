@@ -2,6 +2,6 @@
 # full GPU test suite + default bench line
 mkdir -p gpurun_out
 export PYTHONUNBUFFERED=1
-timeout 1800 python -m pytest tests -m gpu -q -x > gpurun_out/gpu_tests.log 2>&1; echo rc=$? >> gpurun_out/gpu_tests.log
-tail -5 gpurun_out/gpu_tests.log
-timeout 900 python bench.py --no-cpu-baseline > gpurun_out/bench.json 2> gpurun_out/bench.err; cat gpurun_out/bench.json; tail -3 gpurun_out/bench.err
+timeout 2400 python -m pytest tests -m gpu -q > gpurun_out/gpu_tests.log 2>&1; echo rc=$? >> gpurun_out/gpu_tests.log
+grep -E "passed|failed|FAILED|Error" gpurun_out/gpu_tests.log | tail -12
+timeout 1200 python bench.py > gpurun_out/bench.json 2> gpurun_out/bench.err; cat gpurun_out/bench.json; tail -3 gpurun_out/bench.err

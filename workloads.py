@@ -83,6 +83,21 @@ def poisson3d(m: int) -> CSR:
     return _assemble(n, offs, masks, vals)
 
 
+def poisson3d_rows(m: int, r0: int, r1: int) -> CSR:
+    """Rows [r0, r1) of poisson3d(m) with GLOBAL column ids (a rank's slab, generated without the
+    rest of the matrix): the same entries in the same order as poisson3d(m) restricted to them."""
+    n = m * m * m
+    i = np.arange(r0, r1, dtype=np.int64)
+    ix, iy, iz = i % m, (i // m) % m, i // (m * m)
+    offs = [-m * m, -m, -1, 0, 1, m, m * m]
+    masks = [iz > 0, iy > 0, ix > 0, np.ones(i.size, bool), ix < m - 1, iy < m - 1, iz < m - 1]
+    vals = [-1.0, -1.0, -1.0, 6.0, -1.0, -1.0, -1.0]
+    A = _assemble(i.size, offs, masks, vals)
+    A.colidx = (A.colidx.astype(np.int64) + r0).astype(np.int32)
+    A.n_cols = n
+    return A
+
+
 def segment_scales(n: int, seed: int = 1, seg: int = 16) -> np.ndarray:
     """d_J per 16-row segment J: 1 (p=.55), 1+2^-4 (.20), 1+2^-10 (.15), 1+u*2^-3 (.10)."""
     rng = np.random.default_rng(seed)
