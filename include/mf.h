@@ -130,6 +130,9 @@ typedef struct {
                                    Implied when tile_level_counts != NULL. */
     int32_t watchdog_ms;        /* spin watchdog of the grid barriers / ready flags / SpTRSV (0 = 60000 ms);
                                    expiry returns MF_ERR_DEADLOCK */
+    int32_t cg_variant;         /* mf_cg_solve: 0 (default) Alg. 1 (two grid reductions per iteration);
+                                   1 single-reduction CG (Chronopoulos-Gear; one reduction, the dynamic
+                                   switch watching r, the SpMV input of that variant) */
 } mf_solve_opts;
 
 typedef struct {

@@ -109,6 +109,9 @@ def lib():
                            vp, i64, vp, i64, C.POINTER(_Info)]
             L.orc_pcg.argtypes = solver_args; L.orc_pcg.restype = C.c_int
             L.orc_pbicgstab.argtypes = solver_args; L.orc_pbicgstab.restype = C.c_int
+            L.orc_cg_single_reduction.argtypes = [C.POINTER(_Tiles), vp, vp, C.POINTER(_Opts), C.POINTER(_Plan),
+                                                  vp, i64, vp, i64, C.POINTER(_Info)]
+            L.orc_cg_single_reduction.restype = C.c_int
             L.orc_cg_csr.argtypes = [i64, vp, vp, vp, vp, vp, d, i64, vp, i64, C.POINTER(_Info)]
             L.orc_cg_csr.restype = C.c_int
             L.orc_true_relres.argtypes = [i64, vp, vp, vp, vp, vp]; L.orc_true_relres.restype = d
@@ -376,6 +379,18 @@ def cg(A, b, x0=None, tol=1e-10, max_iter=1000, mode=MODE_DYNAMIC, switch_eps=No
     hist_cap = hist_cap or max_iter + 2
     return _solve(lib().orc_pcg, A, b, x0, M, tol, max_iter, mode, switch_eps, switch_absolute, sticky,
                   range_guard, plan, hist_cap)
+
+
+def cg_single_reduction(A, b, x0=None, tol=1e-10, max_iter=1000, mode=MODE_DYNAMIC, switch_eps=None,
+                        switch_absolute=False, sticky=False, range_guard=True, plan=None, hist_cap=None):
+    """The one-reduction (Chronopoulos-Gear) CG variant, same options as cg()."""
+    hist_cap = hist_cap or max_iter + 2
+    L = lib()
+
+    def fn(At, M, b_, x_, o, pl, h, hc, lc, lcc, info):
+        return L.orc_cg_single_reduction(At, b_, x_, o, pl, h, hc, lc, lcc, info)
+    return _solve(fn, A, b, x0, None, tol, max_iter, mode, switch_eps, switch_absolute, sticky, range_guard, plan,
+                  hist_cap)
 
 
 def bicgstab(A, b, x0=None, tol=1e-10, max_iter=1000, mode=MODE_DYNAMIC, switch_eps=None,

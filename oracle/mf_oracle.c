@@ -984,3 +984,84 @@ done:
     free(r); free(rh); free(p); free(mu); free(s); free(th); free(ph); free(sh);
     return st;
 }
+
+/* ------------------------------------------------------------------------------------
+ * 10. Single-reduction CG (the one-barrier variant of Alg. 1; Chronopoulos &
+ *     Gear, "s-step iterative methods", 1989): the two dots of an iteration share ONE reduction
+ *     because delta = (A r, r) replaces (A p, p):
+ *       r0 = b - A~ x0 ; w0 = A~_0 r0 ; gamma0 = (r0, r0) ; delta0 = (w0, r0) ; alpha0 = gamma0/delta0
+ *       beta0 = 0 ; p = s = 0
+ *       loop i: relres_i = sqrt(gamma_i)/||b|| ; stop test as in CG
+ *         p = fma(beta_i, p, r) ; s = fma(beta_i, s, w)          (s = A~ p by recurrence)
+ *         x = fma(alpha_i, p, x) ; r = fma(-alpha_i, s, r)
+ *         w = A~_{i+1} r                                        (the SpMV input is r: the dynamic
+ *                                                                switch watches r)
+ *         gamma' = (r, r) ; delta' = (w, r)                     (one reduction)
+ *         beta' = gamma'/gamma ; t = (beta' * gamma') / alpha ; alpha' = gamma' / (delta' - t)
+ *       breakdown: delta' - t <= 0 or non-finite (SPD => (p', A p') > 0).
+ *     Iterations = loop passes (the SpMVs are iterations + 1).  tau from ||r0|| (v0 = r0).
+ * ---------------------------------------------------------------------------------- */
+int orc_cg_single_reduction(const orc_tiles* A, const double* b, double* x, const orc_opts* o, const orc_plan* plan,
+                            double* hist, int64_t hist_cap, int64_t* level_counts, int64_t lc_cap, orc_info* info) {
+    int64_t n = A->n_rows;
+    if (A->n_rows != A->n_cols) return ORC_ERR_INVALID_ARG;
+    orc_ctx c;
+    if (ctx_init(&c, A, o, plan, level_counts, lc_cap) != ORC_OK) return ORC_ERR_OOM;
+    size_t nb8 = sizeof(double) * (size_t)(n > 0 ? n : 1);
+    double *r = malloc(nb8), *p = calloc((size_t)(n > 0 ? n : 1), sizeof(double)), *s = calloc((size_t)(n > 0 ? n : 1), sizeof(double)),
+           *w = malloc(nb8);
+    int st = ORC_OK;
+    int64_t j = 0;
+    memset(info, 0, sizeof(*info));
+    initial_residual(A, b, x, r);
+    double nb = sqrt(orc_dot(b, b, n, plan));
+    if (nb == 0.0) {
+        for (int64_t i = 0; i < n; ++i) x[i] = 0.0;
+        info->converged = 1; record(hist, hist_cap, 0, 0.0);
+        goto done;
+    }
+    double gamma = orc_dot(r, r, n, plan);
+    ctx_set_tau(&c, sqrt(gamma));
+    double alpha = 0.0, beta = 0.0;
+    {
+        double relres = sqrt(gamma) / nb;
+        if (!(relres < o->tol) && o->max_iter > 0) {      /* the first SpMV only when iterating */
+            ctx_spmv(&c, r, w);
+            double delta = orc_dot(w, r, n, plan);
+            if (!(delta > 0.0) || !isfinite(delta)) { st = ORC_ERR_BREAKDOWN; record(hist, hist_cap, 0, relres); info->rel_residual = relres; goto done; }
+            alpha = gamma / delta;
+        }
+    }
+    for (;; ++j) {
+        double relres = sqrt(gamma) / nb;
+        record(hist, hist_cap, j, relres);
+        info->rel_residual = relres;
+        if (relres < o->tol) { info->converged = 1; break; }
+        if (j == o->max_iter) break;
+        for (int64_t i = 0; i < n; ++i) {
+            p[i] = fma(beta, p[i], r[i]);
+            s[i] = fma(beta, s[i], w[i]);
+            x[i] = fma(alpha, p[i], x[i]);
+            r[i] = fma(-alpha, s[i], r[i]);
+        }
+        ctx_spmv(&c, r, w);
+        double gamma1 = orc_dot(r, r, n, plan);
+        double delta1 = orc_dot(w, r, n, plan);
+        double beta1 = gamma1 / gamma;
+        double t = (beta1 * gamma1) / alpha;
+        double den = delta1 - t;
+        if (!(den > 0.0) || !isfinite(den)) {
+            /* the residual is updated: report it before breaking down */
+            ++j; relres = sqrt(gamma1) / nb; record(hist, hist_cap, j, relres); info->rel_residual = relres;
+            if (relres < o->tol) info->converged = 1; else st = ORC_ERR_BREAKDOWN;
+            break;
+        }
+        alpha = gamma1 / den;
+        beta = beta1;
+        gamma = gamma1;
+    }
+done:
+    info->iterations = j; info->status = st; info->n_spmv = c.n_spmv;
+    free(r); free(p); free(s); free(w); ctx_free(&c);
+    return st;
+}

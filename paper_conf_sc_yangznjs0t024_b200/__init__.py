@@ -108,7 +108,7 @@ class SolveOpts(C.Structure):
                 ("switch_absolute", C.c_int32), ("sticky", C.c_int32), ("range_guard", C.c_int32),
                 ("M", C.c_void_p), ("residual_history", C.c_void_p), ("history_cap", C.c_int64),
                 ("tile_level_counts", C.c_void_p), ("level_counts_cap", C.c_int64), ("collect_stats", C.c_int32),
-                ("watchdog_ms", C.c_int32)]
+                ("watchdog_ms", C.c_int32), ("cg_variant", C.c_int32)]
 
 
 class SolveInfo(C.Structure):
@@ -345,7 +345,8 @@ class SolveResult:
 
 def _solve(fn, A: TileMatrix, b, x0=None, tol=1e-10, max_iter=1000, mode=MODE_DYNAMIC, switch_eps=None,
            switch_absolute=False, range_guard=True, sticky=False, history=True, level_counts=False,
-           collect_stats=False, M=None, stream=None, raise_on_breakdown=True, watchdog_ms=0) -> SolveResult:
+           collect_stats=False, M=None, stream=None, raise_on_breakdown=True, watchdog_ms=0,
+           cg_variant=0) -> SolveResult:
     import torch
     _need_cuda(b, torch.float64, "b")
     x = torch.zeros_like(b) if x0 is None else x0.clone()
@@ -363,6 +364,7 @@ def _solve(fn, A: TileMatrix, b, x0=None, tol=1e-10, max_iter=1000, mode=MODE_DY
         o.tile_level_counts, o.level_counts_cap = lc.ctypes.data, lc.shape[0]
     o.collect_stats = int(collect_stats)
     o.watchdog_ms = int(watchdog_ms)
+    o.cg_variant = int(cg_variant)
     info = SolveInfo()
     st = fn(A._h, _ptr(b), _ptr(x), C.byref(o), C.byref(info), _stream_ptr(stream))
     if st != 0 and (raise_on_breakdown or st != 7):

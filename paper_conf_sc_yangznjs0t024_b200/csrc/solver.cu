@@ -125,7 +125,8 @@ __global__ void dot_final_kernel(const double* __restrict__ slots, int G, double
     if (threadIdx.x == 0) *out = gt;
 }
 
-void* pick_kernel(int maxt, bool bicg, bool dyn, bool count, bool sticky, bool pre) {
+void* pick_kernel(int maxt, bool bicg, bool dyn, bool count, bool sticky, bool pre, bool sr = false) {
+    if (sr) return maxt > 512 ? pick_cgsr_1024(dyn, count, sticky) : pick_cgsr_512(dyn, count, sticky);
     if (maxt > 512) {
         if (pre && bicg) return pick_pbicgstab_1024(dyn, count, sticky);
         if (pre) return pick_pcg_1024(dyn, count, sticky);
@@ -309,6 +310,9 @@ mf_status run_solve(const TileMatrix& A, bool bicg, const double* b, double* x, 
         return fail(MF_ERR_NOT_IMPLEMENTED, "sticky downgrade does not collect per-SpMV level statistics");
     Precond* P = o.M ? const_cast<Precond*>(&o.M->p) : nullptr;
     const bool pre = P != nullptr;
+    const bool sr = !bicg && o.cg_variant == 1;       // single-reduction CG
+    if (sr && pre) return fail(MF_ERR_NOT_IMPLEMENTED, "single-reduction CG with a preconditioner");
+    if (o.cg_variant != 0 && o.cg_variant != 1) return fail(MF_ERR_INVALID_ARG, "cg_variant must be 0 or 1");
     if (pre && P->n != A.n_rows) return fail(MF_ERR_INVALID_ARG, "preconditioner built for another matrix size");
     int dev = 0, sms = 0, smem_optin = 0;
     MF_CUDA(cudaGetDevice(&dev));
@@ -343,7 +347,7 @@ mf_status run_solve(const TileMatrix& A, bool bicg, const double* b, double* x, 
     const size_t smem = fixed + mfk::spmv_smem_bytes(A.ts, nst, A.slot_bytes, A.ecap, B / 32) + (size_t)cap * 8 * nvec + (size_t)pre_smem + 64;
     if ((int64_t)smem > smem_optin) return fail(MF_ERR_UNSUPPORTED, "shared-memory plan exceeds the device limit");
 
-    void* kfn = pick_kernel(B, bicg, dyn, count, sticky, pre);
+    void* kfn = pick_kernel(B, bicg, dyn, count, sticky, pre, sr);
     MF_CUDA(cudaFuncSetAttribute(kfn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
     int per_sm = 0;
     MF_CUDA(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, kfn, B, smem));
@@ -368,13 +372,19 @@ mf_status run_solve(const TileMatrix& A, bool bicg, const double* b, double* x, 
         MF_TRY(ws.get(&sv, pbicg ? n : npv));
         if (spill) MF_TRY(ws.get(&th_g, n));
     }
+    if (sr) {    // p and s of the single-reduction CG (start at 0)
+        MF_TRY(ws.get(&rh, n));
+        MF_TRY(ws.get(&sv, n));
+        MF_CUDA(cudaMemsetAsync(rh, 0, n * sizeof(double), s));
+        MF_CUDA(cudaMemsetAsync(sv, 0, n * sizeof(double), s));
+    }
     if (pre) {
         MF_TRY(ws.get(&pz, bicg ? npv : n));
         if (bicg) MF_TRY(ws.get(&psh, npv));
     }
     // PV vectors: padding rows / slots stay zero
     if (!pbicg) MF_CUDA(cudaMemsetAsync(p, 0, npv * sizeof(double), s));
-    if (sv && !pbicg) MF_CUDA(cudaMemsetAsync(sv, 0, npv * sizeof(double), s));
+    if (sv && !pbicg && !sr) MF_CUDA(cudaMemsetAsync(sv, 0, npv * sizeof(double), s));
     if (pz && bicg) MF_CUDA(cudaMemsetAsync(pz, 0, npv * sizeof(double), s));
     if (psh) MF_CUDA(cudaMemsetAsync(psh, 0, npv * sizeof(double), s));
     MF_TRY(ws.get(&slots, (size_t)2 * NSLOT * G));
@@ -444,7 +454,7 @@ mf_status run_solve(const TileMatrix& A, bool bicg, const double* b, double* x, 
     info->status = (mf_status)(int)hout[3];
     info->kernel_ms = ms;
     info->launches = 1;
-    const int64_t nspmv = (bicg ? 2 : 1) * iters;
+    const int64_t nspmv = (bicg ? 2 : 1) * iters + (sr && iters > 0 ? 1 : 0);
     info->n_spmv = nspmv;
     if (o.residual_history && o.history_cap > 0) {
         const int64_t k = std::min<int64_t>(o.history_cap, std::min<int64_t>(iters + 1, hist_cap));
@@ -479,7 +489,7 @@ mf_status run_solve(const TileMatrix& A, bool bicg, const double* b, double* x, 
     // vectors: CG 48n per iteration (read p,x,r; write x,r,p); BiCGSTAB 72n (read p,x,r,r0*,s;
     // write s,x,r,p); + 16n per SpMV output that cannot stay on chip (capacity rule, SURVEY 8(d):
     // counted when the outputs do not fit the GPU's shared memory, whatever this launch did)
-    const double vec = bicg ? 72.0 : 48.0;
+    const double vec = bicg ? 72.0 : (sr ? 72.0 : 48.0);   // single-reduction CG: read p,s,x,r,w; write p,s,x,r
     int smem_sm = 0;
     MF_CUDA(cudaDeviceGetAttribute(&smem_sm, cudaDevAttrMaxSharedMemoryPerMultiprocessor, dev));
     const bool over_cap = 8.0 * (double)n * (double)nvec > (double)sms * (double)smem_sm;

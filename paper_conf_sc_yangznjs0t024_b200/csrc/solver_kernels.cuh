@@ -114,6 +114,7 @@ __device__ __forceinline__ bool grid_barrier(const SolveArgs& a, Ctx& c) {
     __shared__ int s_abort;
     c.bar_target += (unsigned)a.G;
     __syncthreads();
+    if (a.G == 1) return true;            // one CTA (small matrices): the CTA barrier orders everything
     if (threadIdx.x == 0) {
         const unsigned long long t0 = gtimer();
         red_release_add(a.bar, 1u);       // cumulative release: this CTA's writes (ordered by bar.sync)
@@ -139,6 +140,10 @@ __device__ __forceinline__ void publish(const SolveArgs& a, unsigned epoch) {
 
 __device__ __forceinline__ bool wait_deps(const SolveArgs& a, unsigned epoch) {
     __shared__ int s_abort;
+    if (a.G == 1 && a.stall_cta < 0) {   // one CTA: its own writes, ordered by the CTA barrier
+        __syncthreads();
+        return true;
+    }
     const int lo = a.dep_lo[blockIdx.x], hi = a.dep_hi[blockIdx.x];
     if (threadIdx.x == 0) s_abort = 0;
     __syncthreads();
@@ -451,6 +456,154 @@ __global__ void __launch_bounds__(MAXT, 1) cg_persistent(SolveArgs a) {
             }
             publish(a, (unsigned)(j + 3));
             tm.tick(5);
+        }
+    }
+    if (blockIdx.x == 0 && t == 0) {
+        a.out[0] = (double)j;
+        a.out[1] = converged;
+        a.out[3] = status;
+    }
+    tm.flush(a);
+    if (status == MF_ERR_DEADLOCK && t == 0) atomicExch(a.abort_flag, 1);
+}
+
+// -------------------------------------------------------------------------- single-reduction CG
+// the one-barrier variant of Alg. 1 (Chronopoulos & Gear; oracle
+// orc_cg_single_reduction).  The SpMV input is r (PV layout, levels of r: "the input vector
+// in SpMV"), w = A~ r; (r, r) is accumulated in the vector phase and (w, r) in the SpMV, and both go
+// through ONE grid reduction per iteration.  p and s (= A~ p by recurrence) are plain vectors
+// (a.rh, a.s).  Phases: 0 wait r, 1 SpMV + (w,r), 2 reduce, 3 vector update + (r,r) + publish, 6 init
+template <bool DYN, bool COUNT, bool STK, int MAXT>
+__global__ void __launch_bounds__(MAXT, 1) cgsr_persistent(SolveArgs a) {
+    constexpr int PF = MAXT >= 1024 ? 4 : 8;
+    Smem sm = carve(a, 1);
+    Ctx c;
+    Timer tm;
+    tm.start(sm.timer);
+    const int t = threadIdx.x, B = blockDim.x;
+    const unsigned m = mfk::hw_mask();
+    const int64_t tr0 = a.plan_tr[blockIdx.x], tr1 = a.plan_tr[blockIdx.x + 1];
+    const int64_t R0 = tr0 * 16, Rend = min(tr1 * 16, a.n);
+    const int64_t n = a.n, nr = Rend - R0, nrp = (tr1 - tr0) * 16;
+    const int mu_cap = a.mu_cap;
+    double* __restrict__ X = a.x;
+    double* RP = a.p;                 // r in the PV layout (the SpMV input)
+    double* __restrict__ Pp = a.rh;   // p
+    double* __restrict__ Ss = a.s;    // s
+    double* __restrict__ Wg = a.mu_g;
+    double* __restrict__ Ws = sm.mu;
+    auto w_at = [&](int64_t li) -> double& { return li < mu_cap ? Ws[li] : Wg[R0 + li]; };
+
+    double v2[2] = {0.0, 0.0};
+    bool ok = stage_x0(a, RP, R0, Rend);
+    mfk::spmv_cta<false, false, PF>(a.A, tr0, tr1, RP, 0, sm.sp, 0, nullptr,
+                                    [&](int64_t TR, int ln, double ax, double) {
+                                        const int64_t i = TR * 16 + ln;
+                                        if (i < n) {
+                                            const double bi = a.b[i];
+                                            const double ri = __dsub_rn(bi, ax);
+                                            a.r[i] = ri;
+                                            v2[0] = __fma_rn(bi, bi, v2[0]);
+                                            v2[1] = __fma_rn(ri, ri, v2[1]);
+                                        }
+                                    });
+    ok = grid_reduce<2>(v2, a, c, sm.red) && ok;
+    const double nb = sqrt(v2[0]);
+    double gamma = v2[1], alpha = 0.0, beta = 0.0;
+    int64_t j = 0;
+    int converged = 0, status = ok ? MF_OK : MF_ERR_DEADLOCK;
+    Thresh th{0, 0, 0, 0};
+    if (ok && nb == 0.0) {
+        for (int64_t i = R0 + t; i < Rend; i += B) X[i] = 0.0;
+        converged = 1;
+        if (blockIdx.x == 0 && t == 0 && a.hist_cap > 0) a.hist[0] = 0.0;
+    } else if (ok) {
+        th = make_thresh(a, sqrt(gamma));
+        const double relres0 = __ddiv_rn(sqrt(gamma), nb);
+        bool first = !(relres0 < a.tol) && a.max_iter > 0;
+        if (first) {
+            // r0 -> PV + levels; w0 = A~ r0 with the partial (w0, r0)
+            for (int64_t li = t; li < nrp; li += B) {
+                const int64_t i = R0 + li;
+                const double rv = li < nr ? a.r[i] : 0.0;
+                RP[pv_idx(i)] = rv;
+                int lv = 0;
+                if (DYN) lv = mfk::hw_min_i(li < nr ? mfk::level_of(rv, th) : 4, m);
+                if ((i & 15) == 0) mfk::pv_set_level(RP, i >> 4, lv);
+            }
+            publish(a, 2);
+            if (!wait_deps(a, 2)) status = MF_ERR_DEADLOCK;
+            double d1[1] = {0.0};
+            if (status == MF_OK) {
+                mfk::spmv_cta<DYN, STK, PF>(a.A, tr0, tr1, RP, a.range_guard, sm.sp, 1, nullptr,
+                                            [&](int64_t TR, int ln, double wv, double ov) {
+                                                const int64_t i = TR * 16 + ln;
+                                                if (i < n) { w_at(i - R0) = wv; d1[0] = __fma_rn(wv, ov, d1[0]); }
+                                            });
+                spmv_counts<COUNT, DYN>(a, c, tr0, tr1, RP, sm.ired);
+                if (!grid_reduce<1>(d1, a, c, sm.red)) status = MF_ERR_DEADLOCK;
+            }
+            const double delta = d1[0];
+            if (status == MF_OK && (!(delta > 0.0) || !isfinite(delta))) status = MF_ERR_BREAKDOWN;
+            if (status == MF_OK) alpha = __ddiv_rn(gamma, delta);
+            if (status != MF_OK && blockIdx.x == 0 && t == 0) {
+                if (a.hist_cap > 0) a.hist[0] = relres0;
+                a.out[2] = relres0;
+            }
+        }
+        tm.tick(6);
+        for (; status == MF_OK; ++j) {
+            const double relres = __ddiv_rn(sqrt(gamma), nb);
+            if (blockIdx.x == 0 && t == 0) { if (j < a.hist_cap) a.hist[j] = relres; a.out[2] = relres; }
+            if (relres < a.tol) { converged = 1; break; }
+            if (j == a.max_iter) break;
+            // p = r + beta p ; s = w + beta s ; x += alpha p ; r -= alpha s (own rows), r -> PV +
+            // levels, partial (r, r)
+            double v[2] = {0.0, 0.0};
+            for (int64_t li = t; li < nrp; li += B) {
+                const int64_t i = R0 + li;
+                double rn = 0.0;
+                if (li < nr) {
+                    const double pi = __fma_rn(beta, Pp[i], RP[pv_idx(i)]);
+                    const double si = __fma_rn(beta, Ss[i], w_at(li));
+                    Pp[i] = pi;
+                    Ss[i] = si;
+                    X[i] = __fma_rn(alpha, pi, X[i]);
+                    rn = __fma_rn(-alpha, si, RP[pv_idx(i)]);
+                    RP[pv_idx(i)] = rn;
+                    v[0] = __fma_rn(rn, rn, v[0]);
+                }
+                int lv = 0;
+                if (DYN) lv = mfk::hw_min_i(li < nr ? mfk::level_of(rn, th) : 4, m);
+                if ((i & 15) == 0) mfk::pv_set_level(RP, i >> 4, lv);
+            }
+            publish(a, (unsigned)(j + 3));
+            tm.tick(3);
+            if (!wait_deps(a, (unsigned)(j + 3))) { status = MF_ERR_DEADLOCK; break; }
+            tm.tick(0);
+            mfk::spmv_cta<DYN, STK, PF>(a.A, tr0, tr1, RP, a.range_guard, sm.sp, 1, nullptr,
+                                        [&](int64_t TR, int ln, double wv, double ov) {
+                                            const int64_t i = TR * 16 + ln;
+                                            if (i < n) { w_at(i - R0) = wv; v[1] = __fma_rn(wv, ov, v[1]); }
+                                        });
+            spmv_counts<COUNT, DYN>(a, c, tr0, tr1, RP, sm.ired);
+            tm.tick(1);
+            if (!grid_reduce<2>(v, a, c, sm.red)) { status = MF_ERR_DEADLOCK; break; }
+            tm.tick(2);
+            const double gamma1 = v[0], delta1 = v[1];
+            const double beta1 = __ddiv_rn(gamma1, gamma);
+            const double tq = __ddiv_rn(__dmul_rn(beta1, gamma1), alpha);
+            const double den = __dsub_rn(delta1, tq);
+            if (!(den > 0.0) || !isfinite(den)) {
+                ++j;
+                const double rl = __ddiv_rn(sqrt(gamma1), nb);
+                if (blockIdx.x == 0 && t == 0) { if (j < a.hist_cap) a.hist[j] = rl; a.out[2] = rl; }
+                if (rl < a.tol) converged = 1; else status = MF_ERR_BREAKDOWN;
+                break;
+            }
+            alpha = __ddiv_rn(gamma1, den);
+            beta = beta1;
+            gamma = gamma1;
         }
     }
     if (blockIdx.x == 0 && t == 0) {
@@ -989,6 +1142,8 @@ MF_DECLARE_PICK(pick_pcg_512);
 MF_DECLARE_PICK(pick_pcg_1024);
 MF_DECLARE_PICK(pick_pbicgstab_512);
 MF_DECLARE_PICK(pick_pbicgstab_1024);
+MF_DECLARE_PICK(pick_cgsr_512);
+MF_DECLARE_PICK(pick_cgsr_1024);
 
 #define MF_DEFINE_PICK(NAME, KERNEL, MAXT)                                                        \
     void* NAME(bool dyn, bool count, bool sticky) {                                               \

@@ -484,3 +484,26 @@ def test_full_size_C4_prefix_and_convergence(mf, orc, name):
     full = gfn(Gm, dev(b), M=P, mode=2, max_iter=1000)
     assert full.converged
     assert orc.true_relres(A.rowptr, A.colidx, A.vals, b, full.x.cpu().numpy()) < 1e-9
+
+
+SR_CASES = [("C1-sr", lambda: W.make("C1"), 4, 256, 2), ("C1-sr-G1", lambda: W.make("C1"), 1, 1024, 2),
+            ("C2-32-sr", lambda: W.make("C2", 32), 8, 512, 2), ("C2-32-sr-static", lambda: W.make("C2", 32), 16, 256, 1),
+            ("ragged-sr", lambda: W.poisson2d(33), 3, 64, 2), ("C4spd-sr", lambda: W.make("C4spd", 1 << 12), 6, 256, 2)]
+
+
+@pytest.mark.parametrize("name,make,G,B,mode", SR_CASES, ids=[c[0] for c in SR_CASES])
+def test_single_reduction_cg_parity(mf, orc, name, make, G, B, mode):
+    """Single-reduction CG (one grid reduction per iteration): histories, x and level
+    counts bit-identical to the oracle's orc_cg_single_reduction in kernel order."""
+    A = make()
+    b = W.rhs_ones(A)
+    Gm = mf.TileMatrix.from_host_csr(A, grid_ctas=G, block_threads=B)
+    g, bb, R = Gm.plan()
+    T = oracle_tiles(orc, A)
+    ro = orc.cg_single_reduction(T, b, mode=mode, plan=orc.Plan(g, bb, R), max_iter=3000)
+    rg = mf.cg_solve(Gm, dev(b), mode=mode, max_iter=3000, cg_variant=1, level_counts=mode == 2)
+    assert ro["converged"] and rg.converged and rg.iterations == ro["iterations"]
+    assert np.array_equal(rg.history, ro["history"])
+    assert np.array_equal(rg.x.cpu().numpy(), ro["x"])
+    if mode == 2:
+        assert np.array_equal(rg.level_counts, ro["level_counts"])

@@ -251,3 +251,44 @@ def test_preconditioned_solvers_match_dense(orc, spd):
     assert np.linalg.norm(rp_["x"] - x) / np.linalg.norm(x) < 1e-8
     dyn = fn(T, b, M=M, mode=orc.MODE_DYNAMIC)
     assert dyn["converged"]
+
+
+# ------------------------------------------------------------------ single-reduction CG (f4)
+@pytest.mark.parametrize("n,seed", [(8, 0), (30, 1), (64, 2)])
+def test_cg_single_reduction_matches_dense_solve(orc, n, seed):
+    D = rand_spd(n, seed)
+    A = csr_from_dense(D)
+    b = np.random.default_rng(seed).standard_normal(n)
+    r = orc.cg_single_reduction(tiles(orc, A), b, tol=1e-12, mode=orc.MODE_FP64)
+    assert r["converged"] and r["status"] == 0
+    x = np.linalg.solve(D, b)
+    assert np.linalg.norm(r["x"] - x) / np.linalg.norm(x) < 50 * 1e-10
+
+
+def test_cg_single_reduction_finite_termination(orc):
+    """k distinct eigenvalues: the Krylov method ends in k iterations (exact-arithmetic identity
+    with Alg. 1: same iterates, the recurrences only reorder the dots)."""
+    n, k = 64, 4
+    d = np.repeat(np.array([1.0, 2.0, 5.0, 9.0]), n // k)
+    A = W.CSR(n, n, np.arange(n + 1, dtype=np.int64), np.arange(n, dtype=np.int32), d)
+    r = orc.cg_single_reduction(tiles(orc, A), np.ones(n), tol=1e-12, mode=orc.MODE_FP64)
+    assert r["converged"] and r["iterations"] <= k
+    assert np.allclose(r["x"], 1.0 / d, rtol=1e-11)
+
+
+@pytest.mark.parametrize("name,scale", [("C1", 64), ("C2", 16)])
+def test_cg_single_reduction_tracks_classic_cg(orc, name, scale):
+    """Same Krylov iterates as Alg. 1 up to rounding: residual histories agree to ~1e-6 relative
+    over the first iterations, iteration counts within 2%, same solution (x* = 1)."""
+    A = W.make(name, scale)
+    b = W.rhs_ones(A)
+    T = tiles(orc, A, classify=True)
+    rc = orc.cg(T, b, mode=orc.MODE_FP64)
+    rs = orc.cg_single_reduction(T, b, mode=orc.MODE_FP64)
+    assert rc["converged"] and rs["converged"]
+    assert abs(rs["iterations"] - rc["iterations"]) <= max(2, rc["iterations"] // 50)
+    m = 20
+    assert np.max(np.abs(rs["history"][:m] - rc["history"][:m]) / rc["history"][:m]) < 1e-6
+    assert np.max(np.abs(rs["x"] - 1.0)) < 1e-8
+    dy = orc.cg_single_reduction(T, b, mode=orc.MODE_DYNAMIC)
+    assert dy["converged"] and dy["n_spmv"] == dy["iterations"] + 1
