@@ -4,6 +4,7 @@
 #include <cuda_runtime.h>
 
 #include <mutex>
+#include <unordered_map>
 #include <string>
 
 #include "mf_internal.cuh"
@@ -22,10 +23,18 @@ mf_status fail(mf_status s, const std::string& msg) {
     return s;
 }
 
+// every block remembers which allocator produced it (the hook can change between an allocation
+// and its release: a block is always returned to its own allocator)
+static std::unordered_map<void*, std::pair<void (*)(void*, mf_stream, void*), void*>> g_hooked;
+
 void* dev_alloc(size_t bytes, cudaStream_t s) {
     {
         std::lock_guard<std::mutex> lk(g_alloc_mu);
-        if (g_alloc) return g_alloc(bytes, (mf_stream)s, g_alloc_ctx);
+        if (g_alloc) {
+            void* p = g_alloc(bytes, (mf_stream)s, g_alloc_ctx);
+            if (p) g_hooked[p] = {g_dealloc, g_alloc_ctx};
+            return p;
+        }
     }
     // stream-ordered allocator: keep freed blocks in the device's default pool across
     // synchronisations (release threshold = max) so repeated conversions / solves reuse them
@@ -53,7 +62,13 @@ void dev_free(void* p, cudaStream_t s) {
     if (!p) return;
     {
         std::lock_guard<std::mutex> lk(g_alloc_mu);
-        if (g_dealloc) { g_dealloc(p, (mf_stream)s, g_alloc_ctx); return; }
+        auto it = g_hooked.find(p);
+        if (it != g_hooked.end()) {
+            const auto h = it->second;
+            g_hooked.erase(it);
+            h.first(p, (mf_stream)s, h.second);
+            return;
+        }
     }
     cudaFreeAsync(p, s);
 }

@@ -338,7 +338,9 @@ mf_status run_solve(const TileMatrix& A, bool bicg, const double* b, double* x, 
     if (A.ts) {
         // mu on chip only when the ring still gets >= 3 slots (TMA latency cover)
         const int64_t need_mu = max_rows * 8 * nvec;
-        if (mu_onchip && ring_depth(A, avail - need_mu) >= 3) cap = max_rows;
+        int min_ring = 3;
+        if (const char* ev = getenv("MF_MU_MINRING")) min_ring = std::max(1, atoi(ev));   // tuning knob
+        if (mu_onchip && ring_depth(A, avail - need_mu) >= min_ring) cap = max_rows;
         nst = ring_depth(A, avail - cap * 8 * nvec);
         if (nst < 1) return fail(MF_ERR_UNSUPPORTED, "TMA ring does not fit shared memory");
     } else {

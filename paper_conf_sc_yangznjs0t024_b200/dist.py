@@ -141,6 +141,14 @@ class DistTileMatrix:
         from . import TileMatrix
         return TileMatrix.info(self)
 
+    def export(self, stream=None) -> dict:
+        from . import TileMatrix
+        return TileMatrix.export(self, stream)
+
+    def plan(self):
+        from . import TileMatrix
+        return TileMatrix.plan(self)
+
     def close(self):
         if getattr(self, "_h", None):
             from . import lib

@@ -152,7 +152,7 @@ def test_dist_world1_matches_oracle_and_single_kernel(orc):
             b = W.rhs_ones(A)
             D = dist.DistTileMatrix.from_host_csr(comm, A, 0, A.n_rows)
             assert D.dist_info()["halo_segments"] == 0
-            g, bb, R = mf.TileMatrix.plan(D)
+            g, bb, R = D.plan()
             T = orc.Tiles(A.n_rows, A.n_cols, A.rowptr, A.colidx, A.vals)
             ofn = orc.cg if solver == "cg" else orc.bicgstab
             ro = ofn(T, b, mode=2, plan=orc.Plan(g, bb, R), max_iter=2000)

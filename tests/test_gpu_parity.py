@@ -417,7 +417,8 @@ def test_sptrsv_nonsymmetric_pattern(mf, orc):
     n = 3000
     rows, cols, vals = [], [], []
     for i in range(n):
-        cs = set([i] + [c for c in rng.integers(max(0, i - 40), i, 3)] + [c for c in rng.integers(i, min(n, i + 200), 2)])
+        cs = set([i] + ([int(c) for c in rng.integers(max(0, i - 40), i, 3)] if i > 0 else [])
+                 + [int(c) for c in rng.integers(i, min(n, i + 200), 2)])
         for c in sorted(cs):
             rows.append(i); cols.append(int(c))
             vals.append(8.0 if c == i else float(rng.choice([-1.0, 0.5, -0.25, 1.5])))
