@@ -631,9 +631,10 @@ mf_status dist_solve(const TileMatrix& A, const DistInfo& D, bool bicg, const do
     void* f_mu = dyn ? (bicg ? spmv_fn<true, 2>(B) : spmv_fn<true, 1>(B)) : (bicg ? spmv_fn<false, 2>(B) : spmv_fn<false, 1>(B));
     void* f_th = dyn ? spmv_fn<true, 3>(B) : spmv_fn<false, 3>(B);
     for (void* f : {f_init, f_mu, f_th}) MF_CUDA(cudaFuncSetAttribute(f, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
+    cudaStream_t q = s;   // the stream the iteration is enqueued on (a private one while capturing)
     auto launch_spmv = [&](void* f, const double* in) -> mf_status {
         void* args[] = {&a, (void*)&in};
-        MF_CUDA(cudaLaunchKernel(f, dim3(G), dim3(B), args, smem, s));
+        MF_CUDA(cudaLaunchKernel(f, dim3(G), dim3(B), args, smem, q));
         return MF_OK;
     };
     cudaEvent_t e0, e1;
@@ -656,52 +657,59 @@ mf_status dist_solve(const TileMatrix& A, const DistInfo& D, bool bicg, const do
     MF_CUDA(cudaGetLastError());
     // one iteration, enqueued as a chunk captured in a CUDA graph
     auto one_iter = [&]() -> mf_status {
-        MF_TRY(exchange(D, a.pv, sendbuf, D.nown_seg, a.pv, a.st, s));
+        MF_TRY(exchange(D, a.pv, sendbuf, D.nown_seg, a.pv, a.st, q));
         MF_TRY(launch_spmv(f_mu, a.pv));
-        k_rank_partial<<<1, 32, 0, s>>>(a, bicg ? 2 : 2);
-        MF_TRY(allgather(D, a.part, a.gath, 2, s));
+        k_rank_partial<<<1, 32, 0, q>>>(a, bicg ? 2 : 2);
+        MF_TRY(allgather(D, a.part, a.gath, 2, q));
         if (bicg) {
-            k_bicg_s<<<G, B, 0, s>>>(a);
-            MF_TRY(exchange(D, a.sv, sendbuf, D.nown_seg, a.sv, a.st, s));
+            k_bicg_s<<<G, B, 0, q>>>(a);
+            MF_TRY(exchange(D, a.sv, sendbuf, D.nown_seg, a.sv, a.st, q));
             MF_TRY(launch_spmv(f_th, a.sv));
-            k_rank_partial<<<1, 32, 0, s>>>(a, 2);
-            MF_TRY(allgather(D, a.part, a.gath, 2, s));
-            k_bicg_xr<<<G, B, 0, s>>>(a);
-            k_rank_partial<<<1, 32, 0, s>>>(a, 2);
-            MF_TRY(allgather(D, a.part, a.gath, 2, s));
-            k_bicg_beta<<<1, 1, 0, s>>>(a);
-            k_bicg_p<<<G, B, 0, s>>>(a);
+            k_rank_partial<<<1, 32, 0, q>>>(a, 2);
+            MF_TRY(allgather(D, a.part, a.gath, 2, q));
+            k_bicg_xr<<<G, B, 0, q>>>(a);
+            k_rank_partial<<<1, 32, 0, q>>>(a, 2);
+            MF_TRY(allgather(D, a.part, a.gath, 2, q));
+            k_bicg_beta<<<1, 1, 0, q>>>(a);
+            k_bicg_p<<<G, B, 0, q>>>(a);
         } else {
-            k_cg_alpha<<<1, 1, 0, s>>>(a);
-            k_cg_r<<<G, B, 0, s>>>(a);
-            k_rank_partial<<<1, 32, 0, s>>>(a, 1);
-            MF_TRY(allgather(D, a.part, a.gath, 1, s));
-            k_cg_beta<<<1, 1, 0, s>>>(a);
-            k_cg_xp<<<G, B, 0, s>>>(a);
+            k_cg_alpha<<<1, 1, 0, q>>>(a);
+            k_cg_r<<<G, B, 0, q>>>(a);
+            k_rank_partial<<<1, 32, 0, q>>>(a, 1);
+            MF_TRY(allgather(D, a.part, a.gath, 1, q));
+            k_cg_beta<<<1, 1, 0, q>>>(a);
+            k_cg_xp<<<G, B, 0, q>>>(a);
         }
-        k_cg_stop<<<1, 1, 0, s>>>(a);
-        MF_CUDA(cudaGetLastError());
+        k_cg_stop<<<1, 1, 0, q>>>(a);
+        if (q == s) MF_CUDA(cudaGetLastError());   // while capturing, errors surface at instantiation
         return MF_OK;
     };
     constexpr int CHUNK = 8;
     cudaGraph_t graph = nullptr;
     cudaGraphExec_t gexec = nullptr;
     bool graphed = getenv("MF_DIST_NO_GRAPH") == nullptr;
+    // the chunk is captured on a private stream (the caller's may be the legacy stream, which
+    // cannot capture) and launched on the caller's stream
+    cudaStream_t cap = nullptr;
+    if (graphed && cudaStreamCreateWithFlags(&cap, cudaStreamNonBlocking) != cudaSuccess) graphed = false;
     if (graphed) {
-        if (cudaStreamBeginCapture(s, cudaStreamCaptureModeThreadLocal) != cudaSuccess) graphed = false;
+        if (cudaStreamBeginCapture(cap, cudaStreamCaptureModeRelaxed) != cudaSuccess) graphed = false;
         else {
+            q = cap;
             mf_status cs = MF_OK;
             for (int c = 0; c < CHUNK && cs == MF_OK; ++c) cs = one_iter();
-            const cudaError_t ce = cudaStreamEndCapture(s, &graph);
+            q = s;
+            const cudaError_t ce = cudaStreamEndCapture(cap, &graph);
             if (cs != MF_OK || ce != cudaSuccess || cudaGraphInstantiate(&gexec, graph, 0) != cudaSuccess) {
-                cudaGetLastError();
                 if (graph) cudaGraphDestroy(graph);
                 graph = nullptr;
                 gexec = nullptr;
                 graphed = false;
             }
         }
+        cudaGetLastError();   // a refused capture leaves its error behind; the fallback is the eager chunk
     }
+    if (cap) cudaStreamDestroy(cap);
     int hst[4] = {0, 0, 0, 0};
     int* pin = nullptr;
     MF_CUDA(cudaMallocHost(&pin, 4 * sizeof(int)));

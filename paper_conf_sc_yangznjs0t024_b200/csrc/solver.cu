@@ -338,7 +338,9 @@ mf_status run_solve(const TileMatrix& A, bool bicg, const double* b, double* x, 
     if (A.ts) {
         // mu on chip only when the ring still gets >= 3 slots (TMA latency cover)
         const int64_t need_mu = max_rows * 8 * nvec;
-        int min_ring = 3;
+        // a 2-deep TMA ring already hides the stage loads once mu stays on chip (r02 sweep on C2:
+        // ring 2 + mu on chip 73.0 us/it, ring 5 + mu in HBM 74.6)
+        int min_ring = 2;
         if (const char* ev = getenv("MF_MU_MINRING")) min_ring = std::max(1, atoi(ev));   // tuning knob
         if (mu_onchip && ring_depth(A, avail - need_mu) >= min_ring) cap = max_rows;
         nst = ring_depth(A, avail - cap * 8 * nvec);

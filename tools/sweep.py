@@ -19,8 +19,9 @@ for (G, B), lay in [(sh, l) for sh in shapes for l in layouts]:
     for mode in (mf.MODE_DYNAMIC, mf.MODE_STATIC):
         try:
             T = mf.TileMatrix(A.n_rows, A.n_cols, rp, ci, va, grid_ctas=G, block_threads=B, layout=lay)
-            st = fn(T, b, max_iter=max_iter, mode=mode, collect_stats=True, history=False, raise_on_breakdown=False)
-            r = fn(T, b, max_iter=max_iter, mode=mode, history=False, raise_on_breakdown=False)
+            kw = dict(cg_variant=int(os.environ.get("CGV", "0"))) if fn is mf.cg_solve else {}
+            st = fn(T, b, max_iter=max_iter, mode=mode, collect_stats=True, history=False, raise_on_breakdown=False, **kw)
+            r = fn(T, b, max_iter=max_iter, mode=mode, history=False, raise_on_breakdown=False, **kw)
         except mf.MFError as e:
             print(G, B, "error", e); continue
         it = max(r.iterations, 1)
