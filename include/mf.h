@@ -133,6 +133,12 @@ typedef struct {
     int32_t cg_variant;         /* mf_cg_solve: 0 (default) Alg. 1 (two grid reductions per iteration);
                                    1 single-reduction CG (Chronopoulos-Gear; one reduction, the dynamic
                                    switch watching r, the SpMV input of that variant) */
+    int32_t dist_mode;          /* *_solve_dist only: 0 (default) auto = the device-initiated single kernel
+                                   for CG (2 below), the host-orchestrated path for BiCGSTAB; 1 host-
+                                   orchestrated kernels + NCCL between them; 2 device-
+                                   initiated: ONE persistent kernel per rank that stores the halo
+                                   into the peers' windows over NVLink and reduces across ranks
+                                   itself (Finding 2, across GPUs) */
 } mf_solve_opts;
 
 typedef struct {
@@ -187,20 +193,26 @@ mf_status mf_cg_solve(const mf_tile_matrix* A, const double* b, double* x, const
 mf_status mf_bicgstab_solve(const mf_tile_matrix* A, const double* b, double* x, const mf_solve_opts* opts,
                             mf_solve_info* info, mf_stream stream);
 
-/* ---------------------------------------------------------------- multi-GPU (row blocks, SURVEY 8(b), 8(e))
+/* ---------------------------------------------------------------- multi-GPU (row blocks, SURVEY 8(b), 8(e), 8(f) f1)
  * The paper's solver is single-GPU; the build partitions matrices too large for one GPU
  * (BASELINE configs[4]) into contiguous blocks of whole 16-row tile rows, one block per GPU, one
- * process per GPU.  Communication is NCCL (over NVLink) inside libmf: the caller only ships the
- * 128-byte unique id from rank 0 to the other ranks (e.g. with torch.distributed).
+ * process per GPU.  Communication is inside libmf (NCCL communicator, NVLink): the caller only
+ * ships the 128-byte unique id from rank 0 to the other ranks (e.g. with torch.distributed).
  *
  * Rank k owns rows [row_begin, row_end) (row_begin a multiple of 16; the blocks of all ranks are
  * contiguous, in rank order, and cover the matrix).  It converts its rows as a local tile matrix
- * whose columns are its own 16-element segments followed by the halo segments its rows gather
- * (one-to-one with global segments: tiles, TilePrec and the dynamic levels of Alg. 4 are the
- * global matrix's).  Per iteration: halo exchange of the SpMV input (ncclSend / ncclRecv per
- * peer), the staged tile SpMV, rank partials of every dot (the launch plan's tree) all-gathered
- * and summed in rank order from +0 on every rank (deterministic; one rank == mf_cg_solve bit for
- * bit), every scalar on the device, iterations enqueued as CUDA graphs with a device stop flag.
+ * whose columns are [the halo segments of lower ranks | its own segments | the halo segments of
+ * higher ranks], each part ascending: one-to-one with global segments and in global order, so
+ * tiles, TilePrec, the dynamic levels of Alg. 4 AND every row's fma order are the global
+ * matrix's.  Every dot is the sum, in rank order from +0, of the rank partials (each the launch
+ * plan's tree over the rank's CTAs): identical on every rank, deterministic, and equal to the
+ * oracle's rank-partitioned plan.  Two executions (mf_solve_opts.dist_mode):
+ *  - device-initiated (CG default): one cooperative persistent kernel per rank; producers store
+ *    their boundary segments into the peers' windows (NCCL symmetric windows, peer pointers from
+ *    the NCCL device API) and count arrivals with system-scope release adds; rank partials are
+ *    stored, tagged, into every rank's window; no host involvement per iteration;
+ *  - host-orchestrated: the same steps as separate kernels with ncclSend/Recv and ncclAllGather
+ *    between them, iterations enqueued as CUDA graphs with a device stop flag.
  * All calls are collective over the communicator's ranks. */
 typedef struct mf_comm mf_comm;
 /* host: 128 bytes (ncclUniqueId), created on rank 0 and broadcast to the others by the caller */
@@ -208,6 +220,15 @@ mf_status mf_nccl_unique_id(void* out);
 mf_status mf_comm_create(const void* nccl_unique_id, int32_t nranks, int32_t rank, mf_comm** out);
 mf_status mf_comm_destroy(mf_comm* comm);
 mf_status mf_comm_info(const mf_comm* comm, int32_t* nranks, int32_t* rank);
+/* In-process rank group: nranks host threads of ONE process each drive one rank, all ranks on the
+ * current device (their windows are same-device buffers).  Runs the device-initiated kernel only
+ * (each rank's thread must use its own stream; the kernels run concurrently, so the plan's CTAs of
+ * all ranks must fit the device together: convert with grid_ctas <= SMs / nranks).  Verifies the
+ * multi-rank exchange on a single GPU.  The group outlives its comms. */
+typedef struct mf_local_group mf_local_group;
+mf_status mf_local_group_create(int32_t nranks, mf_local_group** out);
+mf_status mf_local_group_destroy(mf_local_group* g);
+mf_status mf_comm_create_local(mf_local_group* g, int32_t rank, mf_comm** out);
 /* rowptr int64[row_end-row_begin+1] (local, from 0), colidx int32[nnz_local] GLOBAL columns
  * (strictly increasing per row), vals f64[nnz_local]; device pointers.  The handle is freed with
  * mf_tile_matrix_destroy; mf_tile_matrix_info / export describe the LOCAL matrix. */

@@ -54,7 +54,8 @@ class _Tiles(C.Structure):
 
 
 class _Plan(C.Structure):
-    _fields_ = [("G", C.c_int32), ("B", C.c_int32), ("R", C.POINTER(C.c_int64))]
+    _fields_ = [("G", C.c_int32), ("B", C.c_int32), ("R", C.POINTER(C.c_int64)), ("P", C.c_int32),
+                ("Gr", C.POINTER(C.c_int32))]
 
 
 class _Opts(C.Structure):
@@ -309,10 +310,17 @@ def spmv_csr(rowptr, colidx, vals, x):
 class Plan:
     """Kernel-order reduction plan (SURVEY c-7): G CTAs, B threads, CTA g owns rows [R[g], R[g+1])."""
 
-    def __init__(self, G, B, R):
+    def __init__(self, G, B, R, rank_ctas=None):
+        """rank_ctas: CTA boundaries [0, G_0, G_0 + G_1, ..., G] of row-block ranks (each rank's
+        CTAs own its rows): rank partials, summed in rank order from +0 (mf_oracle.c section 6)."""
         self.R = np.ascontiguousarray(R, np.int64)
         assert len(self.R) == G + 1 and B % 32 == 0
-        self._s = _Plan(G, B, self.R.ctypes.data_as(C.POINTER(C.c_int64)))
+        self.Gr = None if rank_ctas is None else np.ascontiguousarray(rank_ctas, np.int32)
+        if self.Gr is not None:
+            assert self.Gr[0] == 0 and self.Gr[-1] == G and np.all(np.diff(self.Gr) >= 0)
+        P = 0 if self.Gr is None else len(self.Gr) - 1
+        gr = None if self.Gr is None else self.Gr.ctypes.data_as(C.POINTER(C.c_int32))
+        self._s = _Plan(G, B, self.R.ctypes.data_as(C.POINTER(C.c_int64)), P, gr)
         self.G, self.B = G, B
 
 

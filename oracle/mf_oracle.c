@@ -467,8 +467,12 @@ void orc_spmv_csr(int64_t n, const int64_t* rowptr, const int32_t* colidx, const
  *      CTA:      tree32 over the W = B/32 warp totals
  *      grid:     tree32 over the G CTA totals
  *    tree32(x[0..c)): lane l sums x[l], x[l+32], ... left to right from +0, then butterfly.
+ *    Row-block ranks (P > 0, the rows of rank q are those of CTAs [Gr[q], Gr[q+1])):
+ *      rank q:   tree32 over its CTA totals (the grid level of q's own launch)
+ *      total:    ((+0 + rank_0) + rank_1) + ... in rank order
+ *    (again a reading: the paper is single-GPU.)
  * ---------------------------------------------------------------------------------- */
-typedef struct { int32_t G; int32_t B; const int64_t* R; } orc_plan;
+typedef struct { int32_t G; int32_t B; const int64_t* R; int32_t P; const int32_t* Gr; } orc_plan;
 
 static double butterfly32(double* v) {
     double nv[32];
@@ -510,7 +514,13 @@ double orc_dot(const double* u, const double* v, int64_t n, const orc_plan* plan
         }
         slot[g] = tree32(wt, W);
     }
-    double r = tree32(slot, plan->G);
+    double r;
+    if (plan->P > 0) {
+        r = 0.0;
+        for (int32_t q = 0; q < plan->P; ++q) r = r + tree32(slot + plan->Gr[q], plan->Gr[q + 1] - plan->Gr[q]);
+    } else {
+        r = tree32(slot, plan->G);
+    }
     free(slot); free(wt);
     return r;
 }

@@ -35,7 +35,8 @@ SYMBOLS = ["mf_default_convert_opts", "mf_default_solve_opts", "mf_set_allocator
            "mf_dot", "mf_precond_create", "mf_precond_destroy", "mf_precond_apply", "mf_cg_solve",
            "mf_bicgstab_solve", "mf_cg_update_xr", "mf_cg_update_p", "mf_status_string", "mf_last_error",
            "mf_abi_version", "mf_nccl_unique_id", "mf_comm_create", "mf_comm_destroy", "mf_comm_info",
-           "mf_tile_matrix_from_csr_dist", "mf_cg_solve_dist", "mf_bicgstab_solve_dist", "mf_dist_info", "mf_dist_plan"]
+           "mf_tile_matrix_from_csr_dist", "mf_cg_solve_dist", "mf_bicgstab_solve_dist", "mf_dist_info", "mf_dist_plan",
+           "mf_local_group_create", "mf_local_group_destroy", "mf_comm_create_local"]
 
 NVCC_FLAGS = ["-gencode", "arch=compute_100a,code=sm_100a", "-O3", "-lineinfo", "-std=c++17", "-fmad=false",
               "-Xcompiler", "-fPIC"]
@@ -108,7 +109,7 @@ class SolveOpts(C.Structure):
                 ("switch_absolute", C.c_int32), ("sticky", C.c_int32), ("range_guard", C.c_int32),
                 ("M", C.c_void_p), ("residual_history", C.c_void_p), ("history_cap", C.c_int64),
                 ("tile_level_counts", C.c_void_p), ("level_counts_cap", C.c_int64), ("collect_stats", C.c_int32),
-                ("watchdog_ms", C.c_int32), ("cg_variant", C.c_int32)]
+                ("watchdog_ms", C.c_int32), ("cg_variant", C.c_int32), ("dist_mode", C.c_int32)]
 
 
 class SolveInfo(C.Structure):
@@ -166,6 +167,9 @@ def lib():
         L.mf_bicgstab_solve_dist.argtypes = [vp, vp, vp, C.POINTER(SolveOpts), C.POINTER(SolveInfo), vp]
         L.mf_dist_info.argtypes = [vp, C.POINTER(i64), C.POINTER(i64), C.POINTER(i64), C.POINTER(i64)]
         L.mf_dist_plan.argtypes = [i64, i32, vp, i32, i64, vp, vp, vp, i64, C.POINTER(i64)]
+        L.mf_local_group_create.argtypes = [i32, C.POINTER(vp)]
+        L.mf_local_group_destroy.argtypes = [vp]
+        L.mf_comm_create_local.argtypes = [vp, i32, C.POINTER(vp)]
         _lib = L
         return L
 
@@ -346,7 +350,7 @@ class SolveResult:
 def _solve(fn, A: TileMatrix, b, x0=None, tol=1e-10, max_iter=1000, mode=MODE_DYNAMIC, switch_eps=None,
            switch_absolute=False, range_guard=True, sticky=False, history=True, level_counts=False,
            collect_stats=False, M=None, stream=None, raise_on_breakdown=True, watchdog_ms=0,
-           cg_variant=0) -> SolveResult:
+           cg_variant=0, dist_mode=0) -> SolveResult:
     import torch
     _need_cuda(b, torch.float64, "b")
     x = torch.zeros_like(b) if x0 is None else x0.clone()
@@ -365,6 +369,7 @@ def _solve(fn, A: TileMatrix, b, x0=None, tol=1e-10, max_iter=1000, mode=MODE_DY
     o.collect_stats = int(collect_stats)
     o.watchdog_ms = int(watchdog_ms)
     o.cg_variant = int(cg_variant)
+    o.dist_mode = int(dist_mode)
     info = SolveInfo()
     st = fn(A._h, _ptr(b), _ptr(x), C.byref(o), C.byref(info), _stream_ptr(stream))
     if st != 0 and (raise_on_breakdown or st != 7):

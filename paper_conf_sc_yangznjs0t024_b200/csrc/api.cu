@@ -142,6 +142,7 @@ void mf_default_solve_opts(mf_solve_opts* o) {
     o->collect_stats = 0;
     o->watchdog_ms = 0;
     o->cg_variant = 0;
+    o->dist_mode = 0;
 }
 
 mf_status mf_set_allocator(void* (*alloc)(size_t, mf_stream, void*), void (*dealloc)(void*, mf_stream, void*),

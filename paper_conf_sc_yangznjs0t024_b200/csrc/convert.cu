@@ -374,8 +374,8 @@ __device__ int owner_of(const int32_t* plan_tr, int G, int64_t TR) {   // CTA ow
 
 // dependency range: CTAs owning the column segments this CTA's tiles gather (square matrices)
 __global__ void deps_kernel(const int32_t* __restrict__ plan_tr, int G, const int64_t* __restrict__ TileRowPtr,
-                            const int32_t* __restrict__ TileColidx, int64_t n_seg_owned, int32_t* dep_lo, int32_t* dep_hi,
-                            int32_t* seg_lo, int32_t* seg_hi) {
+                            const int32_t* __restrict__ TileColidx, int64_t n_seg_owned, int64_t coff, int32_t* dep_lo,
+                            int32_t* dep_hi, int32_t* seg_lo, int32_t* seg_hi) {
     int g = blockIdx.x;
     __shared__ int smin, smax;
     if (threadIdx.x == 0) { smin = INT32_MAX; smax = -1; }
@@ -391,10 +391,13 @@ __global__ void deps_kernel(const int32_t* __restrict__ plan_tr, int G, const in
     if (threadIdx.x == 0) {
         int lo = g, hi = g;
         if (smax >= 0) {
-            // column segments beyond the owned row range (non-square / halo) have no owner CTA
-            int64_t cmin = smin, cmax = smax < n_seg_owned ? smax : n_seg_owned - 1;
-            if (cmin < n_seg_owned) lo = min(lo, owner_of(plan_tr, G, cmin));
-            if (cmax >= 0 && cmin < n_seg_owned) hi = max(hi, owner_of(plan_tr, G, cmax));
+            // column segments outside the owned ones [coff, coff + n_seg_owned) (non-square / halo)
+            // have no owner CTA
+            const int64_t cmin = max((int64_t)smin, coff) - coff, cmax = min((int64_t)smax - coff, n_seg_owned - 1);
+            if (cmin <= cmax) {
+                lo = min(lo, owner_of(plan_tr, G, cmin));
+                hi = max(hi, owner_of(plan_tr, G, cmax));
+            }
         }
         dep_lo[g] = lo;
         dep_hi[g] = hi;
@@ -548,7 +551,7 @@ __global__ void __launch_bounds__(mfk::TS_CCAP) blob_fill_kernel(mfk::TsStage* s
                                                                    const uint2* __restrict__ crec,
                                                                    const uint8_t* __restrict__ vstream, uint8_t* blob,
                                                                    const int32_t* __restrict__ plan_tr, int G, int H,
-                                                                   unsigned long long* maxb) {
+                                                                   int64_t coff, unsigned long long* maxb) {
     __shared__ int32_t hdr[mfk::TS_KCAP + 1];
     __shared__ int16_t cw[mfk::TS_KCAP];                 // warp of each tile row
     __shared__ uint8_t cq[mfk::TS_CCAP];                 // TilePrec of each column
@@ -587,10 +590,12 @@ __global__ void __launch_bounds__(mfk::TS_CCAP) blob_fill_kernel(mfk::TsStage* s
     }
     __syncthreads();
     if (c == 0) {
-        // own window segment: tile column tr0 if [tr0, tr1) lies inside one run, else -1
+        // own window segment: column segment tr0 + coff if the stage's own segments lie inside one
+        // run, else -1
         int own = -1;
+        const int64_t oc0 = st.tr0 + coff, oc1 = st.tr1 + coff;
         for (int i = 0; i < st.nrun; ++i)
-            if (st.run_s[i] <= st.tr0 && st.tr1 <= st.run_s[i] + st.run_n[i]) own = st.run_w[i] + (st.tr0 - st.run_s[i]);
+            if (st.run_s[i] <= oc0 && oc1 <= (int64_t)st.run_s[i] + st.run_n[i]) own = st.run_w[i] + (int)(oc0 - st.run_s[i]);
         int32_t* h = reinterpret_cast<int32_t*>(b);
         h[0] = st.tr0; h[1] = st.tr1; h[2] = nc; h[3] = L.off_desc; h[4] = 0; h[5] = L.off_val; h[6] = own;
         h[7] = (int32_t)(uint32_t)(uint64_t)col0; h[8] = (int32_t)(uint32_t)((uint64_t)col0 >> 32);
@@ -832,7 +837,7 @@ mf_status convert_csr(int64_t n_rows, int64_t n_cols, int64_t nnz, const int64_t
     MF_TRY(alloc(&A->seg_lo, G, s));
     MF_TRY(alloc(&A->seg_hi, G, s));
     plan_kernel<<<(G + 1 + 127) / 128, 128, 0, s>>>(off, ntr, G, A->plan_tr);
-    deps_kernel<<<G, 256, 0, s>>>(A->plan_tr, G, A->TileRowPtr, A->TileColidx, ntr, A->dep_lo, A->dep_hi, A->seg_lo,
+    deps_kernel<<<G, 256, 0, s>>>(A->plan_tr, G, A->TileRowPtr, A->TileColidx, ntr, A->coff, A->dep_lo, A->dep_hi, A->seg_lo,
                                   A->seg_hi);
     MF_CUDA(cudaGetLastError());
     bool ts_failed = false;
@@ -890,7 +895,7 @@ mf_status convert_csr(int64_t n_rows, int64_t n_cols, int64_t nnz, const int64_t
             MF_CUDA(cudaStreamSynchronize(s));
             MF_TRY(alloc(&A->blob, A->blob_bytes + 64, s));
             blob_fill_kernel<<<(unsigned)A->nstg, mfk::TS_CCAP, 0, s>>>(static_cast<mfk::TsStage*>(A->stg), boff, A->tr_slot, A->tr_vb, A->crec,
-                                                                       A->vstream, A->blob, A->plan_tr, G, B / 16, dmax + 1);
+                                                                       A->vstream, A->blob, A->plan_tr, G, B / 16, A->coff, dmax + 1);
             MF_CUDA(cudaGetLastError());
             unsigned long long mb[2] = {0, 0};
             MF_CUDA(cudaMemcpyAsync(mb, dmax + 1, sizeof(mb), cudaMemcpyDeviceToHost, s));
@@ -915,7 +920,9 @@ mf_status convert_csr(int64_t n_rows, int64_t n_cols, int64_t nnz, const int64_t
         cudaEventDestroy(e0);
         cudaEventDestroy(e1);
         dev_free(cost, s); dev_free(cnt, s); dev_free(off, s); dev_free(tmp, s); dev_free(d_err, s);
+        const int64_t coff = A->coff;
         destroy_tiles(A);
+        A->coff = coff;
         mf_convert_opts o2 = o;
         o2.layout = 1;
         return convert_csr(n_rows, n_cols, nnz, rowptr, colidx, vals, o2, s, A);

@@ -27,7 +27,11 @@
 #include <cstring>
 #include <vector>
 
+#include <chrono>
+#include <condition_variable>
 #include <memory>
+#include <mutex>
+#include <nccl_device.h>
 
 #include "kernels.cuh"
 #include "mf_internal.cuh"
@@ -40,9 +44,11 @@ namespace mf {
         if (r_ != ncclSuccess) return ::mf::fail(MF_ERR_NCCL, std::string(#call) + ": " + ncclGetErrorString(r_)); \
     } while (0)
 
+struct LocalGroup;
 struct Comm {
     ncclComm_t nccl = nullptr;
     int nranks = 0, rank = 0;
+    LocalGroup* local = nullptr;     // in-process rank group (ranks emulated on one device)
 };
 
 namespace {
@@ -419,15 +425,61 @@ struct DistWs {
 }  // namespace
 
 // ------------------------------------------------------------------------------------ host
+// In-process rank group: P host threads of one process drive P ranks emulated on ONE device
+// (same-device windows instead of NVLink peers).  Only the device-initiated kernel runs on it;
+// it verifies the multi-rank exchange logic where only one GPU is available.
+struct LocalGroup {
+    int P = 0;
+    std::mutex mu;
+    std::condition_variable cv;
+    int arrived = 0;
+    uint64_t gen = 0;
+    std::vector<std::vector<char>> slot;                 // [rank] all-gather payloads
+    std::vector<std::vector<std::vector<int32_t>>> mail; // [src][dst] exchange payloads
+    bool barrier() {
+        std::unique_lock<std::mutex> lk(mu);
+        const uint64_t g = gen;
+        if (++arrived == P) {
+            arrived = 0;
+            ++gen;
+            cv.notify_all();
+            return true;
+        }
+        return cv.wait_for(lk, std::chrono::seconds(300), [&] { return gen != g; });
+    }
+};
+
 struct DistInfo {
     Comm* comm = nullptr;
     int64_t n_global = 0, row_begin = 0, row_end = 0, nown_seg = 0, nhalo = 0;
+    int64_t nlo = 0;                         // halo segments of lower ranks (they precede the own ones)
     std::vector<int64_t> rank_rows;          // [P + 1] row boundaries of every rank
     std::vector<int64_t> recv_off;           // [P + 1] halo segments per peer (prefix)
     std::vector<int64_t> send_off;           // [P + 1] my segments each peer needs (prefix)
     int32_t* send_idx = nullptr;             // device: my local segment ids, per peer
+    // device-initiated kernel (f1)
+    MgArgs mg{};                             // everything but seg_lo / seg_hi (from the tile matrix)
+    char* win = nullptr;                     // my window
+    size_t win_bytes = 0;
+    bool win_nccl = false;                   // ncclMemAlloc + registered window
+    ncclWindow_t nwin = nullptr;
+    void* dev_arrays = nullptr;              // send lists (one allocation)
+    int* bar_scratch = nullptr;              // stream-ordered cross-rank barrier (ncclAllReduce)
     cudaStream_t owner = nullptr;
-    ~DistInfo() { if (send_idx) dev_free(send_idx, owner); }
+    ~DistInfo() {
+        if (send_idx) dev_free(send_idx, owner);
+        if (dev_arrays) dev_free(dev_arrays, owner);
+        if (bar_scratch) dev_free(bar_scratch, owner);
+        if (win) {
+            if (win_nccl) {
+                cudaStreamSynchronize(owner);
+                if (nwin) ncclCommWindowDeregister(comm->nccl, nwin);
+                ncclMemFree(win);
+            } else {
+                dev_free(win, owner);
+            }
+        }
+    }
 };
 
 namespace {
@@ -442,17 +494,32 @@ __global__ void k_halo_list(const int64_t* __restrict__ flag, const int64_t* __r
     for (int64_t g = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; g < nseg; g += (int64_t)gridDim.x * blockDim.x)
         if (flag[g]) list[pre[g]] = (int32_t)g;
 }
+// Local columns that keep the global order: [halo of lower ranks][own][halo of higher ranks],
+// each part ascending by global segment.  A row's fma chain then visits its tiles in the same
+// order as on one GPU, so every rank's SpMV rows equal the global SpMV rows bit for bit.
 __global__ void k_remap(const int32_t* __restrict__ colidx, int64_t nnz, int64_t row_begin, int64_t seg_lo, int64_t seg_hi,
-                        int64_t nown_seg, const int64_t* __restrict__ pre, int32_t* out) {
+                        int64_t nown_seg, int64_t nlo, const int64_t* __restrict__ pre, int32_t* out) {
     for (int64_t k = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; k < nnz; k += (int64_t)gridDim.x * blockDim.x) {
         const int64_t c = colidx[k], sgm = c >> 4;
-        out[k] = (sgm >= seg_lo && sgm < seg_hi) ? (int32_t)(c - row_begin)
-                                                 : (int32_t)((nown_seg + pre[sgm]) * 16 + (c & 15));
+        int64_t o;
+        if (sgm >= seg_lo && sgm < seg_hi) o = c - row_begin + nlo * 16;
+        else {
+            const int64_t h = pre[sgm];
+            o = (h < nlo ? h : nown_seg + h) * 16 + (c & 15);
+        }
+        out[k] = (int32_t)o;
     }
 }
+__global__ void k_peer_ptrs(ncclWindow_t w, int P, unsigned long long* out) {
+    if ((int)threadIdx.x < P) out[threadIdx.x] = (unsigned long long)ncclGetPeerPointer(w, 0, (int)threadIdx.x);
+}
 
-mf_status exchange(const DistInfo& D, const double* pv, double* sendbuf, int64_t nown_seg, double* pv_ext, const int* st,
-                   cudaStream_t s) {
+// extended segment of a halo block received from rank q (order-preserving layout)
+inline int64_t halo_base(const DistInfo& D, int q) {
+    return q < D.comm->rank ? D.recv_off[q] : D.nown_seg + D.recv_off[q];
+}
+
+mf_status exchange(const DistInfo& D, const double* pv, double* sendbuf, double* pv_own, const int* st, cudaStream_t s) {
     const int P = D.comm->nranks;
     const int64_t nsend = D.send_off[P];
     if (nsend > 0) {
@@ -460,12 +527,13 @@ mf_status exchange(const DistInfo& D, const double* pv, double* sendbuf, int64_t
         k_pack<<<blocks, 256, 0, s>>>(pv, D.send_idx, nsend, sendbuf, st);
         MF_CUDA(cudaGetLastError());
     }
+    double* ext = pv_own - D.nlo * PVS;
     MF_NCCL(ncclGroupStart());
     for (int q = 0; q < P; ++q) {
         if (q == D.comm->rank) continue;
         const int64_t ns = D.send_off[q + 1] - D.send_off[q], nr = D.recv_off[q + 1] - D.recv_off[q];
         if (ns) MF_NCCL(ncclSend(sendbuf + D.send_off[q] * PVS, (size_t)(ns * PVS), ncclDouble, q, D.comm->nccl, s));
-        if (nr) MF_NCCL(ncclRecv(pv_ext + (nown_seg + D.recv_off[q]) * PVS, (size_t)(nr * PVS), ncclDouble, q, D.comm->nccl, s));
+        if (nr) MF_NCCL(ncclRecv(ext + halo_base(D, q) * PVS, (size_t)(nr * PVS), ncclDouble, q, D.comm->nccl, s));
     }
     MF_NCCL(ncclGroupEnd());
     return MF_OK;
@@ -473,6 +541,183 @@ mf_status exchange(const DistInfo& D, const double* pv, double* sendbuf, int64_t
 
 mf_status allgather(const DistInfo& D, const double* part, double* gath, int k, cudaStream_t s) {
     MF_NCCL(ncclAllGather(part, gath, (size_t)k, ncclDouble, D.comm->nccl, s));
+    return MF_OK;
+}
+
+// ---- setup collectives over either backend (host buffers, synchronous)
+mf_status comm_allgather(Comm* c, const void* mine, size_t bytes, void* all, cudaStream_t s) {
+    const int P = c->nranks;
+    if (c->local) {
+        LocalGroup& g = *c->local;
+        g.slot[c->rank].assign((const char*)mine, (const char*)mine + bytes);
+        if (!g.barrier()) return fail(MF_ERR_DEADLOCK, "local rank group: barrier timed out");
+        for (int q = 0; q < P; ++q) std::memcpy((char*)all + q * bytes, g.slot[q].data(), bytes);
+        if (!g.barrier()) return fail(MF_ERR_DEADLOCK, "local rank group: barrier timed out");
+        return MF_OK;
+    }
+    char *d_in = nullptr, *d_all = nullptr;
+    DistWs ws(s);
+    MF_TRY(ws.get(&d_in, bytes));
+    MF_TRY(ws.get(&d_all, bytes * P));
+    MF_CUDA(cudaMemcpyAsync(d_in, mine, bytes, cudaMemcpyHostToDevice, s));
+    MF_NCCL(ncclAllGather(d_in, d_all, bytes, ncclChar, c->nccl, s));
+    MF_CUDA(cudaMemcpyAsync(all, d_all, bytes * P, cudaMemcpyDeviceToHost, s));
+    MF_CUDA(cudaStreamSynchronize(s));
+    return MF_OK;
+}
+// to[q] -> rank q; from[q] (pre-sized by the caller) <- rank q
+mf_status comm_exchange_i32(Comm* c, const std::vector<std::vector<int32_t>>& to, std::vector<std::vector<int32_t>>& from,
+                            cudaStream_t s) {
+    const int P = c->nranks, me = c->rank;
+    if (c->local) {
+        LocalGroup& g = *c->local;
+        for (int q = 0; q < P; ++q) g.mail[me][q] = to[q];
+        if (!g.barrier()) return fail(MF_ERR_DEADLOCK, "local rank group: barrier timed out");
+        for (int q = 0; q < P; ++q) from[q] = g.mail[q][me];
+        if (!g.barrier()) return fail(MF_ERR_DEADLOCK, "local rank group: barrier timed out");
+        return MF_OK;
+    }
+    size_t nt = 0, nf = 0;
+    for (int q = 0; q < P; ++q) { nt += to[q].size(); nf += from[q].size(); }
+    int32_t *dt = nullptr, *df = nullptr;
+    DistWs ws(s);
+    MF_TRY(ws.get(&dt, nt));
+    MF_TRY(ws.get(&df, nf));
+    size_t o = 0;
+    for (int q = 0; q < P; ++q) {
+        if (!to[q].empty()) MF_CUDA(cudaMemcpyAsync(dt + o, to[q].data(), to[q].size() * 4, cudaMemcpyHostToDevice, s));
+        o += to[q].size();
+    }
+    MF_NCCL(ncclGroupStart());
+    size_t ot = 0, of = 0;
+    for (int q = 0; q < P; ++q) {
+        if (q != me && !to[q].empty()) MF_NCCL(ncclSend(dt + ot, to[q].size(), ncclInt32, q, c->nccl, s));
+        if (q != me && !from[q].empty()) MF_NCCL(ncclRecv(df + of, from[q].size(), ncclInt32, q, c->nccl, s));
+        ot += to[q].size();
+        of += from[q].size();
+    }
+    MF_NCCL(ncclGroupEnd());
+    of = 0;
+    for (int q = 0; q < P; ++q) {
+        if (q != me && !from[q].empty()) MF_CUDA(cudaMemcpyAsync(from[q].data(), df + of, from[q].size() * 4, cudaMemcpyDeviceToHost, s));
+        of += from[q].size();
+    }
+    MF_CUDA(cudaStreamSynchronize(s));
+    return MF_OK;
+}
+
+// window layout (bytes): tags u32 [2][P] | counters u64 [P] | reduction slots f64 [2][P][4] | PV
+constexpr int64_t WIN_TAG = 0, WIN_CNT = 64, WIN_RED = 128, WIN_PV = 1024;
+
+// f1 setup: the CTA-ordered store lists, the arrival counts, my halo ranges, the windows
+mf_status mg_setup(DistInfo& D, const TileMatrix& A, const std::vector<int32_t>& req_local, cudaStream_t s) {
+    Comm* c = D.comm;
+    const int P = c->nranks, me = c->rank;
+    if (P > MG_PMAX) return MF_OK;           // only the host-orchestrated path (dist_mode 1)
+    MgArgs& m = D.mg;
+    m.P = P;
+    m.me = me;
+    // my base in every rank's extended vector (all-gathered P x P: row q = rank q's bases)
+    std::vector<int64_t> base(P, 0), base_all((size_t)P * P);
+    for (int r = 0; r < P; ++r) base[r] = r == me ? 0 : halo_base(D, r);
+    MF_TRY(comm_allgather(c, base.data(), P * sizeof(int64_t), base_all.data(), s));
+    // entries (cta, peer, src, dst) in CTA order, peers ascending inside a CTA
+    const int G = A.G;
+    struct E { int32_t cta, peer, src, dst; };
+    std::vector<E> ent;
+    ent.reserve(req_local.size());
+    std::vector<int64_t> tr_end(G);
+    for (int g = 0; g < G; ++g) tr_end[g] = (A.plan_rows_host[g + 1] + 15) / 16;
+    for (int q = 0; q < P; ++q) {
+        if (q == me) continue;
+        for (int64_t k = D.send_off[q]; k < D.send_off[q + 1]; ++k) {
+            const int32_t sg = req_local[k];
+            const int g = (int)(std::upper_bound(tr_end.begin(), tr_end.end(), (int64_t)sg) - tr_end.begin());
+            if (g >= G) return fail(MF_ERR_INVALID_ARG, "requested segment outside the own rows");
+            ent.push_back(E{g, q, sg, (int32_t)(base_all[(size_t)q * P + me] + (k - D.send_off[q]))});
+        }
+    }
+    std::stable_sort(ent.begin(), ent.end(), [](const E& x, const E& y) { return x.cta != y.cta ? x.cta < y.cta : x.peer < y.peer; });
+    const size_t ne = ent.size();
+    std::vector<int32_t> sptr(G + 1, 0), ssrc(ne), sdst(ne);
+    std::vector<int8_t> speer(ne);
+    std::vector<uint8_t> smask(G, 0);
+    for (size_t k = 0; k < ne; ++k) {
+        sptr[ent[k].cta + 1]++;
+        ssrc[k] = ent[k].src; sdst[k] = ent[k].dst; speer[k] = (int8_t)ent[k].peer;
+        smask[ent[k].cta] |= (uint8_t)(1u << ent[k].peer);
+    }
+    for (int g = 0; g < G; ++g) sptr[g + 1] += sptr[g];
+    std::vector<int64_t> nprod_to(P, 0), nprod_all((size_t)P * P);
+    for (int g = 0; g < G; ++g)
+        for (int r = 0; r < P; ++r) nprod_to[r] += (smask[g] >> r) & 1u;
+    MF_TRY(comm_allgather(c, nprod_to.data(), P * sizeof(int64_t), nprod_all.data(), s));
+    for (int r = 0; r < MG_PMAX; ++r) { m.nprod[r] = 0; m.hlo[r] = 0; m.hhi[r] = 0; m.win[r] = nullptr; }
+    for (int r = 0; r < P; ++r) {
+        m.nprod[r] = r == me ? 0 : (int)nprod_all[(size_t)r * P + me];
+        if (r != me) {
+            m.hlo[r] = (int32_t)halo_base(D, r);
+            m.hhi[r] = (int32_t)(halo_base(D, r) + D.recv_off[r + 1] - D.recv_off[r]);
+        }
+    }
+    // device copies of the lists (one allocation: ptr | src | dst | peer | mask)
+    const size_t bytes = (size_t)(G + 1) * 4 + ne * 4 * 2 + ne + (size_t)G + 64;
+    char* d = nullptr;
+    MF_TRY(alloc(&d, bytes, s));
+    D.dev_arrays = d;
+    size_t o = 0;
+    auto put = [&](const void* h, size_t nb) -> char* {
+        char* p = d + o;
+        if (nb) cudaMemcpyAsync(p, h, nb, cudaMemcpyHostToDevice, s);
+        o += (nb + 15) / 16 * 16;
+        return p;
+    };
+    m.send_ptr = reinterpret_cast<const int32_t*>(put(sptr.data(), sptr.size() * 4));
+    m.send_src = reinterpret_cast<const int32_t*>(put(ssrc.data(), ne * 4));
+    m.send_dst = reinterpret_cast<const int32_t*>(put(sdst.data(), ne * 4));
+    m.send_peer = reinterpret_cast<const int8_t*>(put(speer.data(), ne));
+    m.send_mask = reinterpret_cast<const uint8_t*>(put(smask.data(), (size_t)G));
+    if (o > bytes + 64) return fail(MF_ERR_INVALID_ARG, "internal: send list layout");
+    MF_CUDA(cudaGetLastError());
+    // windows: the extended PV vector and the sync words, same size on every rank
+    const int64_t n_ext_seg = D.nown_seg + D.nhalo + 1;
+    int64_t wb = WIN_PV + n_ext_seg * PVS * 8;
+    wb = (wb + 4095) / 4096 * 4096;
+    std::vector<int64_t> wall(P);
+    MF_TRY(comm_allgather(c, &wb, sizeof(wb), wall.data(), s));
+    for (int r = 0; r < P; ++r) wb = std::max(wb, wall[r]);
+    D.win_bytes = (size_t)wb;
+    m.off_tag = WIN_TAG; m.off_cnt = WIN_CNT; m.off_red = WIN_RED; m.off_pv = WIN_PV;
+    if (c->local || P == 1) {
+        MF_TRY(alloc(&D.win, D.win_bytes, s));
+        MF_CUDA(cudaMemsetAsync(D.win, 0, D.win_bytes, s));
+        MF_CUDA(cudaStreamSynchronize(s));
+        std::vector<unsigned long long> ptrs(P);
+        const unsigned long long mine = (unsigned long long)D.win;
+        if (c->local) MF_TRY(comm_allgather(c, &mine, sizeof(mine), ptrs.data(), s));
+        else ptrs[0] = mine;
+        for (int r = 0; r < P; ++r) m.win[r] = (char*)ptrs[r];
+    } else {
+        // NVLink peers: an NCCL symmetric window, the peers' mappings from the device API
+        const ncclTeam_t lsa = ncclTeamLsa(c->nccl);
+        if (lsa.nRanks != P) return fail(MF_ERR_UNSUPPORTED, "device-initiated kernel needs every rank in one NVLink domain");
+        void* wp = nullptr;
+        MF_NCCL(ncclMemAlloc(&wp, D.win_bytes));
+        D.win = (char*)wp;
+        D.win_nccl = true;
+        MF_NCCL(ncclCommWindowRegister(c->nccl, wp, D.win_bytes, &D.nwin, NCCL_WIN_COLL_SYMMETRIC));
+        MF_CUDA(cudaMemsetAsync(D.win, 0, D.win_bytes, s));
+        unsigned long long* dptr = nullptr;
+        DistWs ws(s);
+        MF_TRY(ws.get(&dptr, (size_t)P));
+        k_peer_ptrs<<<1, 32, 0, s>>>(D.nwin, P, dptr);
+        MF_CUDA(cudaGetLastError());
+        std::vector<unsigned long long> ptrs(P);
+        MF_CUDA(cudaMemcpyAsync(ptrs.data(), dptr, P * 8, cudaMemcpyDeviceToHost, s));
+        MF_CUDA(cudaStreamSynchronize(s));
+        for (int r = 0; r < P; ++r) m.win[r] = (char*)ptrs[r];
+        MF_TRY(alloc(&D.bar_scratch, 1, s));
+    }
     return MF_OK;
 }
 
@@ -487,15 +732,9 @@ mf_status dist_create(Comm* comm, int64_t n_global, int64_t row_begin, int64_t r
         return fail(MF_ERR_INVALID_ARG, "row blocks must be aligned to 16-row tile rows");
     DistWs ws(s);
     // every rank's row range (the owners of the halo segments)
-    int64_t *rr_d = nullptr, *rr_all = nullptr;
-    MF_TRY(ws.get(&rr_d, 2));
-    MF_TRY(ws.get(&rr_all, 2 * (size_t)P));
     const int64_t mine[2] = {row_begin, row_end};
-    MF_CUDA(cudaMemcpyAsync(rr_d, mine, sizeof(mine), cudaMemcpyHostToDevice, s));
-    MF_NCCL(ncclAllGather(rr_d, rr_all, 2, ncclInt64, comm->nccl, s));
     std::vector<int64_t> rr(2 * (size_t)P);
-    MF_CUDA(cudaMemcpyAsync(rr.data(), rr_all, rr.size() * 8, cudaMemcpyDeviceToHost, s));
-    MF_CUDA(cudaStreamSynchronize(s));
+    MF_TRY(comm_allgather(comm, mine, sizeof(mine), rr.data(), s));
     std::unique_ptr<DistInfo> D(new DistInfo());
     D->comm = comm; D->n_global = n_global; D->row_begin = row_begin; D->row_end = row_end; D->owner = s;
     D->rank_rows.resize(P + 1);
@@ -515,15 +754,19 @@ mf_status dist_create(Comm* comm, int64_t n_global, int64_t row_begin, int64_t r
     MF_CUDA(cudaMemsetAsync(flag, 0, nseg * 8, s));
     if (nnz > 0) k_mark_halo<<<(unsigned)std::min<int64_t>((nnz + 255) / 256, 148 * 16), 256, 0, s>>>(colidx, nnz, seg_lo, seg_hi, flag);
     MF_TRY(scan_excl_i64(flag, nseg, pre, tmp, s));
-    MF_CUDA(cudaMemcpyAsync(&D->nhalo, pre + nseg, 8, cudaMemcpyDeviceToHost, s));
+    int64_t cnt2[2] = {0, 0};   // halo segments in total, below my block
+    MF_CUDA(cudaMemcpyAsync(&cnt2[0], pre + nseg, 8, cudaMemcpyDeviceToHost, s));
+    MF_CUDA(cudaMemcpyAsync(&cnt2[1], pre + seg_lo, 8, cudaMemcpyDeviceToHost, s));
     MF_CUDA(cudaStreamSynchronize(s));
+    D->nhalo = cnt2[0];
+    D->nlo = cnt2[1];
     int32_t *hlist = nullptr, *col2 = nullptr;
     MF_TRY(ws.get(&hlist, (size_t)D->nhalo));
     MF_TRY(ws.get(&col2, (size_t)nnz));
     k_halo_list<<<(unsigned)std::min<int64_t>((nseg + 255) / 256, 148 * 16), 256, 0, s>>>(flag, pre, nseg, hlist);
     if (nnz > 0)
         k_remap<<<(unsigned)std::min<int64_t>((nnz + 255) / 256, 148 * 16), 256, 0, s>>>(colidx, nnz, row_begin, seg_lo, seg_hi,
-                                                                                    D->nown_seg, pre, col2);
+                                                                                    D->nown_seg, D->nlo, pre, col2);
     MF_CUDA(cudaGetLastError());
     std::vector<int32_t> hl((size_t)D->nhalo);
     if (D->nhalo) MF_CUDA(cudaMemcpyAsync(hl.data(), hlist, hl.size() * 4, cudaMemcpyDeviceToHost, s));
@@ -540,50 +783,79 @@ mf_status dist_create(Comm* comm, int64_t n_global, int64_t row_begin, int64_t r
         }
         for (int q2 = 0; q2 < P; ++q2) D->recv_off[q2 + 1] += D->recv_off[q2];
     }
+    if (D->recv_off[me] != D->nlo) return fail(MF_ERR_INVALID_ARG, "internal: halo order");
     // tell every owner which of its segments I need: counts (all-gathered P x P), then the lists
     std::vector<int64_t> cnt_me(P), cnt_all((size_t)P * P);
     for (int q = 0; q < P; ++q) cnt_me[q] = D->recv_off[q + 1] - D->recv_off[q];
-    int64_t *cm_d = nullptr, *ca_d = nullptr;
-    MF_TRY(ws.get(&cm_d, (size_t)P));
-    MF_TRY(ws.get(&ca_d, (size_t)P * P));
-    MF_CUDA(cudaMemcpyAsync(cm_d, cnt_me.data(), P * 8, cudaMemcpyHostToDevice, s));
-    MF_NCCL(ncclAllGather(cm_d, ca_d, (size_t)P, ncclInt64, comm->nccl, s));
-    MF_CUDA(cudaMemcpyAsync(cnt_all.data(), ca_d, cnt_all.size() * 8, cudaMemcpyDeviceToHost, s));
-    MF_CUDA(cudaStreamSynchronize(s));
+    MF_TRY(comm_allgather(comm, cnt_me.data(), P * sizeof(int64_t), cnt_all.data(), s));
     D->send_off.assign(P + 1, 0);
     for (int q = 0; q < P; ++q) D->send_off[q + 1] = D->send_off[q] + (q == me ? 0 : cnt_all[(size_t)q * P + me]);
-    int32_t* req = nullptr;   // global segment ids requested from me, per peer
-    MF_TRY(ws.get(&req, (size_t)D->send_off[P]));
-    MF_NCCL(ncclGroupStart());
+    std::vector<std::vector<int32_t>> to(P), from(P);
     for (int q = 0; q < P; ++q) {
         if (q == me) continue;
-        const int64_t nr = D->recv_off[q + 1] - D->recv_off[q], ns = D->send_off[q + 1] - D->send_off[q];
-        if (nr) MF_NCCL(ncclSend(hlist + D->recv_off[q], (size_t)nr, ncclInt32, q, comm->nccl, s));
-        if (ns) MF_NCCL(ncclRecv(req + D->send_off[q], (size_t)ns, ncclInt32, q, comm->nccl, s));
+        to[q].assign(hl.begin() + D->recv_off[q], hl.begin() + D->recv_off[q + 1]);
+        from[q].resize((size_t)(D->send_off[q + 1] - D->send_off[q]));
     }
-    MF_NCCL(ncclGroupEnd());
+    MF_TRY(comm_exchange_i32(comm, to, from, s));
     std::vector<int32_t> rq((size_t)D->send_off[P]);
-    if (!rq.empty()) MF_CUDA(cudaMemcpyAsync(rq.data(), req, rq.size() * 4, cudaMemcpyDeviceToHost, s));
-    MF_CUDA(cudaStreamSynchronize(s));
-    for (auto& g : rq) g = (int32_t)(g - seg_lo);              // my local segment ids
+    for (int q = 0; q < P; ++q)
+        for (size_t k = 0; k < from[q].size(); ++k) rq[(size_t)D->send_off[q] + k] = (int32_t)(from[q][k] - seg_lo);   // my local segment ids
+    for (auto g : rq)
+        if (g < 0 || g >= D->nown_seg) return fail(MF_ERR_INVALID_ARG, "peer requested a segment I do not own");
     MF_TRY(alloc(&D->send_idx, std::max<size_t>(rq.size(), 1), s));
     if (!rq.empty()) MF_CUDA(cudaMemcpyAsync(D->send_idx, rq.data(), rq.size() * 4, cudaMemcpyHostToDevice, s));
-    // the local matrix: own segments, then the halo segments
+    // the local matrix: columns [lower halo | own | upper halo]
     const int64_t n_ext = (D->nown_seg + D->nhalo) * 16;
     if (n_ext > INT32_MAX) return fail(MF_ERR_UNSUPPORTED, "local extended vector exceeds 2^31 columns");
+    A->coff = D->nlo;
     MF_TRY(convert_csr(n_local, n_ext, nnz, rowptr, col2, vals, o, s, A));
     MF_CUDA(cudaStreamSynchronize(s));
+    MF_TRY(mg_setup(*D, *A, rq, s));
     *out = D.release();
     return MF_OK;
 }
 
 void dist_destroy(DistInfo* D) { delete D; }
 
+namespace {
+struct MgCtx {
+    DistInfo* D;
+};
+// before every device-initiated solve: clear my window (sync words, extended vector), then a
+// cross-rank barrier so that no peer stores into a window that is still being cleared
+mf_status mg_prelaunch(void* ctx, cudaStream_t s) {
+    DistInfo& D = *static_cast<MgCtx*>(ctx)->D;
+    MF_CUDA(cudaMemsetAsync(D.win, 0, D.win_bytes, s));
+    Comm* c = D.comm;
+    if (c->nranks == 1) return MF_OK;
+    if (c->local) {
+        MF_CUDA(cudaStreamSynchronize(s));
+        if (!c->local->barrier()) return fail(MF_ERR_DEADLOCK, "local rank group: barrier timed out");
+        return MF_OK;
+    }
+    MF_NCCL(ncclAllReduce(D.bar_scratch, D.bar_scratch, 1, ncclInt32, ncclSum, c->nccl, s));   // stream-ordered barrier
+    return MF_OK;
+}
+}  // namespace
+
+mf_status mg_solve(const TileMatrix& A, DistInfo& D, const double* b, double* x, const mf_solve_opts& o, mf_solve_info* info,
+                   cudaStream_t s) {
+    if (D.mg.P == 0 || !D.win) return fail(MF_ERR_UNSUPPORTED, "device-initiated kernel: more ranks than one NVLink domain");
+    MgCtx ctx{&D};
+    MgLaunch L;
+    L.args = D.mg;
+    L.pv_own = reinterpret_cast<double*>(D.win + D.mg.off_pv) + D.nlo * PVS;
+    L.prelaunch = mg_prelaunch;
+    L.ctx = &ctx;
+    return run_solve(A, false, b, x, o, info, s, &L);
+}
+
 mf_status dist_solve(const TileMatrix& A, const DistInfo& D, bool bicg, const double* b, double* x, const mf_solve_opts& o,
                      mf_solve_info* info, cudaStream_t s) {
     if (o.M) return fail(MF_ERR_NOT_IMPLEMENTED, "distributed preconditioned solves");
     if (o.sticky || o.tile_level_counts || o.collect_stats)
         return fail(MF_ERR_NOT_IMPLEMENTED, "distributed solve: sticky variant / level statistics");
+    if (D.comm->local) return fail(MF_ERR_NOT_IMPLEMENTED, "local rank groups run the device-initiated kernel only");
     const int P = D.comm->nranks;
     const int64_t n = A.n_rows;
     int dev = 0, smem_optin = 0;
@@ -595,19 +867,23 @@ mf_status dist_solve(const TileMatrix& A, const DistInfo& D, bool bicg, const do
     DistArgs a{};
     a.A = mfk::Mat{A.n_rows, A.n_cols, A.ntr, A.tr_slot, A.TileRowPtr, A.tile_info, A.sidx, A.blob,
                    reinterpret_cast<const mfk::TsStage*>(A.stg), A.stg_ptr, A.TileNnz, A.ts, (int)A.max_w,
-                   A.plane64, A.plane32, A.plane16, A.plane8, nullptr};
+                   A.plane64, A.plane32, A.plane16, A.plane8, nullptr, A.coff};
     a.G = G; a.plan_tr = A.plan_tr; a.n = n; a.nown_seg = D.nown_seg; a.b = b; a.x = x; a.P = P;
+    // extended PV vectors [lower halo | own | upper halo]; the kernels address the own part
     const int64_t npv = (D.nown_seg + D.nhalo + 1) * PVS;
+    double *pv_ext = nullptr, *sv_ext = nullptr;
     MF_TRY(ws.get(&a.r, (size_t)n));
-    MF_TRY(ws.get(&a.pv, (size_t)npv));
+    MF_TRY(ws.get(&pv_ext, (size_t)npv));
     MF_TRY(ws.get(&a.mu, (size_t)n));
     if (bicg) {
-        MF_TRY(ws.get(&a.sv, (size_t)npv));
+        MF_TRY(ws.get(&sv_ext, (size_t)npv));
         MF_TRY(ws.get(&a.rh, (size_t)n));
         MF_TRY(ws.get(&a.th, (size_t)n));
-        MF_CUDA(cudaMemsetAsync(a.sv, 0, npv * 8, s));
+        MF_CUDA(cudaMemsetAsync(sv_ext, 0, npv * 8, s));
+        a.sv = sv_ext + D.nlo * PVS;
     }
-    MF_CUDA(cudaMemsetAsync(a.pv, 0, npv * 8, s));
+    MF_CUDA(cudaMemsetAsync(pv_ext, 0, npv * 8, s));
+    a.pv = pv_ext + D.nlo * PVS;
     MF_TRY(ws.get(&a.slots, (size_t)4 * G));
     MF_TRY(ws.get(&a.part, 4));
     MF_TRY(ws.get(&a.gath, (size_t)4 * P));
@@ -643,7 +919,7 @@ mf_status dist_solve(const TileMatrix& A, const DistInfo& D, bool bicg, const do
     MF_CUDA(cudaEventRecord(e0, s));
     // init: r0 = b - A~ x0 (x0 staged in the PV layout, halo exchanged), partials (b,b), (r,r)
     k_stage_x0<<<148, 256, 0, s>>>(a, a.pv);
-    MF_TRY(exchange(D, a.pv, sendbuf, D.nown_seg, a.pv, a.st, s));
+    MF_TRY(exchange(D, a.pv, sendbuf, a.pv, a.st, s));
     MF_TRY(launch_spmv(f_init, a.pv));
     k_rank_partial<<<1, 32, 0, s>>>(a, 2);
     MF_TRY(allgather(D, a.part, a.gath, 2, s));
@@ -657,13 +933,13 @@ mf_status dist_solve(const TileMatrix& A, const DistInfo& D, bool bicg, const do
     MF_CUDA(cudaGetLastError());
     // one iteration, enqueued as a chunk captured in a CUDA graph
     auto one_iter = [&]() -> mf_status {
-        MF_TRY(exchange(D, a.pv, sendbuf, D.nown_seg, a.pv, a.st, q));
+        MF_TRY(exchange(D, a.pv, sendbuf, a.pv, a.st, q));
         MF_TRY(launch_spmv(f_mu, a.pv));
         k_rank_partial<<<1, 32, 0, q>>>(a, bicg ? 2 : 2);
         MF_TRY(allgather(D, a.part, a.gath, 2, q));
         if (bicg) {
             k_bicg_s<<<G, B, 0, q>>>(a);
-            MF_TRY(exchange(D, a.sv, sendbuf, D.nown_seg, a.sv, a.st, q));
+            MF_TRY(exchange(D, a.sv, sendbuf, a.sv, a.st, q));
             MF_TRY(launch_spmv(f_th, a.sv));
             k_rank_partial<<<1, 32, 0, q>>>(a, 2);
             MF_TRY(allgather(D, a.part, a.gath, 2, q));
@@ -808,6 +1084,39 @@ mf_status mf_comm_destroy(mf_comm* c) {
     return MF_OK;
 }
 
+struct mf_local_group {
+    mf::LocalGroup g;
+};
+
+mf_status mf_local_group_create(int32_t nranks, mf_local_group** out) {
+    if (!out || nranks < 1 || nranks > mf::MG_PMAX) return mf::fail(MF_ERR_INVALID_ARG, "nranks must be in [1, 8]");
+    mf_local_group* g = new (std::nothrow) mf_local_group();
+    if (!g) return mf::fail(MF_ERR_OOM, "host allocation failed");
+    g->g.P = nranks;
+    g->g.slot.resize(nranks);
+    g->g.mail.assign(nranks, std::vector<std::vector<int32_t>>(nranks));
+    *out = g;
+    return MF_OK;
+}
+
+mf_status mf_local_group_destroy(mf_local_group* g) {
+    delete g;
+    return MF_OK;
+}
+
+mf_status mf_comm_create_local(mf_local_group* g, int32_t rank, mf_comm** out) {
+    if (!g || !out || rank < 0 || rank >= g->g.P) return mf::fail(MF_ERR_INVALID_ARG, "bad group / rank");
+    int sms = 0;
+    MF_TRY(mf::check_device(&sms));
+    mf_comm* c = new (std::nothrow) mf_comm();
+    if (!c) return mf::fail(MF_ERR_OOM, "host allocation failed");
+    c->c.nranks = g->g.P;
+    c->c.rank = rank;
+    c->c.local = &g->g;
+    *out = c;
+    return MF_OK;
+}
+
 mf_status mf_comm_info(const mf_comm* c, int32_t* nranks, int32_t* rank) {
     if (!c) return mf::fail(MF_ERR_INVALID_ARG, "comm is NULL");
     if (nranks) *nranks = c->c.nranks;
@@ -849,6 +1158,13 @@ static mf_status solve_dist(const mf_tile_matrix* A, bool bicg, const double* b,
     mf_default_solve_opts(&o);
     if (opts) o = *opts;
     if (!(o.tol >= 0) || o.max_iter < 0) return mf::fail(MF_ERR_INVALID_ARG, "bad tol / max_iter");
+    if (o.dist_mode < 0 || o.dist_mode > 2) return mf::fail(MF_ERR_INVALID_ARG, "dist_mode must be 0, 1 or 2");
+    const bool device_initiated = o.dist_mode == 2 || (o.dist_mode == 0 && !bicg && !o.M && !o.sticky &&
+                                                       !o.tile_level_counts && !o.collect_stats && A->dist->mg.P > 0);
+    if (device_initiated) {
+        if (bicg) return mf::fail(MF_ERR_NOT_IMPLEMENTED, "device-initiated multi-GPU kernel: BiCGSTAB");
+        return mf::mg_solve(A->m, *A->dist, b, x, o, info, (cudaStream_t)stream);
+    }
     return mf::dist_solve(A->m, *A->dist, bicg, b, x, o, info, (cudaStream_t)stream);
 }
 

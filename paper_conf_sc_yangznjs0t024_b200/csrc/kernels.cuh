@@ -36,6 +36,8 @@ struct Mat {
     const uint8_t* __restrict__ p8;
     uint8_t* stk;                         // sticky variant (P:237 literal): per slice column (TS layout) or
                                           // per tile (compact), bit L set = values lowered to L in place
+    int64_t coff;                         // column segment of row segment 0 (row-block ranks: the halo
+                                          // segments of lower ranks precede the own ones); 0 = square
 };
 
 // ------------------------------------------------------------------------------------------
@@ -549,6 +551,7 @@ __device__ __forceinline__ void spmv_ts(const Mat& A, int64_t tr0c, const double
     const uint32_t* recs = reinterpret_cast<const uint32_t*>(A.stg + s_begin);
     const int NST = sm.nst;
     double* E = sm.ebuf + (size_t)w * sm.ecap * 16;     // decode buffer: ecap columns x 16 doubles
+    const double* xb = pv - A.coff * PVS;                 // column space (pv: the own segments)
     __syncthreads();                          // ring counters / previous phase's smem users
     if (ns == 0) return;
     unsigned long long pol = 0;
@@ -561,7 +564,7 @@ __device__ __forceinline__ void spmv_ts(const Mat& A, int64_t tr0c, const double
         // matrices, e.g. C1); only the x windows are re-staged
         const unsigned rc = (unsigned)sm.ctr[1];
         if (w == 0)
-            for (int k = 0; k < ns; ++k) ts_issue(A.blob, recs[k * 32 + lane], sm.slot(k), sm.blob_cap, sm.full + k, pv, rc == 0, pol);
+            for (int k = 0; k < ns; ++k) ts_issue(A.blob, recs[k * 32 + lane], sm.slot(k), sm.blob_cap, sm.full + k, xb, rc == 0, pol);
         for (int k = 0; k < ns; ++k) {
             mbar_wait(sm.full + k, rc & 1u);
             ts_consume<DYN, STK>(ts_view(sm.slot(k), sm.blob_cap), pv, range_guard, own_mode, ownv, A.n_rows, A.stk, E, emit);
@@ -582,7 +585,7 @@ __device__ __forceinline__ void spmv_ts(const Mat& A, int64_t tr0c, const double
             // the slot's previous use (previous SpMV) finished before the caller's barrier; its
             // "empty" phase completed: wait on it to keep the parity in step
             if (u0 + k >= (unsigned)NST) mbar_wait(sm.empty + isl, iph ^ 1u);
-            ts_issue(A.blob, recs[k * 32 + lane], sm.slot(isl), sm.blob_cap, sm.full + isl, pv, true, pol);
+            ts_issue(A.blob, recs[k * 32 + lane], sm.slot(isl), sm.blob_cap, sm.full + isl, xb, true, pol);
             if (++isl == NST) { isl = 0; iph ^= 1u; }
         }
 #pragma unroll
@@ -594,7 +597,7 @@ __device__ __forceinline__ void spmv_ts(const Mat& A, int64_t tr0c, const double
         if (lane == 0) mbar_arrive(sm.empty + sl);
         if (w == 0 && k + NST < ns) {
             mbar_wait(sm.empty + sl, ph);         // every warp is done with the slot
-            ts_issue(A.blob, pre[0], sm.slot(sl), sm.blob_cap, sm.full + sl, pv, true, pol);
+            ts_issue(A.blob, pre[0], sm.slot(sl), sm.blob_cap, sm.full + sl, xb, true, pol);
 #pragma unroll
             for (int j = 0; j + 1 < TS_PF; ++j) pre[j] = pre[j + 1];
             pre[TS_PF - 1] = k + NST + TS_PF < ns ? recs[(k + NST + TS_PF) * 32 + lane] : 0u;
@@ -686,6 +689,7 @@ template <bool DYN, bool STK, int PF, class Emit>
 __device__ __forceinline__ void spmv_compact(const Mat& A, int64_t tr0, int64_t tr1, const double* pv, int range_guard,
                                              const WinSmem& w, int own_mode, const double* ownv, Emit& emit) {
     const int t = threadIdx.x, B = blockDim.x, H = B >> 4, h = t >> 4, lane = t & 15;
+    const double* xb = pv - A.coff * PVS;     // column space (pv: the own segments)
     __syncthreads();
     if (t < 4) w.pb[t] = t == 0 ? (unsigned long long)A.p64 : t == 1 ? (unsigned long long)A.p32
                        : t == 2 ? (unsigned long long)A.p16 : (unsigned long long)A.p8;
@@ -715,7 +719,7 @@ __device__ __forceinline__ void spmv_compact(const Mat& A, int64_t tr0, int64_t 
         const int nt = w.ht[nw];
         uint32_t* code = reinterpret_cast<uint32_t*>(w.buf);
         for (int i = t; i < nt; i += B) {
-            const uint32_t c = STK ? sticky_code(A, t0 + i, pv, range_guard, true) : tile_code<DYN>(A.tile_info[t0 + i], pv, range_guard);
+            const uint32_t c = STK ? sticky_code(A, t0 + i, xb, range_guard, true) : tile_code<DYN>(A.tile_info[t0 + i], xb, range_guard);
             if (staged) code[i] = c;
         }
         __syncthreads();
@@ -744,13 +748,13 @@ __device__ __forceinline__ void spmv_compact(const Mat& A, int64_t tr0, int64_t 
             if (own_mode == 1) ov = pv[TR * PVS + lane];
             else if (own_mode == 2 && i < A.n_rows) ov = ownv[i];
             double acc = 0.0;
-            acc = slot_block<DYN, STK, PF>(A, w.pb, cur, min(W, PF), sb * 16 + lane, cd, staged, tb_abs, pv, range_guard, acc);
+            acc = slot_block<DYN, STK, PF>(A, w.pb, cur, min(W, PF), sb * 16 + lane, cd, staged, tb_abs, xb, range_guard, acc);
             for (int k = PF; k < W; k += PF) {
                 uint16_t more[PF];
                 const uint16_t* sp = A.sidx + (sb + k) * 16 + lane;
 #pragma unroll
                 for (int q = 0; q < PF; ++q) more[q] = (k + q < W) ? __ldg(sp + q * 16) : mf::SLOT_PAD;
-                acc = slot_block<DYN, STK, PF>(A, w.pb, more, min(W - k, PF), (sb + k) * 16 + lane, cd, staged, tb_abs, pv,
+                acc = slot_block<DYN, STK, PF>(A, w.pb, more, min(W - k, PF), (sb + k) * 16 + lane, cd, staged, tb_abs, xb,
                                                range_guard, acc);
             }
             emit(TR, lane, acc, ov);
@@ -765,7 +769,7 @@ __device__ __forceinline__ void spmv_compact(const Mat& A, int64_t tr0, int64_t 
 template <bool DYN>
 __device__ __forceinline__ void count_levels(const Mat& A, int64_t tr0c, int64_t tr1c, const double* pv, int range_guard, Counts* cnt) {
     for (int64_t i = A.tr_tile[tr0c] + threadIdx.x; i < A.tr_tile[tr1c]; i += blockDim.x) {
-        const int e = (int)(tile_code<DYN>(A.tile_info[i], pv, range_guard) & 7u);
+        const int e = (int)(tile_code<DYN>(A.tile_info[i], pv - A.coff * PVS, range_guard) & 7u);
         cnt->tile(e);
         cnt->nzn(e, (int)(A.tile_nnz[i + 1] - A.tile_nnz[i]));
     }

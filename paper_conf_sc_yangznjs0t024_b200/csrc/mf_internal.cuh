@@ -104,7 +104,44 @@ struct TileMatrix {
     int64_t* plan_rows_host = nullptr;  // host [G+1]
     // byte bookkeeping
     int64_t canonical_bytes = 0, kernel_bytes = 0;
+    // column segment of row segment 0: set by the caller before convert_csr (row-block ranks
+    // whose lower-rank halo segments precede the own ones, dist.cu); 0 = square
+    int64_t coff = 0;
     cudaStream_t owner_stream = nullptr;
+};
+
+constexpr int MG_PMAX = 8;  // ranks of the device-initiated multi-GPU kernel (one NVLink domain)
+
+// Device-initiated multi-GPU solve (Finding 2, applied across GPUs): one
+// persistent kernel per rank, every exchange done by the kernel itself through peer memory.
+// Each rank exposes a window (an NCCL symmetric window over NVLink, or same-device buffers for
+// ranks emulated on one GPU) holding: its extended PV vector (own + halo segments; peers store
+// their boundary segments straight into it), the cross-rank reduction slots with their tags,
+// and one arrival counter per peer.
+struct MgArgs {
+    int P = 0, me = 0;                 // P == 0: single-GPU kernel
+    char* win[MG_PMAX];                // window base of every rank (this process's mapping)
+    int64_t off_pv;                    // byte offset of the extended PV vector in each window
+    int64_t off_red;                   // doubles [2 parities][P][4]
+    int64_t off_tag;                   // u32 [2][P]: reduction number published with the slot
+    int64_t off_cnt;                   // u64 [P]: halo stores completed by CTAs of rank r
+    const int32_t* send_ptr;           // [G+1] entries of each CTA (sorted by CTA, then peer)
+    const int32_t* send_src;           // own segment (relative to the own part)
+    const int32_t* send_dst;           // segment of the peer's extended vector
+    const int8_t* send_peer;
+    const uint8_t* send_mask;          // [G] peers CTA g stores to (bit r)
+    const int32_t* seg_lo;             // [G] extended column segments gathered by CTA g
+    const int32_t* seg_hi;
+    int nprod[MG_PMAX];                // CTAs of rank r that store into my window
+    int32_t hlo[MG_PMAX], hhi[MG_PMAX];   // my extended segments received from rank r
+};
+
+// what run_solve needs to launch the multi-GPU kernel of one rank (dist.cu fills it)
+struct MgLaunch {
+    MgArgs args;
+    double* pv_own;                                      // own part of the window's extended PV vector
+    mf_status (*prelaunch)(void* ctx, cudaStream_t s);   // clear the window, cross-rank barrier
+    void* ctx;
 };
 
 mf_status convert_csr(int64_t n_rows, int64_t n_cols, int64_t nnz, const int64_t* rowptr, const int32_t* colidx,
@@ -121,7 +158,7 @@ mf_status run_cg_xr(const TileMatrix& A, double alpha, const double* p, const do
                     double* rr_host, cudaStream_t s);
 mf_status run_cg_p(const TileMatrix& A, double beta, const double* r, double* p, cudaStream_t s);
 mf_status run_solve(const TileMatrix& A, bool bicg, const double* b, double* x, const mf_solve_opts& o,
-                    mf_solve_info* info, cudaStream_t s);
+                    mf_solve_info* info, cudaStream_t s, const MgLaunch* mgl = nullptr);
 
 }  // namespace mf
 

@@ -140,7 +140,7 @@ void* pick_kernel(int maxt, bool bicg, bool dyn, bool count, bool sticky, bool p
 Mat mat_view(const TileMatrix& A) {
     return Mat{A.n_rows, A.n_cols, A.ntr, A.tr_slot, A.TileRowPtr, A.tile_info, A.sidx, A.blob,
                reinterpret_cast<const mfk::TsStage*>(A.stg), A.stg_ptr, A.TileNnz, A.ts, (int)A.max_w,
-               A.plane64, A.plane32, A.plane16, A.plane8, nullptr};
+               A.plane64, A.plane32, A.plane16, A.plane8, nullptr, A.coff};
 }
 
 // Ring depth of the TMA pipeline for a shared-memory budget (bytes available to the ring)
@@ -297,8 +297,10 @@ static double spmv_model_bytes(const TileMatrix& A, const unsigned long long* c1
 }
 
 mf_status run_solve(const TileMatrix& A, bool bicg, const double* b, double* x, const mf_solve_opts& o,
-                    mf_solve_info* info, cudaStream_t s) {
-    if (A.n_rows != A.n_cols) return fail(MF_ERR_INVALID_ARG, "solve needs a square matrix");
+                    mf_solve_info* info, cudaStream_t s, const MgLaunch* mgl) {
+    if (A.n_rows != A.n_cols && !mgl) return fail(MF_ERR_INVALID_ARG, "solve needs a square matrix");
+    if (mgl && (bicg || o.M || o.sticky || o.cg_variant || o.tile_level_counts || o.collect_stats))
+        return fail(MF_ERR_NOT_IMPLEMENTED, "device-initiated multi-GPU kernel: CG without preconditioner, sticky variant or statistics");
     if (o.max_iter < 0 || o.max_iter > ((int64_t)1 << 40)) return fail(MF_ERR_INVALID_ARG, "max_iter out of range");
     // sticky variant (P:237 literal): dynamic mode only (as in the oracle)
     const bool sticky = o.sticky && o.mode == MF_MODE_DYNAMIC_MIXED;
@@ -351,7 +353,7 @@ mf_status run_solve(const TileMatrix& A, bool bicg, const double* b, double* x, 
     const size_t smem = fixed + mfk::spmv_smem_bytes(A.ts, nst, A.slot_bytes, A.ecap, B / 32) + (size_t)cap * 8 * nvec + (size_t)pre_smem + 64;
     if ((int64_t)smem > smem_optin) return fail(MF_ERR_UNSUPPORTED, "shared-memory plan exceeds the device limit");
 
-    void* kfn = pick_kernel(B, bicg, dyn, count, sticky, pre, sr);
+    void* kfn = mgl ? pick_cgmg(B, dyn) : pick_kernel(B, bicg, dyn, count, sticky, pre, sr);
     MF_CUDA(cudaFuncSetAttribute(kfn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
     int per_sm = 0;
     MF_CUDA(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, kfn, B, smem));
@@ -369,7 +371,8 @@ mf_status run_solve(const TileMatrix& A, bool bicg, const double* b, double* x, 
     unsigned long long *lcounts = nullptr, *bar_ns = nullptr, *phase_ns = nullptr;
     const bool pbicg = pre && bicg;
     MF_TRY(ws.get(&r, n));
-    MF_TRY(ws.get(&p, pbicg ? n : npv));
+    if (mgl) p = mgl->pv_own;             // the window's extended vector (cleared by prelaunch)
+    else MF_TRY(ws.get(&p, pbicg ? n : npv));
     if (spill) MF_TRY(ws.get(&mu_g, n));
     if (bicg) {
         MF_TRY(ws.get(&rh, n));
@@ -387,7 +390,7 @@ mf_status run_solve(const TileMatrix& A, bool bicg, const double* b, double* x, 
         if (bicg) MF_TRY(ws.get(&psh, npv));
     }
     // PV vectors: padding rows / slots stay zero
-    if (!pbicg) MF_CUDA(cudaMemsetAsync(p, 0, npv * sizeof(double), s));
+    if (!pbicg && !mgl) MF_CUDA(cudaMemsetAsync(p, 0, npv * sizeof(double), s));
     if (sv && !pbicg && !sr) MF_CUDA(cudaMemsetAsync(sv, 0, npv * sizeof(double), s));
     if (pz && bicg) MF_CUDA(cudaMemsetAsync(pz, 0, npv * sizeof(double), s));
     if (psh) MF_CUDA(cudaMemsetAsync(psh, 0, npv * sizeof(double), s));
@@ -439,6 +442,12 @@ mf_status run_solve(const TileMatrix& A, bool bicg, const double* b, double* x, 
         a.pflags = P->flags; a.pctr = P->ctr; a.py = P->y; a.pz = pz; a.ps = psh;
     }
 
+    if (mgl) {
+        a.mg = mgl->args;
+        a.mg.seg_lo = A.seg_lo;
+        a.mg.seg_hi = A.seg_hi;
+        MF_TRY(mgl->prelaunch(mgl->ctx, s));
+    }
     Events ev;
     MF_CUDA(cudaEventCreate(&ev.e0));
     MF_CUDA(cudaEventCreate(&ev.e1));

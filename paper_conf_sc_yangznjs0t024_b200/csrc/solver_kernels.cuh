@@ -75,6 +75,7 @@ struct SolveArgs {
     double* pz;                  // PCG: z (normal); PBiCGSTAB: p^ (PV)
     double* ps;                  // PBiCGSTAB: s^ (PV)
     unsigned pe0;                // epoch of the first apply of this solve
+    MgArgs mg;                   // multi-GPU single kernel (P == 0: off)
 };
 
 __device__ __forceinline__ unsigned ld_acquire(const unsigned* p) {
@@ -95,6 +96,7 @@ struct Ctx {
     unsigned bar_target = 0;
     int parity = 0;
     int spmv = 0;
+    unsigned nred = 0;           // cross-rank reductions so far (multi-GPU kernel)
 };
 
 __device__ __forceinline__ void red_release_add(unsigned* p, unsigned v) {
@@ -102,6 +104,28 @@ __device__ __forceinline__ void red_release_add(unsigned* p, unsigned v) {
 }
 // generic-proxy writes of a PV vector -> later bulk copies (async proxy) of other CTAs / this CTA
 __device__ __forceinline__ void fence_proxy_async() { asm volatile("fence.proxy.async.global;" ::: "memory"); }
+// system scope (peer GPUs over NVLink)
+__device__ __forceinline__ unsigned ld_acquire_sys(const unsigned* p) {
+    unsigned v;
+    asm volatile("ld.acquire.sys.global.u32 %0, [%1];" : "=r"(v) : "l"(p) : "memory");
+    return v;
+}
+__device__ __forceinline__ unsigned long long ld_acquire_sys64(const unsigned long long* p) {
+    unsigned long long v;
+    asm volatile("ld.acquire.sys.global.u64 %0, [%1];" : "=l"(v) : "l"(p) : "memory");
+    return v;
+}
+__device__ __forceinline__ double ld_relaxed_sys_f64(const double* p) {
+    double v;
+    asm volatile("ld.relaxed.sys.global.f64 %0, [%1];" : "=d"(v) : "l"(p) : "memory");
+    return v;
+}
+__device__ __forceinline__ void st_release_sys(unsigned* p, unsigned v) {
+    asm volatile("st.release.sys.global.u32 [%0], %1;" ::"l"(p), "r"(v) : "memory");
+}
+__device__ __forceinline__ void red_release_sys_add64(unsigned long long* p, unsigned long long v) {
+    asm volatile("red.release.sys.global.add.u64 [%0], %1;" ::"l"(p), "l"(v) : "memory");
+}
 
 // ---- synchronisation.  Stall time is accumulated in shared memory (spin_ns), not in global
 // memory, so the barrier's critical path is: release-add, acquire-spin, fence.
@@ -131,16 +155,63 @@ __device__ __forceinline__ bool grid_barrier(const SolveArgs& a, Ctx& c) {
     return s_abort == 0;
 }
 
+// Multi-GPU kernel: store this CTA's own segments that peers gather (values + level byte, 144 B
+// each) into the peers' extended vectors, then count the CTA as arrived at each such peer (one
+// system-scope release-add per peer after the CTA barrier and a system fence).
+__device__ __forceinline__ void mg_push(const SolveArgs& a, const double* own) {
+    const MgArgs& m = a.mg;
+    const int e0 = m.send_ptr[blockIdx.x], e1 = m.send_ptr[blockIdx.x + 1];
+    if (e1 == e0) return;
+    for (int k = threadIdx.x; k < (e1 - e0) * PVS; k += blockDim.x) {
+        const int e = e0 + k / PVS, d = k - (k / PVS) * PVS;
+        const double v = __ldcg(own + (int64_t)m.send_src[e] * PVS + d);
+        double* dst = reinterpret_cast<double*>(m.win[m.send_peer[e]] + m.off_pv) + (int64_t)m.send_dst[e] * PVS + d;
+        __stcg(dst, v);
+    }
+    __syncthreads();
+    if (threadIdx.x == 0) {
+        __threadfence_system();
+        const unsigned mask = m.send_mask[blockIdx.x];
+        for (int r = 0; r < m.P; ++r)
+            if (mask & (1u << r))
+                red_release_sys_add64(reinterpret_cast<unsigned long long*>(m.win[r] + m.off_cnt) + m.me, 1ull);
+    }
+}
+
 // all threads: the CTA's writes of the SpMV input are complete -> ready flag `epoch`
-__device__ __forceinline__ void publish(const SolveArgs& a, unsigned epoch) {
+template <bool MG = false>
+__device__ __forceinline__ void publish(const SolveArgs& a, unsigned epoch, const double* own = nullptr) {
     fence_proxy_async();
     __syncthreads();
+    if (MG && a.mg.P > 1) mg_push(a, own);
     if (threadIdx.x == 0 && (int)blockIdx.x != a.stall_cta) st_release(&a.flags[blockIdx.x], epoch);
 }
 
+// Multi-GPU kernel: the halo segments this CTA gathers from rank r are complete once all nprod[r]
+// storing CTAs of r arrived for this epoch (counters are monotone: epoch * nprod[r]).
+__device__ __forceinline__ bool mg_wait_halo(const SolveArgs& a, unsigned epoch, unsigned long long t0) {
+    const MgArgs& m = a.mg;
+    bool ok = true;
+    const int r = threadIdx.x;
+    if (r < m.P && r != m.me && m.nprod[r] > 0 && m.hlo[r] < m.hhi[r]) {
+        const int slo = m.seg_lo[blockIdx.x], shi = m.seg_hi[blockIdx.x];
+        if (shi >= m.hlo[r] && slo < m.hhi[r]) {
+            const unsigned long long* cnt = reinterpret_cast<const unsigned long long*>(m.win[m.me] + m.off_cnt) + r;
+            const unsigned long long target = (unsigned long long)epoch * (unsigned long long)m.nprod[r];
+            while (ld_acquire_sys64(cnt) < target) {
+                if (*(volatile int*)a.abort_flag) { ok = false; break; }
+                if (gtimer() - t0 > a.timeout_ns) { atomicExch(a.abort_flag, 1); ok = false; break; }
+            }
+        }
+    }
+    fence_proxy_async();     // peer (generic-proxy) stores -> this CTA's bulk copies of the halo
+    return ok;
+}
+
+template <bool MG = false>
 __device__ __forceinline__ bool wait_deps(const SolveArgs& a, unsigned epoch) {
     __shared__ int s_abort;
-    if (a.G == 1 && a.stall_cta < 0) {   // one CTA: its own writes, ordered by the CTA barrier
+    if (a.G == 1 && a.stall_cta < 0 && !(MG && a.mg.P > 1)) {   // one CTA: its own writes, ordered by the CTA barrier
         __syncthreads();
         return true;
     }
@@ -148,6 +219,7 @@ __device__ __forceinline__ bool wait_deps(const SolveArgs& a, unsigned epoch) {
     if (threadIdx.x == 0) s_abort = 0;
     __syncthreads();
     const unsigned long long t0 = gtimer();
+    if (MG && a.mg.P > 1 && !mg_wait_halo(a, epoch, t0)) s_abort = 1;
     for (int h = lo + (int)threadIdx.x; h <= hi; h += blockDim.x) {
         while (ld_acquire(&a.flags[h]) < epoch) {
             if (*(volatile int*)a.abort_flag) { s_abort = 1; break; }
@@ -162,7 +234,14 @@ __device__ __forceinline__ bool wait_deps(const SolveArgs& a, unsigned epoch) {
 
 // K doubles: thread fma chains -> warp butterfly -> tree32 over warps -> slot -> barrier ->
 // tree32 over CTAs.  Every thread returns the grid totals.
-template <int K>
+//
+// Multi-GPU kernel (MG, P ranks): the CTA totals of this rank give the rank partial (tree32 over
+// the rank's CTAs); CTA 0 stores it, tagged with the reduction number, into slot [parity][me] of
+// every rank's window; every CTA of every rank then sums the P rank partials in rank order from
+// +0 (identical on all ranks: the oracle's rank-partitioned plan).  Slots alternate parities: a
+// rank can only publish reduction k+2 after every rank published k+1, i.e. after every CTA of
+// every rank read k.
+template <int K, bool MG = false>
 __device__ __forceinline__ bool grid_reduce(double (&v)[K], const SolveArgs& a, Ctx& c, double* red) {
     const int w = threadIdx.x >> 5, l = threadIdx.x & 31, W = blockDim.x >> 5;
 #pragma unroll
@@ -178,12 +257,51 @@ __device__ __forceinline__ bool grid_reduce(double (&v)[K], const SolveArgs& a, 
             if (l == 0) a.slots[((size_t)c.parity * NSLOT + k) * a.G + blockIdx.x] = ct;
         }
     }
-    const bool ok = grid_barrier(a, c);
-    if (w == 0) {
+    bool ok = grid_barrier(a, c);
+    if (!MG || a.mg.P <= 1) {
+        if (w == 0) {
 #pragma unroll
-        for (int k = 0; k < K; ++k) {
-            const double gt = mfk::tree32(a.slots + ((size_t)c.parity * NSLOT + k) * a.G, a.G);
-            if (l == 0) red[128 + k] = gt;
+            for (int k = 0; k < K; ++k) {
+                const double gt = mfk::tree32(a.slots + ((size_t)c.parity * NSLOT + k) * a.G, a.G);
+                if (l == 0) red[128 + k] = (MG && a.mg.P == 1) ? __dadd_rn(0.0, gt) : gt;
+            }
+        }
+    } else {
+        const MgArgs& m = a.mg;
+        const unsigned tag = ++c.nred;
+        const int par = (int)(tag & 1u);
+        if (blockIdx.x == 0 && w == 0) {
+            double gt[K];
+#pragma unroll
+            for (int k = 0; k < K; ++k) gt[k] = mfk::tree32(a.slots + ((size_t)c.parity * NSLOT + k) * a.G, a.G);
+            if (l < m.P) {
+                double* dst = reinterpret_cast<double*>(m.win[l] + m.off_red) + ((size_t)par * m.P + m.me) * 4;
+#pragma unroll
+                for (int k = 0; k < K; ++k) __stcg(dst + k, gt[k]);
+                st_release_sys(reinterpret_cast<unsigned*>(m.win[l] + m.off_tag) + par * m.P + m.me, tag);
+            }
+        }
+        __shared__ int s_ab;
+        if (threadIdx.x == 0) s_ab = 0;
+        __syncthreads();
+        if ((int)threadIdx.x < m.P) {
+            const unsigned* tg = reinterpret_cast<const unsigned*>(m.win[m.me] + m.off_tag) + par * m.P + threadIdx.x;
+            const unsigned long long t0 = gtimer();
+            while ((int)(ld_acquire_sys(tg) - tag) < 0) {
+                if (*(volatile int*)a.abort_flag) { s_ab = 1; break; }
+                if (gtimer() - t0 > a.timeout_ns) { atomicExch(a.abort_flag, 1); s_ab = 1; break; }
+            }
+        }
+        __syncthreads();
+        if (s_ab) ok = false;
+        if (threadIdx.x == 0) {
+            const double* sl = reinterpret_cast<const double*>(m.win[m.me] + m.off_red) + (size_t)par * m.P * 4;
+#pragma unroll
+            for (int k = 0; k < K; ++k) {
+                double t = 0.0;
+                for (int r = 0; r < m.P; ++r) t = __dadd_rn(t, ld_relaxed_sys_f64(sl + r * 4 + k));
+                red[128 + k] = t;
+            }
         }
     }
     __syncthreads();
@@ -285,6 +403,7 @@ struct Timer {
 
 // The SpMV input of the init phase: x0 in the PV layout (own rows, level FP64), published with
 // epoch 1 and awaited, so that r0 = b - A~ x0 runs through the same staged SpMV.
+template <bool MG = false>
 __device__ __forceinline__ bool stage_x0(const SolveArgs& a, double* PV, int64_t R0, int64_t Rend) {
     for (int64_t i = R0 + threadIdx.x; i < Rend; i += blockDim.x) {
         PV[pv_idx(i)] = a.x[i];
@@ -294,8 +413,8 @@ __device__ __forceinline__ bool stage_x0(const SolveArgs& a, double* PV, int64_t
         }
     }
     // padding rows of the last segment (rows >= n) stay 0 (workspace cleared by the host)
-    publish(a, 1);
-    return wait_deps(a, 1);
+    publish<MG>(a, 1, PV);
+    return wait_deps<MG>(a, 1);
 }
 
 // levels of the own segments of a PV vector (Alg. 4): one half-warp per tile row
@@ -316,7 +435,7 @@ __device__ __forceinline__ void pv_levels(const SolveArgs& a, double* PV, int64_
 //         4 reduce rho', 5 x and p update + levels + publish, 6 init
 // Row mapping of every vector phase: thread t takes rows R0 + t + kB (the plan tree); r_{j+1}
 // replaces mu in shared memory, x_{j+1} = x_j + alpha p_j is applied with the p update.
-template <bool DYN, bool COUNT, bool STK, int MAXT>
+template <bool DYN, bool COUNT, bool STK, int MAXT, bool MG = false>
 __global__ void __launch_bounds__(MAXT, 1) cg_persistent(SolveArgs a) {
     constexpr int PF = MAXT >= 1024 ? 4 : 8;
     Smem sm = carve(a, 1);
@@ -338,7 +457,7 @@ __global__ void __launch_bounds__(MAXT, 1) cg_persistent(SolveArgs a) {
 
     // init: r = b - A~ x0 at TilePrec; partial (b,b), (r,r)
     double v2[2] = {0.0, 0.0};
-    bool ok = stage_x0(a, P, R0, Rend);
+    bool ok = stage_x0<MG>(a, P, R0, Rend);
     mfk::spmv_cta<false, false, PF>(a.A, tr0, tr1, P, 0, sm.sp, 0, nullptr,
                                     [&](int64_t TR, int ln, double ax, double) {
                                         const int64_t i = TR * 16 + ln;
@@ -350,7 +469,7 @@ __global__ void __launch_bounds__(MAXT, 1) cg_persistent(SolveArgs a) {
                                             v2[1] = __fma_rn(ri, ri, v2[1]);
                                         }
                                     });
-    ok = grid_reduce<2>(v2, a, c, sm.red) && ok;     // every CTA's init SpMV is done: P may be overwritten
+    ok = grid_reduce<2, MG>(v2, a, c, sm.red) && ok;     // every CTA's init SpMV is done: P may be overwritten
     const double nb = sqrt(v2[0]);
     double rho = v2[1];
     int64_t j = 0;
@@ -370,14 +489,14 @@ __global__ void __launch_bounds__(MAXT, 1) cg_persistent(SolveArgs a) {
             if (DYN) lv = mfk::hw_min_i(i < n ? mfk::level_of(pv, th) : 4, m);
             if ((i & 15) == 0) mfk::pv_set_level(P, i >> 4, lv);
         }
-        publish(a, 2);
+        publish<MG>(a, 2, P);
         tm.tick(6);
         for (;; ++j) {
             const double relres = __ddiv_rn(sqrt(rho), nb);
             if (blockIdx.x == 0 && t == 0) { if (j < a.hist_cap) a.hist[j] = relres; a.out[2] = relres; }
             if (relres < a.tol) { converged = 1; break; }
             if (j == a.max_iter) break;
-            if (!wait_deps(a, (unsigned)(j + 2))) { status = MF_ERR_DEADLOCK; break; }
+            if (!wait_deps<MG>(a, (unsigned)(j + 2))) { status = MF_ERR_DEADLOCK; break; }
             tm.tick(0);
             // step A: mu = A~_j p_j (own tile rows) with the fused partial (mu, p)
             double sg[1] = {0.0};
@@ -393,7 +512,7 @@ __global__ void __launch_bounds__(MAXT, 1) cg_persistent(SolveArgs a) {
             spmv_counts<COUNT, DYN>(a, c, tr0, tr1, P, sm.ired);
             tm.tick(1);
             // step B: sigma = (mu, p) over the grid -> alpha
-            if (!grid_reduce<1>(sg, a, c, sm.red)) { status = MF_ERR_DEADLOCK; break; }
+            if (!grid_reduce<1, MG>(sg, a, c, sm.red)) { status = MF_ERR_DEADLOCK; break; }
             tm.tick(2);
             const double sigma = sg[0];
             if (!(sigma > 0.0) || !isfinite(sigma)) { status = MF_ERR_BREAKDOWN; break; }
@@ -419,7 +538,7 @@ __global__ void __launch_bounds__(MAXT, 1) cg_persistent(SolveArgs a) {
                 }
             }
             tm.tick(3);
-            if (!grid_reduce<1>(rr, a, c, sm.red)) { status = MF_ERR_DEADLOCK; break; }
+            if (!grid_reduce<1, MG>(rr, a, c, sm.red)) { status = MF_ERR_DEADLOCK; break; }
             tm.tick(4);
             const double beta = __ddiv_rn(rr[0], rho);
             rho = rr[0];
@@ -454,7 +573,7 @@ __global__ void __launch_bounds__(MAXT, 1) cg_persistent(SolveArgs a) {
                     }
                 }
             }
-            publish(a, (unsigned)(j + 3));
+            publish<MG>(a, (unsigned)(j + 3), P);
             tm.tick(5);
         }
     }
@@ -1144,6 +1263,8 @@ MF_DECLARE_PICK(pick_pbicgstab_512);
 MF_DECLARE_PICK(pick_pbicgstab_1024);
 MF_DECLARE_PICK(pick_cgsr_512);
 MF_DECLARE_PICK(pick_cgsr_1024);
+// device-initiated multi-GPU CG (SolveArgs::mg set): no statistics, no sticky variant
+void* pick_cgmg(int maxt, bool dyn);
 
 #define MF_DEFINE_PICK(NAME, KERNEL, MAXT)                                                        \
     void* NAME(bool dyn, bool count, bool sticky) {                                               \

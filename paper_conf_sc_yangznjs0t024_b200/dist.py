@@ -101,6 +101,41 @@ class Comm:
             pass
 
 
+class LocalGroup:
+    """In-process rank group (mf_local_group): `nranks` host threads of this process each drive one
+    rank, all on the current GPU.  Only the device-initiated kernel (dist_mode 2) runs on it; it
+    checks the multi-rank exchange where one GPU is all there is.  Each rank's thread must use its
+    own CUDA stream (torch.cuda.stream), and the ranks' plans must fit the GPU together
+    (grid_ctas <= SMs / nranks)."""
+
+    def __init__(self, nranks: int):
+        from . import _check, lib
+        h = C.c_void_p()
+        _check(lib().mf_local_group_create(int(nranks), C.byref(h)))
+        self._h = h
+        self.size = int(nranks)
+
+    def comm(self, rank: int) -> "LocalComm":
+        return LocalComm(self, rank)
+
+    def close(self):
+        if getattr(self, "_h", None):
+            from . import lib
+            lib().mf_local_group_destroy(self._h)
+            self._h = None
+
+
+class LocalComm(Comm):
+    """Rank `rank` of a LocalGroup (an mf_comm without NCCL)."""
+
+    def __init__(self, group: LocalGroup, rank: int):   # noqa: super().__init__ is the NCCL path
+        from . import _check, lib
+        h = C.c_void_p()
+        _check(lib().mf_comm_create_local(group._h, int(rank), C.byref(h)))
+        self._h = h
+        self.size, self.rank, self.group = group.size, int(rank), group
+
+
 class DistTileMatrix:
     """This rank's rows [row_begin, row_end) of an n_global x n_global matrix
     (mf_tile_matrix_from_csr_dist): device CSR with local rowptr and GLOBAL column ids."""

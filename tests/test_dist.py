@@ -157,15 +157,95 @@ def test_dist_world1_matches_oracle_and_single_kernel(orc):
             ofn = orc.cg if solver == "cg" else orc.bicgstab
             ro = ofn(T, b, mode=2, plan=orc.Plan(g, bb, R), max_iter=2000)
             fn = dist.cg_solve if solver == "cg" else dist.bicgstab_solve
-            res = fn(D, torch.from_numpy(b).cuda(), mode=mf.MODE_DYNAMIC, max_iter=2000)
-            assert res.converged and ro["converged"] and res.iterations == ro["iterations"], name
-            assert np.array_equal(res.history, ro["history"]), name
-            assert np.array_equal(res.x.cpu().numpy(), ro["x"]), name
             Ts = mf.TileMatrix.from_host_csr(A)
             sfn = mf.cg_solve if solver == "cg" else mf.bicgstab_solve
             rs = sfn(Ts, torch.from_numpy(b).cuda(), mode=mf.MODE_DYNAMIC, max_iter=2000)
-            assert torch.equal(rs.x, res.x), name
+            # CG: the device-initiated kernel (dist_mode 2) and the host-orchestrated path (1)
+            for dm in ((2, 1) if solver == "cg" else (1,)):
+                res = fn(D, torch.from_numpy(b).cuda(), mode=mf.MODE_DYNAMIC, max_iter=2000, dist_mode=dm)
+                assert res.converged and ro["converged"] and res.iterations == ro["iterations"], (name, dm)
+                assert np.array_equal(res.history, ro["history"]), (name, dm)
+                assert np.array_equal(res.x.cpu().numpy(), ro["x"]), (name, dm)
+                assert torch.equal(rs.x, res.x), (name, dm)
+            if solver == "bicgstab":
+                with pytest.raises(mf.MFError):
+                    fn(D, torch.from_numpy(b).cuda(), dist_mode=2)
+            Ts.close()
             D.close()
         comm.close()
     finally:
         td.destroy_process_group()
+
+
+def _run_local_group(A, P, ctas, mode, max_iter, switch_eps=None):
+    """P ranks in P threads of this process on cuda:0 (mf_local_group), device-initiated CG."""
+    import threading
+    import paper_conf_sc_yangznjs0t024_b200 as mf
+    bnd = dist.partition_rows(A.n_rows, P, A.rowptr)
+    b = W.rhs_ones(A)
+    grp = dist.LocalGroup(P)
+    out, err = [None] * P, []
+
+    def job(k):
+        try:
+            torch.cuda.set_device(0)
+            st = torch.cuda.Stream()
+            with torch.cuda.stream(st):
+                comm = grp.comm(k)
+                D = dist.DistTileMatrix.from_host_csr(comm, A, bnd[k], bnd[k + 1], grid_ctas=ctas)
+                plan = D.plan()
+                bk = torch.from_numpy(np.ascontiguousarray(b[bnd[k]:bnd[k + 1]])).cuda()
+                r = dist.cg_solve(D, bk, mode=mode, max_iter=max_iter, dist_mode=2, watchdog_ms=20000,
+                                  switch_eps=switch_eps, raise_on_breakdown=False)
+                out[k] = (plan, r.x.cpu().numpy(), r.history, r.iterations, r.converged, r.status, D.dist_info())
+                D.close()
+                comm.close()
+        except Exception as e:   # re-raised in the main thread
+            err.append(e)
+
+    th = [threading.Thread(target=job, args=(k,)) for k in range(P)]
+    for t in th:
+        t.start()
+    for t in th:
+        t.join()
+    grp.close()
+    if err:
+        raise err[0]
+    return bnd, out
+
+
+def _rank_plan(orc, bnd, out):
+    R, Gr = [], [0]
+    B = out[0][0][1]
+    for k, o in enumerate(out):
+        g, bb, Rk = o[0]
+        assert bb == B
+        R.extend((np.asarray(Rk[:-1], np.int64) + bnd[k]).tolist())
+        Gr.append(Gr[-1] + g)
+    R.append(bnd[-1])
+    return orc.Plan(Gr[-1], B, np.array(R, np.int64), rank_ctas=Gr)
+
+
+LOCAL_CASES = [("C2", 24, 2, 8), ("C2", 24, 3, 6), ("C1", 64, 2, 4), ("C4spd", 1 << 13, 3, 8)]
+
+
+@pytest.mark.gpu
+@pytest.mark.parametrize("name,scale,P,ctas", LOCAL_CASES)
+def test_local_group_device_initiated_matches_oracle(orc, name, scale, P, ctas):
+    """P ranks emulated on one GPU run the device-initiated kernel (halo stores into the peers'
+    windows, arrival counters, tagged rank partials): histories and x equal the oracle's emulation
+    of the global matrix under the rank-partitioned plan, bit for bit, in dynamic and static mode."""
+    import paper_conf_sc_yangznjs0t024_b200 as mf
+    A = W.make(name, scale)
+    b = W.rhs_ones(A)
+    T = orc.Tiles(A.n_rows, A.n_cols, A.rowptr, A.colidx, A.vals)
+    for mode in (mf.MODE_DYNAMIC, mf.MODE_STATIC):
+        bnd, out = _run_local_group(A, P, ctas, mode, 400)
+        assert sum(o[6]["halo_segments"] for o in out) > 0          # the ranks really exchange
+        plan = _rank_plan(orc, bnd, out)
+        ro = orc.cg(T, b, mode=2 if mode == mf.MODE_DYNAMIC else 1, plan=plan, max_iter=400)
+        x = np.concatenate([o[1] for o in out])
+        for o in out:
+            assert o[5] == 0 and o[3] == ro["iterations"] and o[4] == ro["converged"], (name, mode)
+            assert np.array_equal(o[2], ro["history"]), (name, mode)
+        assert np.array_equal(x, ro["x"]), (name, mode)
