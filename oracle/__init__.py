@@ -75,7 +75,7 @@ class _Sticky(C.Structure):
 
 class _Ilu(C.Structure):
     _fields_ = [("n", C.c_int64), ("rowptr", C.POINTER(C.c_int64)), ("colidx", C.POINTER(C.c_int32)),
-                ("lu", C.POINTER(C.c_double)), ("diag", C.POINTER(C.c_int64))]
+                ("lu", C.POINTER(C.c_double)), ("diag", C.POINTER(C.c_int64)), ("rb_depth", C.c_int32)]
 
 
 def _p(a, ctype):
@@ -335,7 +335,9 @@ def dot(u, v, plan: Plan | None = None) -> float:
 
 # ------------------------------------------------------------------ ILU(0)
 class ILU0:
-    def __init__(self, rowptr, colidx, vals):
+    """ILU(0) factors.  rb_depth = 0: row-by-row substitution; d > 0: the recursive block
+    SpTRSV of P:166 with d levels of splitting (mf_oracle.c rb_lower / rb_upper)."""
+    def __init__(self, rowptr, colidx, vals, rb_depth: int = 0):
         self.rowptr = np.ascontiguousarray(rowptr, np.int64)
         self.colidx = np.ascontiguousarray(colidx, np.int32)
         vals = _f64(vals)
@@ -348,7 +350,7 @@ class ILU0:
         self._s = _Ilu(self.n, self.rowptr.ctypes.data_as(C.POINTER(C.c_int64)),
                        self.colidx.ctypes.data_as(C.POINTER(C.c_int32)),
                        self.lu.ctypes.data_as(C.POINTER(C.c_double)),
-                       self.diag.ctypes.data_as(C.POINTER(C.c_int64)))
+                       self.diag.ctypes.data_as(C.POINTER(C.c_int64)), int(rb_depth))
 
     def apply(self, r):
         r = _f64(r)

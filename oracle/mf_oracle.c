@@ -26,6 +26,9 @@
  *   orc_cg / orc_bicgstab       numpy.linalg.solve, finite termination, A-orthogonality,
  *                               recurrence gap, x* = 1.
  *   orc_ilu0 / orc_ilu_apply    tridiagonal ILU(0) == exact LU; (LU)_ij == A_ij on pattern.
+ *   rb_lower / rb_upper         (recursive block SpTRSV) exact integer triangular systems
+ *                               solved in Python integers; scipy-free dense back substitution
+ *                               within the forward-error bound; depth 0 == substitution.
  *   orc_pcg / orc_pbicgstab     numpy.linalg.solve on small systems.
  * The dynamic switch's effect on iteration counts is "parity unpinned".
  */
@@ -545,6 +548,7 @@ typedef struct {
 
 typedef struct {            /* optional ILU(0) preconditioner (CSR, L\U in one array) */
     int64_t n; const int64_t* rowptr; const int32_t* colidx; const double* lu; const int64_t* diag;
+    int32_t rb_depth;       /* 0: row-by-row substitution; d > 0: recursive block SpTRSV of depth d */
 } orc_ilu;
 
 static void ilu_apply(const orc_ilu* M, const double* r, double* z);
@@ -834,8 +838,73 @@ int orc_ilu0(int64_t n, const int64_t* rowptr, const int32_t* colidx, const doub
     return ORC_OK;
 }
 
+/* Recursive block SpTRSV ("we recursively divide a triangular matrix into two smaller
+ * triangular blocks and one square block.  The SpTRSV operation is utilized for the triangular
+ * blocks, and SpMV is applied to the square blocks"; the algorithm of [41]).  Readings (DESIGN.md
+ * R27): a block of rows [lo, hi) with hi - lo >= 2 and depth > 0 splits at mid = lo + (hi - lo) / 2;
+ * the square block's SpMV forms s_i = sum_k t_ik v_k over its columns (one fma chain from +0,
+ * ascending k) and the right-hand side is then updated once, rhs_i = rhs_i - s_i; a leaf (depth 0
+ * or one row) is the row-by-row substitution restricted to the columns inside the leaf.
+ *
+ * Lower (unit diagonal, the strict lower part of lu): rows [lo, hi), the contributions of the
+ * columns < lo already subtracted from y[lo..hi) (y holds the right-hand side on entry).
+ * Order: solve(lo, mid); square rows [mid, hi) x columns [lo, mid); solve(mid, hi). */
+static void rb_lower(const orc_ilu* M, double* y, int64_t lo, int64_t hi, int depth) {
+    if (depth == 0 || hi - lo < 2) {
+        for (int64_t i = lo; i < hi; ++i) {
+            double acc = y[i];
+            for (int64_t k = M->rowptr[i]; k < M->diag[i]; ++k)
+                if (M->colidx[k] >= lo) acc = fma(-M->lu[k], y[M->colidx[k]], acc);
+            y[i] = acc;
+        }
+        return;
+    }
+    int64_t mid = lo + (hi - lo) / 2;
+    rb_lower(M, y, lo, mid, depth - 1);
+    for (int64_t i = mid; i < hi; ++i) {                 /* square block: SpMV, then the update */
+        double s = 0.0;
+        for (int64_t k = M->rowptr[i]; k < M->diag[i]; ++k) {
+            int64_t c = M->colidx[k];
+            if (c >= lo && c < mid) s = fma(M->lu[k], y[c], s);
+        }
+        y[i] = y[i] - s;
+    }
+    rb_lower(M, y, mid, hi, depth - 1);
+}
+/* Upper (diagonal u_ii in lu): rows [lo, hi), the contributions of the columns >= hi already
+ * subtracted from z[lo..hi) (z holds the right-hand side on entry).  Order: solve(mid, hi);
+ * square rows [lo, mid) x columns [mid, hi); solve(lo, mid).  Leaf rows descending. */
+static void rb_upper(const orc_ilu* M, double* z, int64_t lo, int64_t hi, int depth) {
+    if (depth == 0 || hi - lo < 2) {
+        for (int64_t i = hi - 1; i >= lo; --i) {
+            double acc = z[i];
+            for (int64_t k = M->diag[i] + 1; k < M->rowptr[i + 1]; ++k)
+                if (M->colidx[k] < hi) acc = fma(-M->lu[k], z[M->colidx[k]], acc);
+            z[i] = acc / M->lu[M->diag[i]];
+        }
+        return;
+    }
+    int64_t mid = lo + (hi - lo) / 2;
+    rb_upper(M, z, mid, hi, depth - 1);
+    for (int64_t i = lo; i < mid; ++i) {
+        double s = 0.0;
+        for (int64_t k = M->diag[i] + 1; k < M->rowptr[i + 1]; ++k) {
+            int64_t c = M->colidx[k];
+            if (c >= mid && c < hi) s = fma(M->lu[k], z[c], s);
+        }
+        z[i] = z[i] - s;
+    }
+    rb_upper(M, z, lo, mid, depth - 1);
+}
+
 static void ilu_apply(const orc_ilu* M, const double* r, double* z) {
     int64_t n = M->n;
+    if (M->rb_depth > 0) {
+        memcpy(z, r, sizeof(double) * (size_t)n);
+        rb_lower(M, z, 0, n, M->rb_depth);
+        rb_upper(M, z, 0, n, M->rb_depth);
+        return;
+    }
     double* y = malloc(sizeof(double) * (size_t)n);
     for (int64_t i = 0; i < n; ++i) {
         double acc = r[i];
