@@ -182,8 +182,28 @@ mf_status mf_levels(const double* v, int64_t n, const double* th, uint8_t* level
 /* (u, v) with the matrix's launch-plan reduction tree; host result. */
 mf_status mf_dot(const mf_tile_matrix* A, const double* u, const double* v, double* out, mf_stream stream);
 
-/* ILU(0) preconditioner of the stored matrix.  z = M^-1 r via SpTRSV kernels. */
+/* ILU(0) preconditioner of the stored matrix.  z = M^-1 r via SpTRSV kernels.
+ * Factorisation on the host (IKJ order, FP64 factors of the stored values; setup, not per iteration).
+ * Triangular solves (mf_precond_opts.sptrsv):
+ *  - MF_SPTRSV_SYNC_FREE: row-by-row substitution, rows grabbed in chunks, per-row ready flags;
+ *  - MF_SPTRSV_RECURSIVE_BLOCK: the recursive block SpTRSV of P:166 ([41]): each triangle of rows
+ *    [lo, hi) splits at mid = lo + 16*floor((hi-lo)/32) into two triangles (solved recursively,
+ *    rb_depth levels; leaves by the sync-free solve) and one square block (an SpMV s = T v, then
+ *    rhs -= s).  mf_precond_apply runs it as one kernel per node (the paper's multi-kernel method);
+ *    the persistent PCG / PBiCGSTAB kernels run the same node sequence with grid barriers between
+ *    nodes.  rb_depth 0 = auto (leaves of about 2^14 rows).  Results equal the oracle's
+ *    rb_lower / rb_upper bit for bit (reading R27).
+ * mf_precond_create(A, kind, ...) == mf_precond_create_ex with sptrsv = MF_SPTRSV_SYNC_FREE. */
+typedef enum { MF_SPTRSV_SYNC_FREE = 0, MF_SPTRSV_RECURSIVE_BLOCK = 1 } mf_sptrsv_algo;
+typedef struct {
+    mf_precond_kind kind;   /* MF_PRECOND_ILU0 */
+    int32_t sptrsv;         /* mf_sptrsv_algo */
+    int32_t rb_depth;       /* recursive block levels, 1..24; 0 = auto */
+} mf_precond_opts;
 mf_status mf_precond_create(const mf_tile_matrix* A, mf_precond_kind kind, mf_stream stream, mf_precond** out);
+mf_status mf_precond_create_ex(const mf_tile_matrix* A, const mf_precond_opts* opts, mf_stream stream, mf_precond** out);
+/* host: recursive block depth (0 = sync-free), nodes of the L and U trees */
+mf_status mf_precond_info(const mf_precond* M, int32_t* rb_depth, int32_t* nodes_l, int32_t* nodes_u);
 mf_status mf_precond_destroy(mf_precond* M);
 mf_status mf_precond_apply(const mf_precond* M, const double* r, double* z, mf_stream stream);
 

@@ -32,7 +32,8 @@ STATUS = {0: "MF_OK", 1: "MF_ERR_INVALID_ARG", 2: "MF_ERR_UNSORTED_CSR", 3: "MF_
 # every symbol include/mf.h declares
 SYMBOLS = ["mf_default_convert_opts", "mf_default_solve_opts", "mf_set_allocator", "mf_tile_matrix_from_csr",
            "mf_tile_matrix_destroy", "mf_tile_matrix_info", "mf_tile_matrix_export", "mf_spmv", "mf_levels",
-           "mf_dot", "mf_precond_create", "mf_precond_destroy", "mf_precond_apply", "mf_cg_solve",
+           "mf_dot", "mf_precond_create", "mf_precond_create_ex", "mf_precond_info", "mf_precond_destroy",
+           "mf_precond_apply", "mf_cg_solve",
            "mf_bicgstab_solve", "mf_cg_update_xr", "mf_cg_update_p", "mf_status_string", "mf_last_error",
            "mf_abi_version", "mf_nccl_unique_id", "mf_comm_create", "mf_comm_destroy", "mf_comm_info",
            "mf_tile_matrix_from_csr_dist", "mf_cg_solve_dist", "mf_bicgstab_solve_dist", "mf_dist_info", "mf_dist_plan",
@@ -151,6 +152,8 @@ def lib():
         L.mf_levels.argtypes = [vp, i64, vp, vp, vp]
         L.mf_dot.argtypes = [vp, vp, vp, C.POINTER(d), vp]
         L.mf_precond_create.argtypes = [vp, C.c_int, vp, C.POINTER(vp)]
+        L.mf_precond_create_ex.argtypes = [vp, C.POINTER(PrecondOpts), vp, C.POINTER(vp)]
+        L.mf_precond_info.argtypes = [vp, C.POINTER(i32), C.POINTER(i32), C.POINTER(i32)]
         L.mf_precond_destroy.argtypes = [vp]
         L.mf_precond_apply.argtypes = [vp, vp, vp, vp]
         L.mf_cg_solve.argtypes = [vp, vp, vp, C.POINTER(SolveOpts), C.POINTER(SolveInfo), vp]
@@ -391,15 +394,29 @@ def bicgstab_solve(A: TileMatrix, b, **kw) -> SolveResult:
     return _solve(lib().mf_bicgstab_solve, A, b, **kw)
 
 
-class Precond:
-    """ILU(0) of the stored matrix; z = M^-1 r by SpTRSV kernels."""
+SPTRSV_SYNC_FREE, SPTRSV_RECURSIVE_BLOCK = 0, 1
 
-    def __init__(self, A: TileMatrix, kind: int = 1, stream=None):
+
+class PrecondOpts(C.Structure):
+    _fields_ = [("kind", C.c_int), ("sptrsv", C.c_int32), ("rb_depth", C.c_int32)]
+
+
+class Precond:
+    """ILU(0) of the stored matrix; z = M^-1 r by SpTRSV kernels.  sptrsv =
+    SPTRSV_RECURSIVE_BLOCK selects the recursive block SpTRSV of P:166 (rb_depth levels, 0 = auto)."""
+
+    def __init__(self, A: TileMatrix, kind: int = 1, stream=None, sptrsv: int = SPTRSV_SYNC_FREE, rb_depth: int = 0):
         h = C.c_void_p()
         self._h = None
-        _check(lib().mf_precond_create(A._h, int(kind), _stream_ptr(stream), C.byref(h)))
+        o = PrecondOpts(int(kind), int(sptrsv), int(rb_depth))
+        _check(lib().mf_precond_create_ex(A._h, C.byref(o), _stream_ptr(stream), C.byref(h)))
         self._h = h
         self.n = A.n_rows
+
+    def info(self) -> dict:
+        d, nl, nu = C.c_int32(), C.c_int32(), C.c_int32()
+        _check(lib().mf_precond_info(self._h, C.byref(d), C.byref(nl), C.byref(nu)))
+        return {"rb_depth": d.value, "nodes_l": nl.value, "nodes_u": nu.value}
 
     def apply(self, r, out=None, stream=None):
         import torch

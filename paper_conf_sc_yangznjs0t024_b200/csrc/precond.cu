@@ -151,6 +151,52 @@ __global__ void __launch_bounds__(256) sptrsv_kernel(TriCSR T, const double* __r
                                     abort_flag, 20ull * 1000000000ull);
 }
 
+__global__ void __launch_bounds__(256) rb_square_kernel(const int64_t* __restrict__ rp, const int32_t* __restrict__ ci,
+                                                        const double* __restrict__ val, int64_t r0, int64_t r1, double* v) {
+    mfk::rb_square_rows(rp, ci, val, r0, r1, v, (int64_t)blockIdx.x * blockDim.x + threadIdx.x, (int64_t)gridDim.x * blockDim.x);
+}
+
+// Recursive block partition of a factor (precond.cuh RbNode; oracle rb_lower / rb_upper).
+// M: the ILU(0) factors in one CSR (columns ascending per row), diag[i] = position of a_ii.
+struct RbHost {
+    std::vector<RbNode> nodes;
+    std::vector<int64_t> rp;
+    std::vector<int32_t> ci;
+    std::vector<double> v;
+    int nleaves = 0;
+};
+int64_t rb_mid(int64_t lo, int64_t hi) { return lo + 16 * ((hi - lo) / 32); }
+// one node: rows [r0, r1), entries of row i with column in [c0, c1) (and, for leaves, in the
+// strict triangle), columns stored minus `cshift`
+void rb_emit(RbHost& T, const HostCSR& M, const std::vector<int64_t>& diag, bool lower, bool leaf, int64_t r0, int64_t r1,
+             int64_t c0, int64_t c1, int64_t cshift) {
+    RbNode nd{r0, r1, (int64_t)T.rp.size(), leaf ? 1 : 0, leaf ? T.nleaves++ : -1};
+    T.nodes.push_back(nd);
+    for (int64_t i = r0; i < r1; ++i) {
+        T.rp.push_back((int64_t)T.ci.size());
+        const int64_t q0 = lower ? M.rp[i] : diag[i] + 1, q1 = lower ? diag[i] : M.rp[i + 1];
+        for (int64_t q = q0; q < q1; ++q) {
+            const int64_t c = M.ci[q];
+            if (c >= c0 && c < c1) { T.ci.push_back((int32_t)(c - cshift)); T.v.push_back(M.v[q]); }
+        }
+    }
+    T.rp.push_back((int64_t)T.ci.size());
+}
+void rb_lower(RbHost& T, const HostCSR& M, const std::vector<int64_t>& diag, int64_t lo, int64_t hi, int depth) {
+    if (depth == 0 || hi - lo < 32) { rb_emit(T, M, diag, true, true, lo, hi, lo, hi, lo); return; }
+    const int64_t mid = rb_mid(lo, hi);
+    rb_lower(T, M, diag, lo, mid, depth - 1);
+    rb_emit(T, M, diag, true, false, mid, hi, lo, mid, 0);
+    rb_lower(T, M, diag, mid, hi, depth - 1);
+}
+void rb_upper(RbHost& T, const HostCSR& M, const std::vector<int64_t>& diag, int64_t lo, int64_t hi, int depth) {
+    if (depth == 0 || hi - lo < 32) { rb_emit(T, M, diag, false, true, lo, hi, lo, hi, lo); return; }
+    const int64_t mid = rb_mid(lo, hi);
+    rb_upper(T, M, diag, mid, hi, depth - 1);
+    rb_emit(T, M, diag, false, false, lo, mid, mid, hi, 0);
+    rb_upper(T, M, diag, lo, mid, depth - 1);
+}
+
 template <class T>
 mf_status upload(T** d, const std::vector<T>& h, cudaStream_t s) {
     MF_TRY(alloc(d, h.size(), s));
@@ -171,6 +217,39 @@ mf_status run_precond_apply(Precond& P, const double* r, double* z, cudaStream_t
     }
     const unsigned e = ++P.epoch;
     const int blocks = (int)std::min<int64_t>((P.n + 255) / 256, (int64_t)sms * 8);
+    if (P.rb_depth > 0) {
+        // the multi-kernel recursive block SpTRSV: one launch per node, in place on y
+        const int nctr = P.Lrb.nleaves + P.Urb.nleaves;
+        MF_CUDA(cudaMemsetAsync(P.ctr, 0, (size_t)(nctr + 1) * sizeof(unsigned long long), s));
+        int* abort_flag = reinterpret_cast<int*>(P.ctr + nctr);
+        MF_CUDA(cudaMemcpyAsync(P.y, r, P.n * sizeof(double), cudaMemcpyDeviceToDevice, s));
+        for (int pass = 0; pass < 2; ++pass) {
+            const RbTree& T = pass == 0 ? P.Lrb : P.Urb;
+            for (const RbNode& nd : T.h) {
+                const int64_t m = nd.r1 - nd.r0;
+                const int nb = (int)std::max<int64_t>(1, std::min<int64_t>((m + 255) / 256, (int64_t)sms * 8));
+                if (nd.leaf) {
+                    unsigned long long* c = P.ctr + (pass == 0 ? 0 : P.Lrb.nleaves) + nd.leaf_idx;
+                    if (pass == 0)
+                        sptrsv_kernel<true><<<nb, 256, 0, s>>>(TriCSR{T.rp + nd.rp_off, T.ci, T.v}, nullptr, m, P.y + nd.r0,
+                                                               P.y + nd.r0, P.flags + nd.r0, 2 * e + 1, 0u, c, abort_flag);
+                    else
+                        sptrsv_kernel<false><<<nb, 256, 0, s>>>(TriCSR{T.rp + nd.rp_off, T.ci, T.v}, P.udiag + nd.r0, m,
+                                                                P.y + nd.r0, P.y + nd.r0, P.flags + nd.r0, 2 * e + 2, 0u, c,
+                                                                abort_flag);
+                } else {
+                    rb_square_kernel<<<nb, 256, 0, s>>>(T.rp + nd.rp_off, T.ci, T.v, nd.r0, nd.r1, P.y);
+                }
+            }
+        }
+        MF_CUDA(cudaGetLastError());
+        MF_CUDA(cudaMemcpyAsync(z, P.y, P.n * sizeof(double), cudaMemcpyDeviceToDevice, s));
+        int ab = 0;
+        MF_CUDA(cudaMemcpyAsync(&ab, abort_flag, sizeof(int), cudaMemcpyDeviceToHost, s));
+        MF_CUDA(cudaStreamSynchronize(s));
+        if (ab) return fail(MF_ERR_DEADLOCK, "triangular-solve watchdog expired");
+        return MF_OK;
+    }
     MF_CUDA(cudaMemsetAsync(P.ctr, 0, 3 * sizeof(unsigned long long), s));
     int* abort_flag = reinterpret_cast<int*>(P.ctr + 2);
     sptrsv_kernel<true><<<blocks, 256, 0, s>>>(P.L, nullptr, P.n, r, P.y, P.flags, 2 * e + 1, 0u, P.ctr, abort_flag);
@@ -185,13 +264,15 @@ mf_status run_precond_apply(Precond& P, const double* r, double* z, cudaStream_t
 
 void destroy_precond(Precond* P) {
     cudaStream_t s = P->owner_stream;
-    void* ptrs[] = {P->L.rp, P->L.ci, P->L.v, P->U.rp, P->U.ci, P->U.v, P->udiag, P->flags, P->ctr, P->y, P->z};
+    void* ptrs[] = {P->L.rp, P->L.ci, P->L.v, P->U.rp, P->U.ci, P->U.v, P->udiag, P->flags, P->ctr, P->y, P->z,
+                    P->Lrb.nodes, P->Lrb.rp, P->Lrb.ci, P->Lrb.v, P->Urb.nodes, P->Urb.rp, P->Urb.ci, P->Urb.v};
     for (void* p : ptrs) if (p) dev_free(p, s);
     *P = Precond();
 }
 
-mf_status build_precond(const TileMatrix& A, cudaStream_t s, Precond* P) {
+mf_status build_precond(const TileMatrix& A, int rb_depth, cudaStream_t s, Precond* P) {
     if (A.n_rows != A.n_cols) return fail(MF_ERR_INVALID_ARG, "ILU(0) needs a square matrix");
+    if (rb_depth < 0 || rb_depth > 24) return fail(MF_ERR_INVALID_ARG, "rb_depth must be in [0, 24]");
     P->owner_stream = s;
     P->n = A.n_rows;
     HostCSR M;
@@ -212,12 +293,30 @@ mf_status build_precond(const TileMatrix& A, cudaStream_t s, Precond* P) {
     MF_TRY(upload(&P->L.rp, lrp, s)); MF_TRY(upload(&P->L.ci, lci, s)); MF_TRY(upload(&P->L.v, lv, s));
     MF_TRY(upload(&P->U.rp, urp, s)); MF_TRY(upload(&P->U.ci, uci, s)); MF_TRY(upload(&P->U.v, uv, s));
     MF_TRY(upload(&P->udiag, ud, s));
+    int nctr = 4;
+    P->rb_depth = rb_depth;
+    if (rb_depth > 0) {
+        RbHost HL, HU;
+        rb_lower(HL, M, diag, 0, n, rb_depth);
+        rb_upper(HU, M, diag, 0, n, rb_depth);
+        for (int k = 0; k < 2; ++k) {
+            RbHost& H = k == 0 ? HL : HU;
+            RbTree& T = k == 0 ? P->Lrb : P->Urb;
+            MF_TRY(upload(&T.nodes, H.nodes, s));
+            MF_TRY(upload(&T.rp, H.rp, s));
+            MF_TRY(upload(&T.ci, H.ci, s));
+            MF_TRY(upload(&T.v, H.v, s));
+            T.h = H.nodes;
+            T.nleaves = H.nleaves;
+        }
+        nctr = std::max(nctr, HL.nleaves + HU.nleaves + 1);
+    }
     MF_TRY(alloc(&P->flags, (size_t)n + 1, s));
-    MF_TRY(alloc(&P->ctr, 4, s));
+    MF_TRY(alloc(&P->ctr, (size_t)nctr, s));
     MF_TRY(alloc(&P->y, n, s));
     MF_TRY(alloc(&P->z, n, s));
     MF_CUDA(cudaMemsetAsync(P->flags, 0, (n + 1) * sizeof(unsigned), s));
-    MF_CUDA(cudaMemsetAsync(P->ctr, 0, 4 * sizeof(unsigned long long), s));
+    MF_CUDA(cudaMemsetAsync(P->ctr, 0, (size_t)nctr * sizeof(unsigned long long), s));
     MF_CUDA(cudaStreamSynchronize(s));
     P->nnz_l = (int64_t)lv.size();
     P->nnz_u = (int64_t)uv.size();
@@ -233,19 +332,44 @@ using namespace mf;
 extern "C" {
 
 mf_status mf_precond_create(const mf_tile_matrix* A, mf_precond_kind kind, mf_stream stream, mf_precond** out) {
-    if (!A || !out) return fail(MF_ERR_INVALID_ARG, "NULL argument");
+    mf_precond_opts o{kind, 0, 0};
+    return mf_precond_create_ex(A, &o, stream, out);
+}
+
+mf_status mf_precond_create_ex(const mf_tile_matrix* A, const mf_precond_opts* opts, mf_stream stream, mf_precond** out) {
+    if (!A || !out || !opts) return fail(MF_ERR_INVALID_ARG, "NULL argument");
     *out = nullptr;
+    const mf_precond_kind kind = opts->kind;
     if (kind != MF_PRECOND_ILU0) return fail(MF_ERR_INVALID_ARG, "only MF_PRECOND_ILU0 is defined (P:164)");
+    if (opts->sptrsv != MF_SPTRSV_SYNC_FREE && opts->sptrsv != MF_SPTRSV_RECURSIVE_BLOCK)
+        return fail(MF_ERR_INVALID_ARG, "sptrsv must be MF_SPTRSV_SYNC_FREE or MF_SPTRSV_RECURSIVE_BLOCK");
+    int depth = 0;
+    if (opts->sptrsv == MF_SPTRSV_RECURSIVE_BLOCK) {
+        depth = opts->rb_depth;
+        if (depth == 0) {   // auto: leaves of about 2^14 rows, at least one split
+            depth = 1;
+            while (depth < 12 && (A->m.n_rows >> (depth + 1)) >= 16384) ++depth;
+        }
+        if (depth < 1 || depth > 24) return fail(MF_ERR_INVALID_ARG, "rb_depth must be in [1, 24] (0 = auto)");
+    }
     MF_TRY(check_device(nullptr));
     mf_precond* h = new (std::nothrow) mf_precond();
     if (!h) return fail(MF_ERR_OOM, "host allocation failed");
-    mf_status st = build_precond(A->m, (cudaStream_t)stream, &h->p);
+    mf_status st = build_precond(A->m, depth, (cudaStream_t)stream, &h->p);
     if (st != MF_OK) {
         destroy_precond(&h->p);
         delete h;
         return st;
     }
     *out = h;
+    return MF_OK;
+}
+
+mf_status mf_precond_info(const mf_precond* M, int32_t* rb_depth, int32_t* nodes_l, int32_t* nodes_u) {
+    if (!M) return fail(MF_ERR_INVALID_ARG, "NULL argument");
+    if (rb_depth) *rb_depth = M->p.rb_depth;
+    if (nodes_l) *nodes_l = (int32_t)M->p.Lrb.h.size();
+    if (nodes_u) *nodes_u = (int32_t)M->p.Urb.h.size();
     return MF_OK;
 }
 

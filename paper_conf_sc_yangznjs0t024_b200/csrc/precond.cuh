@@ -1,6 +1,8 @@
 // precond.cuh -- ILU(0) factors on the device and the sync-free triangular solve.
 #pragma once
 
+#include <vector>
+
 #include "mf_internal.cuh"
 
 namespace mf {
@@ -11,8 +13,33 @@ struct TriCSR {
     double* v = nullptr;
 };
 
+// Recursive block SpTRSV (the algorithm of [41]; oracle rb_lower / rb_upper, reading R27):
+// the triangle of rows [lo, hi) splits at mid = lo + 16 * floor((hi - lo) / 32) into two triangles
+// and one square block, down to `depth` levels (or fewer than 32 rows).  The nodes are stored in
+// execution order: lower  = solve(lo, mid), square rows [mid, hi) x cols [lo, mid), solve(mid, hi);
+// upper = solve(mid, hi), square rows [lo, mid) x cols [mid, hi), solve(lo, mid).  Each node owns a
+// CSR slice of the factor: a leaf the entries with both row and column inside it (columns stored
+// relative to r0, so the leaf is a standalone triangular solve), a square the entries of its
+// rectangle (global columns).
+struct RbNode {
+    int64_t r0, r1;      // rows [r0, r1)
+    int64_t rp_off;      // first of the node's (r1 - r0 + 1) row pointers in the tree's rp array
+    int32_t leaf;        // 1 triangle, 0 square block
+    int32_t leaf_idx;    // leaves: ordinal among the tree's leaves; squares: -1
+};
+struct RbTree {
+    RbNode* nodes = nullptr;       // device copy
+    std::vector<RbNode> h;         // host copy (execution order)
+    int64_t* rp = nullptr;
+    int32_t* ci = nullptr;
+    double* v = nullptr;
+    int nleaves = 0;
+};
+
 struct Precond {
     int64_t n = 0;
+    int rb_depth = 0;             // 0: sync-free substitution; > 0: recursive block SpTRSV
+    RbTree Lrb, Urb;
     TriCSR L, U;                  // L: strict lower part (unit diagonal implied); U: strict upper part
     double* udiag = nullptr;      // u_ii
     unsigned* flags = nullptr;    // [n+1] row-ready epochs (forward 2e+1, backward 2e+2)
@@ -24,7 +51,7 @@ struct Precond {
     cudaStream_t owner_stream = nullptr;
 };
 
-mf_status build_precond(const TileMatrix& A, cudaStream_t s, Precond* P);
+mf_status build_precond(const TileMatrix& A, int rb_depth, cudaStream_t s, Precond* P);
 void destroy_precond(Precond* P);
 mf_status run_precond_apply(Precond& P, const double* r, double* z, cudaStream_t s);
 
@@ -127,6 +154,21 @@ __device__ void sptrsv_chunked(const int64_t* __restrict__ rp, const int32_t* __
             ready[t] = 1;
             st_release_u32(&flags[i], flag_val);
         }
+    }
+}
+
+// Square block of the recursive block SpTRSV ("SpMV is applied to the square blocks"): rows
+// [r0, r1) of the node, one thread per row: s = sum_k t_ik v_k (one fma chain from +0, ascending k),
+// then v_i = v_i - s (in place on the solve's vector).  Rows i = r0 + first + k*stride.
+__device__ __forceinline__ void rb_square_rows(const int64_t* __restrict__ rp, const int32_t* __restrict__ ci,
+                                               const double* __restrict__ val, int64_t r0, int64_t r1, double* v,
+                                               int64_t first, int64_t stride) {
+    for (int64_t i = r0 + first; i < r1; i += stride) {
+        const int64_t lo = rp[i - r0], hi = rp[i - r0 + 1];
+        if (lo == hi) continue;                   // v_i - (+0) == v_i
+        double sacc = 0.0;
+        for (int64_t q = lo; q < hi; ++q) sacc = __fma_rn(val[q], __ldcg(v + ci[q]), sacc);
+        v[i] = __dsub_rn(__ldcg(v + i), sacc);
     }
 }
 

@@ -440,6 +440,11 @@ mf_status run_solve(const TileMatrix& A, bool bicg, const double* b, double* x, 
         a.Lrp = P->L.rp; a.Lci = P->L.ci; a.Lv = P->L.v;
         a.Urp = P->U.rp; a.Uci = P->U.ci; a.Uv = P->U.v; a.Ud = P->udiag;
         a.pflags = P->flags; a.pctr = P->ctr; a.py = P->y; a.pz = pz; a.ps = psh;
+        if (P->rb_depth > 0) {
+            a.rb = 1;
+            a.Lnodes = P->Lrb.nodes; a.nLn = (int)P->Lrb.h.size(); a.Lbrp = P->Lrb.rp; a.Lbci = P->Lrb.ci; a.Lbv = P->Lrb.v;
+            a.Unodes = P->Urb.nodes; a.nUn = (int)P->Urb.h.size(); a.Ubrp = P->Urb.rp; a.Ubci = P->Urb.ci; a.Ubv = P->Urb.v;
+        }
     }
 
     if (mgl) {

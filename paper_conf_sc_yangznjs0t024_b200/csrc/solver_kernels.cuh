@@ -75,6 +75,10 @@ struct SolveArgs {
     double* pz;                  // PCG: z (normal); PBiCGSTAB: p^ (PV)
     double* ps;                  // PBiCGSTAB: s^ (PV)
     unsigned pe0;                // epoch of the first apply of this solve
+    // recursive block SpTRSV (rb == 0: sync-free substitution over the whole factor)
+    int rb;
+    const RbNode* Lnodes; int nLn; const int64_t* Lbrp; const int32_t* Lbci; const double* Lbv;
+    const RbNode* Unodes; int nUn; const int64_t* Ubrp; const int32_t* Ubci; const double* Ubv;
     MgArgs mg;                   // multi-GPU single kernel (P == 0: off)
 };
 
@@ -934,9 +938,57 @@ struct PcState {
     unsigned apply = 0;
 };
 
+// Recursive block SpTRSV inside the persistent kernel: the node sequence of the
+// precond.cuh trees in place on py (in copied to py first, py copied to out at the end); a leaf is
+// the sync-free chunked solve of its rows (all CTAs grab chunks), a square block is spread over
+// all CTAs' threads (one thread per row); a grid barrier separates consecutive nodes.
 template <bool OUTPV>
-__device__ __forceinline__ bool precond_apply(const SolveArgs& a, PcState& ps, const Smem& sm, const double* in, double* out,
-                                              int64_t R0, int64_t Rend) {
+__device__ __noinline__ bool precond_apply_rb(const SolveArgs& a, PcState& ps, const Smem& sm, Ctx& c, const double* in,
+                                              double* out, int64_t R0, int64_t Rend) {
+    const unsigned e = a.pe0 + ps.apply++;
+    const unsigned vf = 2 * e + 1, vb = 2 * e + 2;
+    const int B = blockDim.x;
+    for (int64_t i = R0 + threadIdx.x; i < Rend; i += B) a.py[i] = in[i];
+    bool ok = grid_barrier(a, c);
+    for (int pass = 0; pass < 2 && ok; ++pass) {
+        const RbNode* nodes = pass == 0 ? a.Lnodes : a.Unodes;
+        const int nn = pass == 0 ? a.nLn : a.nUn;
+        const int64_t* brp = pass == 0 ? a.Lbrp : a.Ubrp;
+        const int32_t* bci = pass == 0 ? a.Lbci : a.Ubci;
+        const double* bv = pass == 0 ? a.Lbv : a.Ubv;
+        for (int k = 0; k < nn && ok; ++k) {
+            const RbNode nd = nodes[k];
+            const int64_t m = nd.r1 - nd.r0;
+            if (nd.leaf) {
+                const int64_t nch = (m + B - 1) / B;
+                if (pass == 0) {
+                    mfk::sptrsv_chunked<true, false>(brp + nd.rp_off, bci, bv, nullptr, m, a.py + nd.r0, a.py + nd.r0,
+                                                     a.pflags + nd.r0, vf, 0u, a.pctr, ps.base_f, sm.tys, sm.tready, sm.tchunk,
+                                                     a.abort_flag, a.timeout_ns);
+                    ps.base_f += (unsigned long long)(nch + a.G);
+                } else {
+                    mfk::sptrsv_chunked<false, false>(brp + nd.rp_off, bci, bv, a.Ud + nd.r0, m, a.py + nd.r0, a.py + nd.r0,
+                                                      a.pflags + nd.r0, vb, 0u, a.pctr + 1, ps.base_b, sm.tys, sm.tready,
+                                                      sm.tchunk, a.abort_flag, a.timeout_ns);
+                    ps.base_b += (unsigned long long)(nch + a.G);
+                }
+            } else {
+                mfk::rb_square_rows(brp + nd.rp_off, bci, bv, nd.r0, nd.r1, a.py, (int64_t)blockIdx.x * B + threadIdx.x,
+                                    (int64_t)a.G * B);
+            }
+            __threadfence();
+            ok = grid_barrier(a, c) && *(volatile int*)a.abort_flag == 0;
+        }
+    }
+    for (int64_t i = R0 + threadIdx.x; i < Rend; i += B) out[OUTPV ? pv_idx(i) : i] = __ldcg(a.py + i);
+    __syncthreads();
+    return ok;
+}
+
+template <bool OUTPV>
+__device__ __forceinline__ bool precond_apply(const SolveArgs& a, PcState& ps, const Smem& sm, Ctx& c, const double* in,
+                                              double* out, int64_t R0, int64_t Rend) {
+    if (a.rb) return precond_apply_rb<OUTPV>(a, ps, sm, c, in, out, R0, Rend);
     const unsigned e = a.pe0 + ps.apply++;
     const unsigned vf = 2 * e + 1, vb = 2 * e + 2;
     const int64_t nch = (a.n + blockDim.x - 1) / blockDim.x;
@@ -999,7 +1051,7 @@ __global__ void __launch_bounds__(MAXT, 1) pcg_persistent(SolveArgs a) {
         converged = 1;
         if (blockIdx.x == 0 && t == 0 && a.hist_cap > 0) a.hist[0] = 0.0;
     } else if (ok) {
-        if (!precond_apply<false>(a, pcs, sm, Rv, Z, R0, Rend)) status = MF_ERR_DEADLOCK;
+        if (!precond_apply<false>(a, pcs, sm, c, Rv, Z, R0, Rend)) status = MF_ERR_DEADLOCK;
         double v3[2] = {0.0, 0.0};
         for (int64_t li = t; li < nr; li += B) {
             const int64_t i = R0 + li;
@@ -1051,7 +1103,7 @@ __global__ void __launch_bounds__(MAXT, 1) pcg_persistent(SolveArgs a) {
             if (!grid_reduce<1>(r1, a, c, sm.red)) { status = MF_ERR_DEADLOCK; break; }   // r complete too
             rr = r1[0];
             tm.tick(4);
-            if (!precond_apply<false>(a, pcs, sm, Rv, Z, R0, Rend)) { status = MF_ERR_DEADLOCK; break; }
+            if (!precond_apply<false>(a, pcs, sm, c, Rv, Z, R0, Rend)) { status = MF_ERR_DEADLOCK; break; }
             tm.tick(5);
             double rz[1] = {0.0};
             for (int64_t li = t; li < nr; li += B) {
@@ -1143,7 +1195,7 @@ __global__ void __launch_bounds__(MAXT, 1) pbicgstab_persistent(SolveArgs a) {
             if (relres < a.tol) { converged = 1; break; }
             if (j == a.max_iter) break;
             // p^ = M^-1 p (p complete: the previous grid reduction / the init reduction)
-            if (!precond_apply<true>(a, pcs, sm, P, PH, R0, Rend)) { status = MF_ERR_DEADLOCK; break; }
+            if (!precond_apply<true>(a, pcs, sm, c, P, PH, R0, Rend)) { status = MF_ERR_DEADLOCK; break; }
             if (j == 0) {          // tau from ||p^_0|| (the first SpMV input)
                 double pp[1] = {0.0};
                 for (int64_t li = t; li < nr; li += B) { const double v = PH[pv_idx(R0 + li)]; pp[0] = __fma_rn(v, v, pp[0]); }
@@ -1172,7 +1224,7 @@ __global__ void __launch_bounds__(MAXT, 1) pbicgstab_persistent(SolveArgs a) {
             }
             if (!grid_barrier(a, c)) { status = MF_ERR_DEADLOCK; break; }    // s complete
             tm.tick(3);
-            if (!precond_apply<true>(a, pcs, sm, S, SH, R0, Rend)) { status = MF_ERR_DEADLOCK; break; }
+            if (!precond_apply<true>(a, pcs, sm, c, S, SH, R0, Rend)) { status = MF_ERR_DEADLOCK; break; }
             pv_levels<DYN>(a, SH, tr0, tr1, th);
             publish(a, ++epoch);
             if (!wait_deps(a, epoch)) { status = MF_ERR_DEADLOCK; break; }

@@ -343,6 +343,63 @@ def test_preconditioned_solve_parity(mf, orc, name, make, solver, mode, G, B):
     assert np.array_equal(rg2.x.cpu().numpy(), ro["x"])
 
 
+RB_APPLY_CASES = [("C4spd-14", lambda: W.make("C4spd", 1 << 14), [1, 3, 0]),
+                  ("C4ind-13", lambda: W.make("C4ind", 1 << 13), [2, 6]),
+                  ("ragged-1000", lambda: W.suitesparse_like(1000, seed=8, spd=False), [1, 4, 20]),
+                  ("C2-16", lambda: W.make("C2", 16), [3])]
+
+
+@pytest.mark.parametrize("name,make,depths", RB_APPLY_CASES, ids=[c[0] for c in RB_APPLY_CASES])
+def test_rb_precond_apply_bit_exact(mf, orc, name, make, depths):
+    """Recursive block SpTRSV (reading R27), multi-kernel apply: z bit-identical to the
+    oracle's rb_lower / rb_upper at the same depth (auto depth: the depth the library reports)."""
+    A = make()
+    T = oracle_tiles(orc, A)
+    rp, ci, sv = T.stored_csr()
+    G = mf.TileMatrix.from_host_csr(A)
+    rng = np.random.default_rng(7)
+    for d in depths:
+        P = mf.Precond(G, sptrsv=mf.SPTRSV_RECURSIVE_BLOCK, rb_depth=d)
+        inf = P.info()
+        assert inf["rb_depth"] == (d if d else inf["rb_depth"]) and inf["rb_depth"] >= 1
+        M = orc.ILU0(rp, ci, sv, rb_depth=inf["rb_depth"])
+        for _ in range(2):
+            r = rng.standard_normal(A.n_rows)
+            assert np.array_equal(P.apply(dev(r)).cpu().numpy(), M.apply(r))
+        P.close()
+
+
+RB_SOLVE_CASES = [
+    ("C4spd-13-dyn-rb3", lambda: W.make("C4spd", 1 << 13), "cg", 2, 3, 6, 256),
+    ("C4spd-14-static-rb2", lambda: W.make("C4spd", 1 << 14), "cg", 1, 2, 0, 0),
+    ("C4ind-13-dyn-rb4", lambda: W.make("C4ind", 1 << 13), "bicgstab", 2, 4, 5, 128),
+    ("C3-48-pbicg-rb2", lambda: W.make("C3", 48), "bicgstab", 2, 2, 3, 256),
+]
+
+
+@pytest.mark.parametrize("name,make,solver,mode,depth,G,B", RB_SOLVE_CASES, ids=[c[0] for c in RB_SOLVE_CASES])
+def test_rb_preconditioned_solve_parity(mf, orc, name, make, solver, mode, depth, G, B):
+    """PCG / PBiCGSTAB with the recursive block SpTRSV inside the persistent kernel (node sequence
+    with grid barriers): histories and x bit-identical to the oracle at the same depth."""
+    A = make()
+    b = W.rhs_ones(A)
+    Gm = mf.TileMatrix.from_host_csr(A, grid_ctas=G, block_threads=B)
+    g, bb, R = Gm.plan()
+    T = oracle_tiles(orc, A)
+    rp, ci, sv = T.stored_csr()
+    M = orc.ILU0(rp, ci, sv, rb_depth=depth)
+    P = mf.Precond(Gm, sptrsv=mf.SPTRSV_RECURSIVE_BLOCK, rb_depth=depth)
+    ofn = orc.cg if solver == "cg" else orc.bicgstab
+    gfn = mf.cg_solve if solver == "cg" else mf.bicgstab_solve
+    ro = ofn(T, b, M=M, mode=mode, plan=orc.Plan(g, bb, R), max_iter=500)
+    rg = gfn(Gm, dev(b), M=P, mode=mode, max_iter=500)
+    assert ro["converged"] and rg.converged and rg.iterations == ro["iterations"]
+    assert np.array_equal(rg.history, ro["history"])
+    assert np.array_equal(rg.x.cpu().numpy(), ro["x"])
+    rg2 = gfn(Gm, dev(b), M=P, mode=mode, max_iter=500)
+    assert np.array_equal(rg2.x.cpu().numpy(), ro["x"])
+
+
 STICKY_CASES = [
     # name, matrix, solver, G, B   (tile-synchronous layout; the sticky state lives per slice column)
     ("C1-sticky", lambda: W.make("C1"), "cg", 4, 256),

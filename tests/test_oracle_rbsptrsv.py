@@ -51,13 +51,13 @@ def _exact_solve(n, rp, ci, lu, diag, r):
     return y, z
 
 
-@pytest.mark.parametrize("n,seed,depth", [(37, 1, 1), (37, 1, 3), (64, 2, 2), (64, 2, 6), (101, 3, 4), (101, 3, 30)])
+@pytest.mark.parametrize("n,seed,depth", [(77, 1, 1), (77, 1, 3), (160, 2, 2), (160, 2, 6), (301, 3, 4), (301, 3, 30)])
 def test_rb_integer_exact(orc, n, seed, depth):
     rp, ci, vals, rng = _int_factors(n, seed)
     M = orc.ILU0(rp, ci, vals, rb_depth=depth)
     diag = M.diag
     for attempt in range(50):
-        lu = rng.choice(np.array([-1.0, 1.0, 2.0, -2.0, 0.0]), size=len(ci))
+        lu = rng.choice(np.array([-1.0, 1.0, 2.0, -2.0, 0.0]), p=[0.15, 0.15, 0.05, 0.05, 0.6], size=len(ci))
         lu[diag] = rng.choice(np.array([1.0, -1.0]), size=n)
         r = rng.integers(-3, 4, size=n).astype(np.float64)
         y, z = _exact_solve(n, rp, ci, lu, diag, r)
