@@ -202,8 +202,21 @@ typedef struct {
 } mf_precond_opts;
 mf_status mf_precond_create(const mf_tile_matrix* A, mf_precond_kind kind, mf_stream stream, mf_precond** out);
 mf_status mf_precond_create_ex(const mf_tile_matrix* A, const mf_precond_opts* opts, mf_stream stream, mf_precond** out);
-/* host: recursive block depth (0 = sync-free), nodes of the L and U trees */
-mf_status mf_precond_info(const mf_precond* M, int32_t* rb_depth, int32_t* nodes_l, int32_t* nodes_u);
+/* Scheduling of the triangular solves (either algorithm above): the library measures the depth of
+ * the L and U dependency DAGs at creation; with fewer than 64 rows per level on average (e.g. C4:
+ * 2^20 rows, 2.8e5 levels) the triangles -- or the recursive-block leaves -- are solved by ONE CTA
+ * sweeping 32-row windows (warp shuffles inside a window, shared-memory ready counters between
+ * windows) instead of grid-wide chunks with global ready flags; the arithmetic is identical.
+ * Every fma chain runs in the order the substitution produces the unknowns: forward ascending
+ * column, backward descending column (reading R20). */
+typedef struct {
+    int32_t rb_depth;           /* 0: substitution over the whole factor */
+    int32_t nodes_l, nodes_u;   /* recursive block nodes (0 without) */
+    int32_t sweep;              /* 1: one-CTA sweep schedule */
+    int64_t depth_l, depth_u;   /* levels of the L / U dependency DAGs */
+    int64_t nnz_l, nnz_u;       /* strict-triangle entries of the factors */
+} mf_precond_stats;
+mf_status mf_precond_info(const mf_precond* M, mf_precond_stats* out /* host */);
 mf_status mf_precond_destroy(mf_precond* M);
 mf_status mf_precond_apply(const mf_precond* M, const double* r, double* z, mf_stream stream);
 

@@ -810,7 +810,10 @@ double orc_true_relres(int64_t n, const int64_t* rowptr, const int32_t* colidx, 
  *    ILU(0), FP64 factors).  IKJ variant on A's pattern (Saad, Alg. 10.4).
  *    L unit lower (strict lower part of lu), U upper including the diagonal.
  *    Forward  y_i = r_i - sum_{k<i} l_ik y_k      (fma chain, ascending k)
- *    Backward z_i = (y_i - sum_{k>i} u_ik z_k) / u_ii  (fma chain, ascending k)
+ *    Backward z_i = (y_i - sum_{k>i} u_ik z_k) / u_ii  (fma chain, descending k)
+ *    Each chain runs in the order the substitution produces its unknowns (ascending for the
+ *    forward solve, descending for the backward solve: the most recent unknown enters last);
+ *    the paper fixes no order (reading R20).
  * ---------------------------------------------------------------------------------- */
 int orc_ilu0(int64_t n, const int64_t* rowptr, const int32_t* colidx, const double* vals,
              double* lu, int64_t* diag) {
@@ -844,13 +847,15 @@ int orc_ilu0(int64_t n, const int64_t* rowptr, const int32_t* colidx, const doub
  * R27): a block of rows [lo, hi) with hi - lo >= 2 and depth > 0 splits at mid = lo + (hi - lo) / 2;
  * the square block's SpMV forms s_i = sum_k t_ik v_k over its columns (one fma chain from +0,
  * ascending k) and the right-hand side is then updated once, rhs_i = rhs_i - s_i; a leaf (depth 0
- * or one row) is the row-by-row substitution restricted to the columns inside the leaf.
+ * or fewer than 32 rows) is the row-by-row substitution restricted to the columns inside the leaf.
+ * Split points are multiples of 16 (one tile row): mid = lo + 16 * floor((hi - lo) / 32).
  *
  * Lower (unit diagonal, the strict lower part of lu): rows [lo, hi), the contributions of the
  * columns < lo already subtracted from y[lo..hi) (y holds the right-hand side on entry).
  * Order: solve(lo, mid); square rows [mid, hi) x columns [lo, mid); solve(mid, hi). */
+static int64_t rb_mid(int64_t lo, int64_t hi) { return lo + 16 * ((hi - lo) / 32); }
 static void rb_lower(const orc_ilu* M, double* y, int64_t lo, int64_t hi, int depth) {
-    if (depth == 0 || hi - lo < 2) {
+    if (depth == 0 || hi - lo < 32) {
         for (int64_t i = lo; i < hi; ++i) {
             double acc = y[i];
             for (int64_t k = M->rowptr[i]; k < M->diag[i]; ++k)
@@ -859,7 +864,7 @@ static void rb_lower(const orc_ilu* M, double* y, int64_t lo, int64_t hi, int de
         }
         return;
     }
-    int64_t mid = lo + (hi - lo) / 2;
+    int64_t mid = rb_mid(lo, hi);
     rb_lower(M, y, lo, mid, depth - 1);
     for (int64_t i = mid; i < hi; ++i) {                 /* square block: SpMV, then the update */
         double s = 0.0;
@@ -875,16 +880,16 @@ static void rb_lower(const orc_ilu* M, double* y, int64_t lo, int64_t hi, int de
  * subtracted from z[lo..hi) (z holds the right-hand side on entry).  Order: solve(mid, hi);
  * square rows [lo, mid) x columns [mid, hi); solve(lo, mid).  Leaf rows descending. */
 static void rb_upper(const orc_ilu* M, double* z, int64_t lo, int64_t hi, int depth) {
-    if (depth == 0 || hi - lo < 2) {
+    if (depth == 0 || hi - lo < 32) {
         for (int64_t i = hi - 1; i >= lo; --i) {
             double acc = z[i];
-            for (int64_t k = M->diag[i] + 1; k < M->rowptr[i + 1]; ++k)
+            for (int64_t k = M->rowptr[i + 1] - 1; k > M->diag[i]; --k)
                 if (M->colidx[k] < hi) acc = fma(-M->lu[k], z[M->colidx[k]], acc);
             z[i] = acc / M->lu[M->diag[i]];
         }
         return;
     }
-    int64_t mid = lo + (hi - lo) / 2;
+    int64_t mid = rb_mid(lo, hi);
     rb_upper(M, z, mid, hi, depth - 1);
     for (int64_t i = lo; i < mid; ++i) {
         double s = 0.0;
@@ -913,7 +918,7 @@ static void ilu_apply(const orc_ilu* M, const double* r, double* z) {
     }
     for (int64_t i = n - 1; i >= 0; --i) {
         double acc = y[i];
-        for (int64_t k = M->diag[i] + 1; k < M->rowptr[i + 1]; ++k) acc = fma(-M->lu[k], z[M->colidx[k]], acc);
+        for (int64_t k = M->rowptr[i + 1] - 1; k > M->diag[i]; --k) acc = fma(-M->lu[k], z[M->colidx[k]], acc);
         z[i] = acc / M->lu[M->diag[i]];
     }
     free(y);

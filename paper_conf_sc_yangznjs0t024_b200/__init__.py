@@ -153,7 +153,7 @@ def lib():
         L.mf_dot.argtypes = [vp, vp, vp, C.POINTER(d), vp]
         L.mf_precond_create.argtypes = [vp, C.c_int, vp, C.POINTER(vp)]
         L.mf_precond_create_ex.argtypes = [vp, C.POINTER(PrecondOpts), vp, C.POINTER(vp)]
-        L.mf_precond_info.argtypes = [vp, C.POINTER(i32), C.POINTER(i32), C.POINTER(i32)]
+        L.mf_precond_info.argtypes = [vp, C.POINTER(PrecondStats)]
         L.mf_precond_destroy.argtypes = [vp]
         L.mf_precond_apply.argtypes = [vp, vp, vp, vp]
         L.mf_cg_solve.argtypes = [vp, vp, vp, C.POINTER(SolveOpts), C.POINTER(SolveInfo), vp]
@@ -401,6 +401,11 @@ class PrecondOpts(C.Structure):
     _fields_ = [("kind", C.c_int), ("sptrsv", C.c_int32), ("rb_depth", C.c_int32)]
 
 
+class PrecondStats(C.Structure):
+    _fields_ = [("rb_depth", C.c_int32), ("nodes_l", C.c_int32), ("nodes_u", C.c_int32), ("sweep", C.c_int32),
+                ("depth_l", C.c_int64), ("depth_u", C.c_int64), ("nnz_l", C.c_int64), ("nnz_u", C.c_int64)]
+
+
 class Precond:
     """ILU(0) of the stored matrix; z = M^-1 r by SpTRSV kernels.  sptrsv =
     SPTRSV_RECURSIVE_BLOCK selects the recursive block SpTRSV of P:166 (rb_depth levels, 0 = auto)."""
@@ -414,9 +419,9 @@ class Precond:
         self.n = A.n_rows
 
     def info(self) -> dict:
-        d, nl, nu = C.c_int32(), C.c_int32(), C.c_int32()
-        _check(lib().mf_precond_info(self._h, C.byref(d), C.byref(nl), C.byref(nu)))
-        return {"rb_depth": d.value, "nodes_l": nl.value, "nodes_u": nu.value}
+        st = PrecondStats()
+        _check(lib().mf_precond_info(self._h, C.byref(st)))
+        return {f: getattr(st, f) for f, _ in PrecondStats._fields_}
 
     def apply(self, r, out=None, stream=None):
         import torch

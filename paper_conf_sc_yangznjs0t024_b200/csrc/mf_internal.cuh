@@ -142,6 +142,10 @@ struct MgLaunch {
     double* pv_own;                                      // own part of the window's extended PV vector
     mf_status (*prelaunch)(void* ctx, cudaStream_t s);   // clear the window, cross-rank barrier
     void* ctx;
+    // in-process rank group (all ranks on one device): a plain launch, because concurrent
+    // cooperative launches of the ranks' kernels are refused / serialised by the driver, and the
+    // ranks' grids must run side by side (co-residency is the caller's plan: G * nranks <= SMs)
+    bool plain_launch = false;
 };
 
 mf_status convert_csr(int64_t n_rows, int64_t n_cols, int64_t nnz, const int64_t* rowptr, const int32_t* colidx,

@@ -151,6 +151,30 @@ __global__ void __launch_bounds__(256) sptrsv_kernel(TriCSR T, const double* __r
                                     abort_flag, 20ull * 1000000000ull);
 }
 
+// one-CTA sweep triangular solve (precond.cuh sweep_solve): deep dependency DAGs
+template <bool FWD>
+__global__ void __launch_bounds__(128) sweep_kernel(TriCSR T, const double* __restrict__ diag, int64_t n, const double* in,
+                                                   double* out, int* abort_flag) {
+    extern __shared__ __align__(16) unsigned char sw_smem[];
+    if (!mfk::sweep_solve<FWD, false>(T.rp, T.ci, T.v, diag, n, in, out, sw_smem, abort_flag, 20ull * 1000000000ull) &&
+        threadIdx.x == 0)
+        atomicExch(abort_flag, 1);
+}
+
+// levels of the dependency DAG of a triangular factor (host): longest path, in solve order
+int64_t dag_depth(int64_t n, const std::vector<int64_t>& rp, const std::vector<int32_t>& ci, bool fwd) {
+    std::vector<int32_t> lev(n, 0);
+    int64_t mx = n > 0 ? 1 : 0;
+    for (int64_t p = 0; p < n; ++p) {
+        const int64_t i = fwd ? p : n - 1 - p;
+        int32_t l = 0;
+        for (int64_t q = rp[i]; q < rp[i + 1]; ++q) l = std::max(l, lev[ci[q]] + 1);
+        lev[i] = l;
+        mx = std::max<int64_t>(mx, l + 1);
+    }
+    return mx;
+}
+
 __global__ void __launch_bounds__(256) rb_square_kernel(const int64_t* __restrict__ rp, const int32_t* __restrict__ ci,
                                                         const double* __restrict__ val, int64_t r0, int64_t r1, double* v) {
     mfk::rb_square_rows(rp, ci, val, r0, r1, v, (int64_t)blockIdx.x * blockDim.x + threadIdx.x, (int64_t)gridDim.x * blockDim.x);
@@ -228,7 +252,15 @@ mf_status run_precond_apply(Precond& P, const double* r, double* z, cudaStream_t
             for (const RbNode& nd : T.h) {
                 const int64_t m = nd.r1 - nd.r0;
                 const int nb = (int)std::max<int64_t>(1, std::min<int64_t>((m + 255) / 256, (int64_t)sms * 8));
-                if (nd.leaf) {
+                if (nd.leaf && P.sweep) {
+                    const size_t sb = mfk::sweep_smem_bytes();
+                    if (pass == 0)
+                        sweep_kernel<true><<<1, 128, sb, s>>>(TriCSR{T.rp + nd.rp_off, T.ci, T.v}, nullptr, m, P.y + nd.r0,
+                                                              P.y + nd.r0, abort_flag);
+                    else
+                        sweep_kernel<false><<<1, 128, sb, s>>>(TriCSR{T.rp + nd.rp_off, T.ci, T.v}, P.udiag + nd.r0, m,
+                                                               P.y + nd.r0, P.y + nd.r0, abort_flag);
+                } else if (nd.leaf) {
                     unsigned long long* c = P.ctr + (pass == 0 ? 0 : P.Lrb.nleaves) + nd.leaf_idx;
                     if (pass == 0)
                         sptrsv_kernel<true><<<nb, 256, 0, s>>>(TriCSR{T.rp + nd.rp_off, T.ci, T.v}, nullptr, m, P.y + nd.r0,
@@ -252,6 +284,17 @@ mf_status run_precond_apply(Precond& P, const double* r, double* z, cudaStream_t
     }
     MF_CUDA(cudaMemsetAsync(P.ctr, 0, 3 * sizeof(unsigned long long), s));
     int* abort_flag = reinterpret_cast<int*>(P.ctr + 2);
+    if (P.sweep) {
+        const size_t sb = mfk::sweep_smem_bytes();
+        sweep_kernel<true><<<1, 128, sb, s>>>(P.L, nullptr, P.n, r, P.y, abort_flag);
+        sweep_kernel<false><<<1, 128, sb, s>>>(P.U, P.udiag, P.n, P.y, z, abort_flag);
+        MF_CUDA(cudaGetLastError());
+        int ab = 0;
+        MF_CUDA(cudaMemcpyAsync(&ab, abort_flag, sizeof(int), cudaMemcpyDeviceToHost, s));
+        MF_CUDA(cudaStreamSynchronize(s));
+        if (ab) return fail(MF_ERR_DEADLOCK, "triangular-solve watchdog expired");
+        return MF_OK;
+    }
     sptrsv_kernel<true><<<blocks, 256, 0, s>>>(P.L, nullptr, P.n, r, P.y, P.flags, 2 * e + 1, 0u, P.ctr, abort_flag);
     sptrsv_kernel<false><<<blocks, 256, 0, s>>>(P.U, P.udiag, P.n, P.y, z, P.flags, 2 * e + 2, 2 * e + 1, P.ctr + 1, abort_flag);
     MF_CUDA(cudaGetLastError());
@@ -295,6 +338,16 @@ mf_status build_precond(const TileMatrix& A, int rb_depth, cudaStream_t s, Preco
     MF_TRY(upload(&P->udiag, ud, s));
     int nctr = 4;
     P->rb_depth = rb_depth;
+    // one-CTA sweep when the DAG is too deep for grid-wide parallelism (< 64 rows per level)
+    P->depth_l = dag_depth(n, lrp, lci, true);
+    P->depth_u = dag_depth(n, urp, uci, false);
+    P->sweep = n > 0 && (double)n / (double)std::max(P->depth_l, P->depth_u) < 64.0 ? 1 : 0;
+    if (const char* ev = getenv("MF_SPTRSV_SWEEP")) P->sweep = atoi(ev) != 0;   // experiments / tests
+    if (P->sweep) {
+        const int sb = (int)mfk::sweep_smem_bytes();
+        MF_CUDA(cudaFuncSetAttribute((const void*)sweep_kernel<true>, cudaFuncAttributeMaxDynamicSharedMemorySize, sb));
+        MF_CUDA(cudaFuncSetAttribute((const void*)sweep_kernel<false>, cudaFuncAttributeMaxDynamicSharedMemorySize, sb));
+    }
     if (rb_depth > 0) {
         RbHost HL, HU;
         rb_lower(HL, M, diag, 0, n, rb_depth);
@@ -365,11 +418,16 @@ mf_status mf_precond_create_ex(const mf_tile_matrix* A, const mf_precond_opts* o
     return MF_OK;
 }
 
-mf_status mf_precond_info(const mf_precond* M, int32_t* rb_depth, int32_t* nodes_l, int32_t* nodes_u) {
-    if (!M) return fail(MF_ERR_INVALID_ARG, "NULL argument");
-    if (rb_depth) *rb_depth = M->p.rb_depth;
-    if (nodes_l) *nodes_l = (int32_t)M->p.Lrb.h.size();
-    if (nodes_u) *nodes_u = (int32_t)M->p.Urb.h.size();
+mf_status mf_precond_info(const mf_precond* M, mf_precond_stats* out) {
+    if (!M || !out) return fail(MF_ERR_INVALID_ARG, "NULL argument");
+    out->rb_depth = M->p.rb_depth;
+    out->nodes_l = (int32_t)M->p.Lrb.h.size();
+    out->nodes_u = (int32_t)M->p.Urb.h.size();
+    out->sweep = M->p.sweep;
+    out->depth_l = M->p.depth_l;
+    out->depth_u = M->p.depth_u;
+    out->nnz_l = M->p.nnz_l;
+    out->nnz_u = M->p.nnz_u;
     return MF_OK;
 }
 

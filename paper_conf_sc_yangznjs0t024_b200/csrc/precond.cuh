@@ -39,6 +39,8 @@ struct RbTree {
 struct Precond {
     int64_t n = 0;
     int rb_depth = 0;             // 0: sync-free substitution; > 0: recursive block SpTRSV
+    int sweep = 0;                // 1: triangular solves (or rb leaves) by the one-CTA sweep (deep DAGs)
+    int64_t depth_l = 0, depth_u = 0;   // levels of the L / U dependency DAGs
     RbTree Lrb, Urb;
     TriCSR L, U;                  // L: strict lower part (unit diagonal implied); U: strict upper part
     double* udiag = nullptr;      // u_ii
@@ -73,8 +75,9 @@ __device__ __forceinline__ void st_release_u32(unsigned* p, unsigned v) {
 }
 
 // Sync-free chunked triangular solve, called by all threads of a CTA (any number of CTAs).
-//   FWD:  out_i = in_i - sum_{k<i} T_ik out_k                 rows ascending
-//   !FWD: out_i = (in_i - sum_{k>i} T_ik out_k) / diag_i       rows descending
+//   FWD:  out_i = in_i - sum_{k<i} T_ik out_k                 rows ascending, k ascending
+//   !FWD: out_i = (in_i - sum_{k>i} T_ik out_k) / diag_i       rows descending, k descending
+// (each fma chain in the order the substitution produces the unknowns, reading R20)
 // Chunks of blockDim.x consecutive rows (in solve order) are grabbed with one atomicAdd on
 // *ctr (values base, base+1, ...), so a chunk only waits on chunks grabbed earlier or on
 // earlier rows of its own chunk: deadlock-free without co-residency.  Inside a chunk a row
@@ -129,7 +132,9 @@ __device__ void sptrsv_chunked(const int64_t* __restrict__ rp, const int32_t* __
             if (wait_val) sp_wait_flag(&flags[i], wait_val, abort_flag, t0, timeout_ns);
             double acc = __ldcg(in + i);
             const int64_t lo = rp[i], hi = rp[i + 1];
-            for (int64_t q = lo; q < hi; ++q) {
+            // chain in solve order of the columns: forward ascending, backward descending (R20)
+            for (int64_t qq = lo; qq < hi; ++qq) {
+                const int64_t q = FWD ? qq : lo + hi - 1 - qq;
                 const int64_t k = ci[q];
                 const int64_t pk = FWD ? k : n - 1 - k;     // position of k in solve order (< pos)
                 double xk;
@@ -170,6 +175,137 @@ __device__ __forceinline__ void rb_square_rows(const int64_t* __restrict__ rp, c
         for (int64_t q = lo; q < hi; ++q) sacc = __fma_rn(val[q], __ldcg(v + ci[q]), sacc);
         v[i] = __dsub_rn(__ldcg(v + i), sacc);
     }
+}
+
+// ------------------------------------------------------------------------------------------
+// Sweep triangular solve: ONE CTA (its first SW_WARPS warps), for factors whose dependency DAG is
+// too deep for grid-wide parallelism (C4: 2^20 rows, 2.8e5 levels, ~4 rows per level -- a grid
+// barrier or a cross-SM flag per level would cost microseconds per level).  Same arithmetic as
+// sptrsv_chunked (and the oracle): position p in solve order is row i = FWD ? p : n-1-p; row i's
+// chain runs over its entries in solve order of their columns; !FWD divides by diag_i last.
+//
+// Windows of 32 consecutive positions; warp w takes windows w, w + SW_WARPS, ...; lane l owns
+// position 32*win + l.  Per window: (1) the warp stages the window's CSR range (contiguous: the
+// rows of a window are consecutive) in its shared-memory buffer with coalesced loads; (2) entries
+// whose column lies in an earlier window are consumed in chain order, the warp waiting (warp-
+// uniform) until the window holding the column is complete -- most of this overlaps the previous
+// window's sweep; (3) the in-window sweep: step s finalises lane s (all its remaining entries have
+// earlier in-window positions, consumed at earlier steps) and broadcasts the value by shuffle to the
+// lanes whose next entry is position 32*win + s.  Values of recent windows are kept in a shared
+// ring; older ones are read back from `out`.  `done` counts completed windows (in order).
+constexpr int SW_WARPS = 4;
+constexpr int SW_CAP = 1024;       // staged entries per warp and window (larger windows read global)
+constexpr int SW_RING = 2048;      // recent solution values kept in shared memory (positions)
+__host__ __device__ constexpr size_t sweep_smem_bytes() {
+    return (size_t)SW_WARPS * SW_CAP * (8 + 4) + (size_t)SW_RING * 8 + 64;
+}
+template <bool FWD, bool OUTPV>
+__device__ __noinline__ bool sweep_solve(const int64_t* __restrict__ rp, const int32_t* __restrict__ ci,
+                                         const double* __restrict__ val, const double* __restrict__ diag, int64_t n,
+                                         const double* in, double* out, unsigned char* smem, int* abort_flag,
+                                         unsigned long long timeout_ns) {
+    const int t = threadIdx.x, w = t >> 5, lane = t & 31;
+    double* ring = reinterpret_cast<double*>(smem);
+    double* sval = ring + SW_RING;
+    int32_t* sci = reinterpret_cast<int32_t*>(sval + (size_t)SW_WARPS * SW_CAP);
+    volatile int* done = reinterpret_cast<volatile int*>(sci + (size_t)SW_WARPS * SW_CAP);
+    auto oidx = [](int64_t i) -> int64_t { return OUTPV ? ((i >> 4) * 18 + (i & 15)) : i; };
+    if (t == 0) { done[0] = 0; done[1] = 0; }
+    __syncthreads();
+    if (w >= SW_WARPS) return true;
+    double* wv = sval + (size_t)w * SW_CAP;
+    int32_t* wc = sci + (size_t)w * SW_CAP;
+    const int64_t nwin = (n + 31) >> 5;
+    const unsigned long long t0 = sp_timer();
+    const unsigned FULL = 0xffffffffu;
+    bool ok = true;
+    // spin (warp-uniform) until at least `need` windows are complete
+    auto wait_done = [&](int64_t need) {
+        for (unsigned sp = 0; done[0] < need; ++sp)
+            if ((sp & 1023u) == 1023u && (*(volatile int*)abort_flag || sp_timer() - t0 > timeout_ns)) {
+                atomicExch(abort_flag, 1);
+                ok = false;
+                done[1] = 1;
+                break;
+            }
+        __syncwarp();
+    };
+    for (int64_t win = w; win < nwin && ok && !done[1]; win += SW_WARPS) {
+        const int64_t p0 = win << 5, p = p0 + lane;
+        const bool valid = p < n;
+        const int64_t i = FWD ? p : n - 1 - p;
+        const int64_t lo = valid ? rp[i] : 0, hi = valid ? rp[i + 1] : 0;
+        // the window's CSR range: rows p0 .. p0+31 in solve order are consecutive rows
+        const int64_t plast = min(p0 + 31, n - 1);
+        const int64_t e0 = FWD ? rp[p0] : rp[n - 1 - plast];
+        const int64_t e1 = FWD ? rp[plast + 1] : rp[n - p0];
+        const bool staged = e1 - e0 <= SW_CAP;
+        if (staged)
+            for (int64_t j = lane; j < e1 - e0; j += 32) { wc[j] = __ldg(ci + e0 + j); wv[j] = __ldg(val + e0 + j); }
+        __syncwarp();
+        const double dg = (!FWD && valid) ? diag[i] : 1.0;
+        double acc = valid ? __ldcg(in + i) : 0.0;
+        const int cnt = (int)(hi - lo);
+        int k = 0;
+        int64_t pc = INT64_MAX;      // position of the current entry's column
+        double v = 0.0;
+        int32_t col = 0;
+        auto load_entry = [&]() {
+            if (k < cnt) {
+                const int64_t q = FWD ? lo + k : hi - 1 - k;
+                col = staged ? wc[q - e0] : __ldg(ci + q);
+                v = staged ? wv[q - e0] : __ldg(val + q);
+                pc = FWD ? (int64_t)col : n - 1 - col;
+            } else {
+                pc = INT64_MAX;
+            }
+        };
+        load_entry();
+        // (2) entries in earlier windows, in chain order: a lane consumes its next entry as soon as
+        // the window holding the column is complete; the warp waits only when no lane can proceed
+        const int64_t ring_lo = p0 - SW_RING + (int64_t)SW_WARPS * 32;   // ring slots not yet reused
+        while (true) {
+            const int dn = done[0];
+            __threadfence_block();                 // acquire: values of the completed windows
+            const bool need = pc < p0;
+            const bool ready = need && (pc >> 5) < dn;
+            if (ready) {
+                const double yv = pc >= ring_lo ? ring[pc & (SW_RING - 1)] : __ldcg(out + oidx(col));
+                acc = __fma_rn(-v, yv, acc);
+                ++k;
+                load_entry();
+            }
+            if (!__any_sync(FULL, pc < p0)) break;
+            if (!__any_sync(FULL, ready)) {
+                wait_done(dn + 1);
+                if (!ok) break;
+            }
+        }
+        if (!ok) break;
+        // (3) in-window sweep
+        double fin = 0.0;
+#pragma unroll 4
+        for (int sstep = 0; sstep < 32; ++sstep) {
+            if (lane == sstep) fin = FWD ? acc : __ddiv_rn(acc, dg);
+            const double ys = __shfl_sync(FULL, fin, sstep);
+            if (pc == p0 + sstep) {
+                acc = __fma_rn(-v, ys, acc);
+                ++k;
+                load_entry();
+            }
+        }
+        if (valid) {
+            out[oidx(i)] = fin;
+            ring[p & (SW_RING - 1)] = fin;
+        }
+        __threadfence_block();
+        __syncwarp();
+        wait_done(win);            // windows complete in order
+        if (!ok) break;
+        if (lane == 0) done[0] = (int)(win + 1);
+        __syncwarp();
+    }
+    return ok;
 }
 
 }  // namespace mfk

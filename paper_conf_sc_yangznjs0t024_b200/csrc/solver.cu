@@ -209,7 +209,7 @@ mf_status run_spmv(const TileMatrix& A, const double* x, double* y, const uint8_
         if (level) fn = counts_host ? (void*)spmv_kernel<true, true, 512> : (void*)spmv_kernel<true, false, 512>;
         else fn = counts_host ? (void*)spmv_kernel<false, true, 512> : (void*)spmv_kernel<false, false, 512>;
     }
-    MF_CUDA(cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
+    MF_CUDA(cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, smem_optin));
     const int32_t* plan = A.plan_tr;
     int slot_bytes = A.slot_bytes, blob_cap = A.blob_cap, nst_a = nst, ecap = A.ecap;
     void* args[] = {&M, (void*)&plan, (void*)&pv, (void*)&y, &range_guard, &dcnt, &nst_a, &slot_bytes, &blob_cap, &ecap};
@@ -330,7 +330,7 @@ mf_status run_solve(const TileMatrix& A, bool bicg, const double* b, double* x, 
     for (int g = 0; g < G; ++g) max_rows = std::max(max_rows, A.plan_rows_host[g + 1] - A.plan_rows_host[g]);
     // shared memory: fixed + SpMV region (TMA ring or compact buffers) + mu (and theta) + SpTRSV
     const size_t fixed = fixed_smem_bytes();
-    const int64_t pre_smem = pre ? (int64_t)B * 12 + 32 : 0;
+    const int64_t pre_smem = pre ? (int64_t)B * 12 + 32 + (P->sweep ? (int64_t)mfk::sweep_smem_bytes() + 32 : 0) : 0;
     const int64_t ebytes = A.ts ? (int64_t)(B / 32) * A.ecap * 128 : 0;
     const int64_t avail = (int64_t)smem_optin - (int64_t)fixed - pre_smem - 128 - (int64_t)mfk::TS_CTRL_BYTES - ebytes;
     int64_t cap = 0;
@@ -354,7 +354,10 @@ mf_status run_solve(const TileMatrix& A, bool bicg, const double* b, double* x, 
     if ((int64_t)smem > smem_optin) return fail(MF_ERR_UNSUPPORTED, "shared-memory plan exceeds the device limit");
 
     void* kfn = mgl ? pick_cgmg(B, dyn) : pick_kernel(B, bicg, dyn, count, sticky, pre, sr);
-    MF_CUDA(cudaFuncSetAttribute(kfn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
+    // the opt-in maximum, not this launch's size: concurrent solves (rank threads of a local group,
+    // other streams) share the function attribute, and a smaller value set by one would make
+    // another's larger launch invalid
+    MF_CUDA(cudaFuncSetAttribute(kfn, cudaFuncAttributeMaxDynamicSharedMemorySize, smem_optin));
     int per_sm = 0;
     MF_CUDA(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, kfn, B, smem));
     if (per_sm * sms < G) return fail(MF_ERR_INVALID_ARG, "plan G exceeds co-resident CTAs for this launch");
@@ -440,6 +443,7 @@ mf_status run_solve(const TileMatrix& A, bool bicg, const double* b, double* x, 
         a.Lrp = P->L.rp; a.Lci = P->L.ci; a.Lv = P->L.v;
         a.Urp = P->U.rp; a.Uci = P->U.ci; a.Uv = P->U.v; a.Ud = P->udiag;
         a.pflags = P->flags; a.pctr = P->ctr; a.py = P->y; a.pz = pz; a.ps = psh;
+        a.psweep = P->sweep;
         if (P->rb_depth > 0) {
             a.rb = 1;
             a.Lnodes = P->Lrb.nodes; a.nLn = (int)P->Lrb.h.size(); a.Lbrp = P->Lrb.rp; a.Lbci = P->Lrb.ci; a.Lbv = P->Lrb.v;
@@ -458,7 +462,8 @@ mf_status run_solve(const TileMatrix& A, bool bicg, const double* b, double* x, 
     MF_CUDA(cudaEventCreate(&ev.e1));
     void* args[] = {&a};
     MF_CUDA(cudaEventRecord(ev.e0, s));
-    MF_CUDA(cudaLaunchCooperativeKernel(kfn, dim3(G), dim3(B), args, smem, s));
+    if (mgl && mgl->plain_launch) MF_CUDA(cudaLaunchKernel(kfn, dim3(G), dim3(B), args, smem, s));
+    else MF_CUDA(cudaLaunchCooperativeKernel(kfn, dim3(G), dim3(B), args, smem, s));
     MF_CUDA(cudaEventRecord(ev.e1, s));
     double hout[8];
     MF_CUDA(cudaMemcpyAsync(hout, out, sizeof(hout), cudaMemcpyDeviceToHost, s));

@@ -77,6 +77,7 @@ struct SolveArgs {
     unsigned pe0;                // epoch of the first apply of this solve
     // recursive block SpTRSV (rb == 0: sync-free substitution over the whole factor)
     int rb;
+    int psweep;                  // 1: triangular solves by the one-CTA sweep (deep dependency DAGs)
     const RbNode* Lnodes; int nLn; const int64_t* Lbrp; const int32_t* Lbci; const double* Lbv;
     const RbNode* Unodes; int nUn; const int64_t* Ubrp; const int32_t* Ubci; const double* Ubv;
     MgArgs mg;                   // multi-GPU single kernel (P == 0: off)
@@ -350,6 +351,7 @@ struct Smem {
     double* tys;     // [B] triangular-solve chunk values (preconditioned)
     int* tready;     // [B]
     long long* tchunk;
+    unsigned char* sweep;   // sweep triangular solve buffers (precond.cuh sweep_smem_bytes), CTA 0
     double* red;     // [4*32 + 8]
     int* ired;       // [16]
     unsigned long long* timer;   // [NPHASE + 1]
@@ -379,6 +381,7 @@ __device__ __forceinline__ Smem carve(const SolveArgs& a, int nvec) {
     s.tys = s.mu + (size_t)nvec * a.mu_cap;
     s.tready = reinterpret_cast<int*>(s.tys + blockDim.x);
     s.tchunk = reinterpret_cast<long long*>(s.tready + blockDim.x + 2);
+    s.sweep = smem_raw + mfk::ts_r16((int)(reinterpret_cast<unsigned char*>(s.tchunk + 2) - smem_raw));
     return s;
 }
 
@@ -959,7 +962,16 @@ __device__ __noinline__ bool precond_apply_rb(const SolveArgs& a, PcState& ps, c
         for (int k = 0; k < nn && ok; ++k) {
             const RbNode nd = nodes[k];
             const int64_t m = nd.r1 - nd.r0;
-            if (nd.leaf) {
+            if (nd.leaf && a.psweep) {
+                if (blockIdx.x == 0) {
+                    const bool sok = pass == 0
+                        ? mfk::sweep_solve<true, false>(brp + nd.rp_off, bci, bv, nullptr, m, a.py + nd.r0, a.py + nd.r0,
+                                                         sm.sweep, a.abort_flag, a.timeout_ns)
+                        : mfk::sweep_solve<false, false>(brp + nd.rp_off, bci, bv, a.Ud + nd.r0, m, a.py + nd.r0,
+                                                          a.py + nd.r0, sm.sweep, a.abort_flag, a.timeout_ns);
+                    if (!sok && threadIdx.x == 0) atomicExch(a.abort_flag, 1);
+                }
+            } else if (nd.leaf) {
                 const int64_t nch = (m + B - 1) / B;
                 if (pass == 0) {
                     mfk::sptrsv_chunked<true, false>(brp + nd.rp_off, bci, bv, nullptr, m, a.py + nd.r0, a.py + nd.r0,
@@ -989,6 +1001,21 @@ template <bool OUTPV>
 __device__ __forceinline__ bool precond_apply(const SolveArgs& a, PcState& ps, const Smem& sm, Ctx& c, const double* in,
                                               double* out, int64_t R0, int64_t Rend) {
     if (a.rb) return precond_apply_rb<OUTPV>(a, ps, sm, c, in, out, R0, Rend);
+    if (a.psweep) {
+        // one CTA sweeps L then U (the other CTAs wait in the grid barrier)
+        ps.apply++;
+        if (blockIdx.x == 0) {
+            bool sok = mfk::sweep_solve<true, false>(a.Lrp, a.Lci, a.Lv, nullptr, a.n, in, a.py, sm.sweep, a.abort_flag,
+                                                     a.timeout_ns);
+            __syncthreads();
+            if (sok)
+                sok = mfk::sweep_solve<false, OUTPV>(a.Urp, a.Uci, a.Uv, a.Ud, a.n, a.py, out, sm.sweep, a.abort_flag,
+                                                     a.timeout_ns);
+            if (!sok && threadIdx.x == 0) atomicExch(a.abort_flag, 1);
+        }
+        __threadfence();
+        return grid_barrier(a, c) && *(volatile int*)a.abort_flag == 0;
+    }
     const unsigned e = a.pe0 + ps.apply++;
     const unsigned vf = 2 * e + 1, vb = 2 * e + 2;
     const int64_t nch = (a.n + blockDim.x - 1) / blockDim.x;

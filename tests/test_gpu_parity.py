@@ -369,6 +369,40 @@ def test_rb_precond_apply_bit_exact(mf, orc, name, make, depths):
         P.close()
 
 
+SCHED_CASES = [("C4spd-14", lambda: W.make("C4spd", 1 << 14), "cg", 2),
+               ("C4ind-13", lambda: W.make("C4ind", 1 << 13), "bicgstab", 2),
+               ("C2-16", lambda: W.make("C2", 16), "cg", 2),
+               ("ragged-1000", lambda: W.suitesparse_like(1000, seed=8, spd=False), "bicgstab", 1)]
+
+
+@pytest.mark.parametrize("sweep", ["0", "1"])
+@pytest.mark.parametrize("rb", [0, 3])
+@pytest.mark.parametrize("name,make,solver,mode", SCHED_CASES, ids=[c[0] for c in SCHED_CASES])
+def test_sptrsv_schedules_bit_exact(mf, orc, monkeypatch, name, make, solver, mode, rb, sweep):
+    """Both schedules of the triangular solves (grid-wide sync-free chunks / one-CTA sweep), with
+    and without the recursive blocks: apply and preconditioned solve bit-identical to the oracle."""
+    monkeypatch.setenv("MF_SPTRSV_SWEEP", sweep)
+    A = make()
+    T = oracle_tiles(orc, A)
+    rp, ci, sv = T.stored_csr()
+    G = mf.TileMatrix.from_host_csr(A, grid_ctas=6, block_threads=256)
+    kw = dict(sptrsv=mf.SPTRSV_RECURSIVE_BLOCK, rb_depth=rb) if rb else {}
+    P = mf.Precond(G, **kw)
+    assert P.info()["sweep"] == int(sweep)
+    M = orc.ILU0(rp, ci, sv, rb_depth=rb)
+    r = np.random.default_rng(3).standard_normal(A.n_rows)
+    assert np.array_equal(P.apply(dev(r)).cpu().numpy(), M.apply(r))
+    g, bb, R = G.plan()
+    b = W.rhs_ones(A)
+    ofn = orc.cg if solver == "cg" else orc.bicgstab
+    gfn = mf.cg_solve if solver == "cg" else mf.bicgstab_solve
+    ro = ofn(T, b, M=M, mode=mode, plan=orc.Plan(g, bb, R), max_iter=300)
+    rg = gfn(G, dev(b), M=P, mode=mode, max_iter=300)
+    assert rg.iterations == ro["iterations"] and rg.converged == bool(ro["converged"])
+    assert np.array_equal(rg.history, ro["history"])
+    assert np.array_equal(rg.x.cpu().numpy(), ro["x"])
+
+
 RB_SOLVE_CASES = [
     ("C4spd-13-dyn-rb3", lambda: W.make("C4spd", 1 << 13), "cg", 2, 3, 6, 256),
     ("C4spd-14-static-rb2", lambda: W.make("C4spd", 1 << 14), "cg", 1, 2, 0, 0),
