@@ -907,7 +907,7 @@ mf_status dist_solve(const TileMatrix& A, const DistInfo& D, bool bicg, const do
     void* f_init = spmv_fn<false, 0>(B);
     void* f_mu = dyn ? (bicg ? spmv_fn<true, 2>(B) : spmv_fn<true, 1>(B)) : (bicg ? spmv_fn<false, 2>(B) : spmv_fn<false, 1>(B));
     void* f_th = dyn ? spmv_fn<true, 3>(B) : spmv_fn<false, 3>(B);
-    for (void* f : {f_init, f_mu, f_th}) MF_CUDA(cudaFuncSetAttribute(f, cudaFuncAttributeMaxDynamicSharedMemorySize, smem_optin));
+    for (void* f : {f_init, f_mu, f_th}) MF_TRY(set_max_dyn_smem(f, smem_optin));
     cudaStream_t q = s;   // the stream the iteration is enqueued on (a private one while capturing)
     auto launch_spmv = [&](void* f, const double* in) -> mf_status {
         void* args[] = {&a, (void*)&in};

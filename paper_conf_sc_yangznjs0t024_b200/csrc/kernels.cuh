@@ -181,7 +181,7 @@ struct TsSmem {
     double* ebuf;                   // per-warp decode buffers: ecap columns x 16 doubles per warp
     int nst, slot_bytes, blob_cap, ecap;
     unsigned long long* full;       // [TS_NSTMAX]
-    unsigned long long* empty;      // [TS_NSTMAX]
+    unsigned long long* empty;      // [TS_NSTMAX] release counters: warps done with the slot's stage
     unsigned long long* ctr;        // [0] stages issued so far (ring position); [1] resident SpMVs done
     __device__ __forceinline__ unsigned char* slot(int s) const { return base + (size_t)s * slot_bytes; }
 };
@@ -214,8 +214,10 @@ static __device__ __noinline__ void mbar_wait_slow(unsigned long long* b, unsign
     unsigned long long t0;
     asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t0));
     for (unsigned k = 1;; ++k) {
-        if (mbar_try_suspend(b, parity)) return;   // the warp sleeps (<= 2 us) until the phase completes
-        if ((k & 63u) == 0) {
+        // try_wait suspends the warp in hardware until the phase completes or a time limit passes:
+        // the loop issues a few instructions per wake-up, the timer is read rarely
+        if (mbar_try(b, parity)) return;
+        if ((k & 1023u) == 0) {
             unsigned long long t1;
             asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t1));
             if (t1 - t0 > 20ull * 1000000000ull) __trap();
@@ -249,7 +251,7 @@ __device__ __forceinline__ void ts_init(const TsSmem& sm) {
     if (threadIdx.x == 0) {
         for (int s = 0; s < TS_NSTMAX; ++s) {
             mbar_init(sm.full + s, 1);
-            mbar_init(sm.empty + s, blockDim.x >> 5);
+            sm.empty[s] = 0ull;       // release counter of the slot (warps done with it)
         }
         sm.ctr[0] = 0ull;
         sm.ctr[1] = 0ull;
@@ -573,34 +575,46 @@ __device__ __forceinline__ void spmv_ts(const Mat& A, int64_t tr0c, const double
         if (t == 0) sm.ctr[1] = rc + 1;
         return;
     }
-    // streaming: ring position u0 (slot = u mod NST, phase = (u / NST) & 1), 32-bit counters
+    // streaming: ring position u0 (slot = u mod NST, phase = (u / NST) & 1), 32-bit counters.
+    // Warp 0 fills the ring; afterwards the LAST warp to release a slot (a shared-memory counter per
+    // slot) refills it with stage k + NST, so no warp ever waits for the others to drain a slot.
+    // Every warp reads the record of stage k + NST while it waits for stage k (one word per lane).
     const unsigned u0 = (unsigned)sm.ctr[0];
+    const unsigned NW = blockDim.x >> 5;
     int sl = (int)(u0 % (unsigned)NST);
     unsigned ph = (u0 / (unsigned)NST) & 1u;
-    uint32_t pre[TS_PF];                      // warp 0: records of stages k + NST .. k + NST + TS_PF - 1
     if (w == 0) {
         int isl = sl;
-        unsigned iph = ph;
         for (int k = 0; k < min(ns, NST); ++k) {
-            // the slot's previous use (previous SpMV) finished before the caller's barrier; its
-            // "empty" phase completed: wait on it to keep the parity in step
-            if (u0 + k >= (unsigned)NST) mbar_wait(sm.empty + isl, iph ^ 1u);
             ts_issue(A.blob, recs[k * 32 + lane], sm.slot(isl), sm.blob_cap, sm.full + isl, xb, true, pol);
-            if (++isl == NST) { isl = 0; iph ^= 1u; }
+            if (++isl == NST) isl = 0;
         }
-#pragma unroll
-        for (int j = 0; j < TS_PF; ++j) pre[j] = NST + j < ns ? recs[(NST + j) * 32 + lane] : 0u;
     }
     for (int k = 0; k < ns; ++k) {
+        const bool refill = k + NST < ns;
+        const uint32_t rnext = refill ? __ldg(recs + (size_t)(k + NST) * 32 + lane) : 0u;
         mbar_wait(sm.full + sl, ph);
         ts_consume<DYN, STK>(ts_view(sm.slot(sl), sm.blob_cap), pv, range_guard, own_mode, ownv, A.n_rows, A.stk, E, emit);
-        if (lane == 0) mbar_arrive(sm.empty + sl);
-        if (w == 0 && k + NST < ns) {
-            mbar_wait(sm.empty + sl, ph);         // every warp is done with the slot
-            ts_issue(A.blob, pre[0], sm.slot(sl), sm.blob_cap, sm.full + sl, xb, true, pol);
-#pragma unroll
-            for (int j = 0; j + 1 < TS_PF; ++j) pre[j] = pre[j + 1];
-            pre[TS_PF - 1] = k + NST + TS_PF < ns ? recs[(k + NST + TS_PF) * 32 + lane] : 0u;
+        unsigned old = 0;
+        if (lane == 0) {
+            __threadfence_block();                                   // release: this warp's reads of the slot
+            old = atomicAdd(reinterpret_cast<unsigned*>(sm.empty + sl), 1u);
+        }
+        old = __shfl_sync(0xffffffffu, old, 0);
+        if (old == NW - 1) {                                         // every warp is done with the slot
+            if (lane == 0) {
+                *reinterpret_cast<volatile unsigned*>(sm.empty + sl) = 0u;
+                __threadfence_block();                               // acquire: the other warps' reads
+                asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
+            }
+            __syncwarp();
+            if (refill) {
+                if (pol == 0) {
+                    pol = policy_evict_first();
+                    asm volatile("fence.proxy.async.global;" ::: "memory");
+                }
+                ts_issue(A.blob, rnext, sm.slot(sl), sm.blob_cap, sm.full + sl, xb, true, pol);
+            }
         }
         if (++sl == NST) { sl = 0; ph ^= 1u; }
     }

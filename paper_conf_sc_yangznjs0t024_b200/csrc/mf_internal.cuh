@@ -148,6 +148,15 @@ struct MgLaunch {
     bool plain_launch = false;
 };
 
+// Dynamic shared memory limit of a kernel = the opt-in maximum minus its static shared memory.
+// Set to the maximum (not to one launch's size): concurrent solves share the function attribute.
+inline mf_status set_max_dyn_smem(const void* fn, int smem_optin) {
+    cudaFuncAttributes fa;
+    MF_CUDA(cudaFuncGetAttributes(&fa, fn));
+    MF_CUDA(cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, smem_optin - (int)fa.sharedSizeBytes));
+    return MF_OK;
+}
+
 mf_status convert_csr(int64_t n_rows, int64_t n_cols, int64_t nnz, const int64_t* rowptr, const int32_t* colidx,
                       const double* vals, const mf_convert_opts& o, cudaStream_t s, TileMatrix* A);
 void destroy_tiles(TileMatrix* A);

@@ -209,7 +209,7 @@ mf_status run_spmv(const TileMatrix& A, const double* x, double* y, const uint8_
         if (level) fn = counts_host ? (void*)spmv_kernel<true, true, 512> : (void*)spmv_kernel<true, false, 512>;
         else fn = counts_host ? (void*)spmv_kernel<false, true, 512> : (void*)spmv_kernel<false, false, 512>;
     }
-    MF_CUDA(cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, smem_optin));
+    MF_TRY(set_max_dyn_smem(fn, smem_optin));
     const int32_t* plan = A.plan_tr;
     int slot_bytes = A.slot_bytes, blob_cap = A.blob_cap, nst_a = nst, ecap = A.ecap;
     void* args[] = {&M, (void*)&plan, (void*)&pv, (void*)&y, &range_guard, &dcnt, &nst_a, &slot_bytes, &blob_cap, &ecap};
@@ -357,7 +357,7 @@ mf_status run_solve(const TileMatrix& A, bool bicg, const double* b, double* x, 
     // the opt-in maximum, not this launch's size: concurrent solves (rank threads of a local group,
     // other streams) share the function attribute, and a smaller value set by one would make
     // another's larger launch invalid
-    MF_CUDA(cudaFuncSetAttribute(kfn, cudaFuncAttributeMaxDynamicSharedMemorySize, smem_optin));
+    MF_TRY(set_max_dyn_smem(kfn, smem_optin));
     int per_sm = 0;
     MF_CUDA(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, kfn, B, smem));
     if (per_sm * sms < G) return fail(MF_ERR_INVALID_ARG, "plan G exceeds co-resident CTAs for this launch");
