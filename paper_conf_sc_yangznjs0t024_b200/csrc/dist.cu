@@ -836,6 +836,13 @@ mf_status mg_prelaunch(void* ctx, cudaStream_t s) {
     MF_NCCL(ncclAllReduce(D.bar_scratch, D.bar_scratch, 1, ncclInt32, ncclSum, c->nccl, s));   // stream-ordered barrier
     return MF_OK;
 }
+// local group: every rank thread has enqueued its kernel (see MgLaunch::postlaunch)
+mf_status mg_postlaunch(void* ctx) {
+    DistInfo& D = *static_cast<MgCtx*>(ctx)->D;
+    Comm* c = D.comm;
+    if (c->local && c->nranks > 1 && !c->local->barrier()) return fail(MF_ERR_DEADLOCK, "local rank group: barrier timed out");
+    return MF_OK;
+}
 }  // namespace
 
 mf_status mg_solve(const TileMatrix& A, DistInfo& D, const double* b, double* x, const mf_solve_opts& o, mf_solve_info* info,
@@ -848,6 +855,7 @@ mf_status mg_solve(const TileMatrix& A, DistInfo& D, const double* b, double* x,
     L.prelaunch = mg_prelaunch;
     L.ctx = &ctx;
     L.plain_launch = D.comm->local != nullptr;
+    L.postlaunch = mg_postlaunch;
     return run_solve(A, false, b, x, o, info, s, &L);
 }
 

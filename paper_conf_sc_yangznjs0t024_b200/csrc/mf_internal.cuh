@@ -146,6 +146,9 @@ struct MgLaunch {
     // cooperative launches of the ranks' kernels are refused / serialised by the driver, and the
     // ranks' grids must run side by side (co-residency is the caller's plan: G * nranks <= SMs)
     bool plain_launch = false;
+    // after the launch call returned, before any blocking call (local group: a host barrier, so
+    // every rank's kernel is enqueued before a thread blocks in the driver on its own kernel)
+    mf_status (*postlaunch)(void* ctx) = nullptr;
 };
 
 // Dynamic shared memory limit of a kernel = the opt-in maximum minus its static shared memory.

@@ -65,6 +65,8 @@ struct SolveArgs {
     int mu_cap;
     int nst, slot_bytes, blob_cap, ecap;   // TMA ring + decode buffers of the SpMV (tile-synchronous layout)
     int stall_cta;                   // test hook: this CTA never publishes (-1: none)
+    int cluster;                     // 1: the whole grid is ONE thread-block cluster (G <= 16): grid
+                                     // barriers and the SpMV-input wait are hardware cluster barriers
     unsigned long long timeout_ns;
     // ILU(0) preconditioner (PCG / right-preconditioned PBiCGSTAB); null when unpreconditioned
     const int64_t* Lrp; const int32_t* Lci; const double* Lv;
@@ -139,9 +141,22 @@ __device__ unsigned long long* spin_ns_smem() {
     return &spin_ns;
 }
 
+// every thread of every CTA of the cluster; orders (release / acquire, cluster scope) all prior
+// memory accesses of the cluster's threads, global memory included
+__device__ __forceinline__ void cluster_sync_all() {
+    unsigned long long t0 = 0;
+    if (threadIdx.x == 0) t0 = gtimer();
+    asm volatile("barrier.cluster.arrive.release.aligned;\n\tbarrier.cluster.wait.acquire.aligned;" ::: "memory");
+    if (threadIdx.x == 0) *spin_ns_smem() += gtimer() - t0;
+}
+
 __device__ __forceinline__ bool grid_barrier(const SolveArgs& a, Ctx& c) {
     __shared__ int s_abort;
     c.bar_target += (unsigned)a.G;
+    if (a.cluster) {                      // all CTAs in one cluster: barrier.cluster (release / acquire)
+        cluster_sync_all();
+        return true;
+    }
     __syncthreads();
     if (a.G == 1) return true;            // one CTA (small matrices): the CTA barrier orders everything
     if (threadIdx.x == 0) {
@@ -216,6 +231,10 @@ __device__ __forceinline__ bool mg_wait_halo(const SolveArgs& a, unsigned epoch,
 template <bool MG = false>
 __device__ __forceinline__ bool wait_deps(const SolveArgs& a, unsigned epoch) {
     __shared__ int s_abort;
+    if (a.cluster && a.stall_cta < 0 && !(MG && a.mg.P > 1)) {  // one cluster: every CTA published (barrier)
+        cluster_sync_all();
+        return true;
+    }
     if (a.G == 1 && a.stall_cta < 0 && !(MG && a.mg.P > 1)) {   // one CTA: its own writes, ordered by the CTA barrier
         __syncthreads();
         return true;
