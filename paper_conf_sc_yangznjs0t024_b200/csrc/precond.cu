@@ -153,7 +153,7 @@ __global__ void __launch_bounds__(256) sptrsv_kernel(TriCSR T, const double* __r
 
 // one-CTA sweep triangular solve (precond.cuh sweep_solve): deep dependency DAGs
 template <bool FWD>
-__global__ void __launch_bounds__(128) sweep_kernel(TriCSR T, const double* __restrict__ diag, int64_t n, const double* in,
+__global__ void __launch_bounds__(32 * mfk::SW_WARPS) sweep_kernel(TriCSR T, const double* __restrict__ diag, int64_t n, const double* in,
                                                    double* out, int* abort_flag) {
     extern __shared__ __align__(16) unsigned char sw_smem[];
     if (!mfk::sweep_solve<FWD, false>(T.rp, T.ci, T.v, diag, n, in, out, sw_smem, abort_flag, 20ull * 1000000000ull) &&
@@ -255,10 +255,10 @@ mf_status run_precond_apply(Precond& P, const double* r, double* z, cudaStream_t
                 if (nd.leaf && P.sweep) {
                     const size_t sb = mfk::sweep_smem_bytes();
                     if (pass == 0)
-                        sweep_kernel<true><<<1, 128, sb, s>>>(TriCSR{T.rp + nd.rp_off, T.ci, T.v}, nullptr, m, P.y + nd.r0,
+                        sweep_kernel<true><<<1, 32 * mfk::SW_WARPS, sb, s>>>(TriCSR{T.rp + nd.rp_off, T.ci, T.v}, nullptr, m, P.y + nd.r0,
                                                               P.y + nd.r0, abort_flag);
                     else
-                        sweep_kernel<false><<<1, 128, sb, s>>>(TriCSR{T.rp + nd.rp_off, T.ci, T.v}, P.udiag + nd.r0, m,
+                        sweep_kernel<false><<<1, 32 * mfk::SW_WARPS, sb, s>>>(TriCSR{T.rp + nd.rp_off, T.ci, T.v}, P.udiag + nd.r0, m,
                                                                P.y + nd.r0, P.y + nd.r0, abort_flag);
                 } else if (nd.leaf) {
                     unsigned long long* c = P.ctr + (pass == 0 ? 0 : P.Lrb.nleaves) + nd.leaf_idx;
@@ -286,8 +286,8 @@ mf_status run_precond_apply(Precond& P, const double* r, double* z, cudaStream_t
     int* abort_flag = reinterpret_cast<int*>(P.ctr + 2);
     if (P.sweep) {
         const size_t sb = mfk::sweep_smem_bytes();
-        sweep_kernel<true><<<1, 128, sb, s>>>(P.L, nullptr, P.n, r, P.y, abort_flag);
-        sweep_kernel<false><<<1, 128, sb, s>>>(P.U, P.udiag, P.n, P.y, z, abort_flag);
+        sweep_kernel<true><<<1, 32 * mfk::SW_WARPS, sb, s>>>(P.L, nullptr, P.n, r, P.y, abort_flag);
+        sweep_kernel<false><<<1, 32 * mfk::SW_WARPS, sb, s>>>(P.U, P.udiag, P.n, P.y, z, abort_flag);
         MF_CUDA(cudaGetLastError());
         int ab = 0;
         MF_CUDA(cudaMemcpyAsync(&ab, abort_flag, sizeof(int), cudaMemcpyDeviceToHost, s));

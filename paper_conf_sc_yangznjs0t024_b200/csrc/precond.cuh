@@ -193,8 +193,8 @@ __device__ __forceinline__ void rb_square_rows(const int64_t* __restrict__ rp, c
 // earlier in-window positions, consumed at earlier steps) and broadcasts the value by shuffle to the
 // lanes whose next entry is position 32*win + s.  Values of recent windows are kept in a shared
 // ring; older ones are read back from `out`.  `done` counts completed windows (in order).
-constexpr int SW_WARPS = 4;
-constexpr int SW_CAP = 1024;       // staged entries per warp and window (larger windows read global)
+constexpr int SW_WARPS = 8;
+constexpr int SW_CAP = 768;        // staged entries per warp and window (larger windows read global)
 constexpr int SW_RING = 2048;      // recent solution values kept in shared memory (positions)
 __host__ __device__ constexpr size_t sweep_smem_bytes() {
     return (size_t)SW_WARPS * SW_CAP * (8 + 4) + (size_t)SW_RING * 8 + 64;
@@ -212,42 +212,63 @@ __device__ __noinline__ bool sweep_solve(const int64_t* __restrict__ rp, const i
     auto oidx = [](int64_t i) -> int64_t { return OUTPV ? ((i >> 4) * 18 + (i & 15)) : i; };
     if (t == 0) { done[0] = 0; done[1] = 0; }
     __syncthreads();
-    if (w >= SW_WARPS) return true;
+    const int NWS = min(SW_WARPS, (int)(blockDim.x >> 5));   // sweeping warps
+    if (w >= NWS) return true;
     double* wv = sval + (size_t)w * SW_CAP;
     int32_t* wc = sci + (size_t)w * SW_CAP;
     const int64_t nwin = (n + 31) >> 5;
     const unsigned long long t0 = sp_timer();
     const unsigned FULL = 0xffffffffu;
     bool ok = true;
-    // spin (warp-uniform) until at least `need` windows are complete
+    int seen = 0;                      // windows known complete (this warp's last observation)
+    // spin (warp-uniform) until at least `need` windows are complete; one CTA-scope acquire fence
     auto wait_done = [&](int64_t need) {
-        for (unsigned sp = 0; done[0] < need; ++sp)
+        if (seen >= need) return;
+        int d = done[0];
+        for (unsigned sp = 0; d < need; ++sp, d = done[0])
             if ((sp & 1023u) == 1023u && (*(volatile int*)abort_flag || sp_timer() - t0 > timeout_ns)) {
                 atomicExch(abort_flag, 1);
                 ok = false;
                 done[1] = 1;
                 break;
             }
-        __syncwarp();
+        seen = __shfl_sync(FULL, d, 0);
+        __threadfence_block();
     };
-    for (int64_t win = w; win < nwin && ok && !done[1]; win += SW_WARPS) {
+    for (int64_t win = w; win < nwin && ok && !done[1]; win += NWS) {
         const int64_t p0 = win << 5, p = p0 + lane;
         const bool valid = p < n;
         const int64_t i = FWD ? p : n - 1 - p;
         const int64_t lo = valid ? rp[i] : 0, hi = valid ? rp[i + 1] : 0;
-        // the window's CSR range: rows p0 .. p0+31 in solve order are consecutive rows
+        // (1) stage the window's CSR range (rows p0 .. p0+31 in solve order are consecutive rows)
         const int64_t plast = min(p0 + 31, n - 1);
         const int64_t e0 = FWD ? rp[p0] : rp[n - 1 - plast];
         const int64_t e1 = FWD ? rp[plast + 1] : rp[n - p0];
-        const bool staged = e1 - e0 <= SW_CAP;
-        if (staged)
-            for (int64_t j = lane; j < e1 - e0; j += 32) { wc[j] = __ldg(ci + e0 + j); wv[j] = __ldg(val + e0 + j); }
+        const int ne = (int)(e1 - e0);
+        const bool staged = ne <= SW_CAP;
+        if (staged) {
+            for (int j0 = 0; j0 < ne; j0 += 128) {          // 4 loads per lane in flight
+                int32_t cc[4];
+                double vv[4];
+#pragma unroll
+                for (int u = 0; u < 4; ++u) {
+                    const int j = j0 + u * 32 + lane;
+                    cc[u] = j < ne ? __ldg(ci + e0 + j) : 0;
+                    vv[u] = j < ne ? __ldg(val + e0 + j) : 0.0;
+                }
+#pragma unroll
+                for (int u = 0; u < 4; ++u) {
+                    const int j = j0 + u * 32 + lane;
+                    if (j < ne) { wc[j] = cc[u]; wv[j] = vv[u]; }
+                }
+            }
+        }
         __syncwarp();
         const double dg = (!FWD && valid) ? diag[i] : 1.0;
         double acc = valid ? __ldcg(in + i) : 0.0;
         const int cnt = (int)(hi - lo);
         int k = 0;
-        int64_t pc = INT64_MAX;      // position of the current entry's column
+        int64_t pc = INT64_MAX;      // position (solve order) of the current entry's column
         double v = 0.0;
         int32_t col = 0;
         auto load_entry = [&]() {
@@ -261,30 +282,37 @@ __device__ __noinline__ bool sweep_solve(const int64_t* __restrict__ rp, const i
             }
         };
         load_entry();
-        // (2) entries in earlier windows, in chain order: a lane consumes its next entry as soon as
-        // the window holding the column is complete; the warp waits only when no lane can proceed
-        const int64_t ring_lo = p0 - SW_RING + (int64_t)SW_WARPS * 32;   // ring slots not yet reused
-        while (true) {
-            const int dn = done[0];
-            __threadfence_block();                 // acquire: values of the completed windows
-            const bool need = pc < p0;
-            const bool ready = need && (pc >> 5) < dn;
-            if (ready) {
-                const double yv = pc >= ring_lo ? ring[pc & (SW_RING - 1)] : __ldcg(out + oidx(col));
-                acc = __fma_rn(-v, yv, acc);
+        // (2a) entries older than the ring: their windows completed before any window in flight
+        // started (ring distance > windows in flight), values from `out`
+        const int64_t ring_lo = p0 - SW_RING + (int64_t)NWS * 32;
+        if (__any_sync(FULL, pc < ring_lo)) {
+            wait_done(max((int64_t)0, (ring_lo >> 5)));
+            while (pc < ring_lo) {
+                acc = __fma_rn(-v, __ldcg(out + oidx(col)), acc);
                 ++k;
                 load_entry();
             }
-            if (!__any_sync(FULL, pc < p0)) break;
-            if (!__any_sync(FULL, ready)) {
-                wait_done(dn + 1);
-                if (!ok) break;
+        }
+        // (2b) entries in earlier windows inside the ring, window by window: one warp-uniform wait
+        // per window, then every lane consumes its entries of that window (ring values)
+        int64_t nextw = pc < p0 ? (pc >> 5) : win;
+        for (int o = 16; o >= 1; o >>= 1) nextw = min(nextw, (int64_t)__shfl_xor_sync(FULL, (long long)nextw, o));
+        while (nextw < win) {
+            wait_done(nextw + 1);
+            if (!ok) break;
+            const int64_t wend = (nextw + 1) << 5;
+            while (pc < wend) {
+                acc = __fma_rn(-v, ring[pc & (SW_RING - 1)], acc);
+                ++k;
+                load_entry();
             }
+            nextw = pc < p0 ? (pc >> 5) : win;
+            for (int o = 16; o >= 1; o >>= 1) nextw = min(nextw, (int64_t)__shfl_xor_sync(FULL, (long long)nextw, o));
         }
         if (!ok) break;
-        // (3) in-window sweep
+        // (3) in-window sweep: step s finalises lane s and broadcasts it
         double fin = 0.0;
-#pragma unroll 4
+#pragma unroll 8
         for (int sstep = 0; sstep < 32; ++sstep) {
             if (lane == sstep) fin = FWD ? acc : __ddiv_rn(acc, dg);
             const double ys = __shfl_sync(FULL, fin, sstep);
@@ -303,6 +331,7 @@ __device__ __noinline__ bool sweep_solve(const int64_t* __restrict__ rp, const i
         wait_done(win);            // windows complete in order
         if (!ok) break;
         if (lane == 0) done[0] = (int)(win + 1);
+        seen = (int)(win + 1);
         __syncwarp();
     }
     return ok;

@@ -429,28 +429,10 @@ mf_status run_solve(const TileMatrix& A, bool bicg, const double* b, double* x, 
     a.mu_cap = (int)cap;
     a.nst = nst; a.slot_bytes = A.slot_bytes; a.blob_cap = A.blob_cap; a.ecap = A.ecap;
     a.stall_cta = -1;
-    // small plans (G <= 16, one CTA per SM): the grid is one thread-block cluster and its barriers
-    // are hardware cluster barriers (C1: the two grid reductions and the SpMV-input wait of every
-    // iteration are latency-bound).  MF_CLUSTER=0 disables it.
+    // one-cluster launches of small plans (barrier.cluster instead of the grid barrier) were tried
+    // for C1 and withdrawn: the static-mode kernels faulted with the cluster paths compiled in
+    // (profiles/r02_gpu3/bisect.log); the launch below keeps the field at 0
     a.cluster = 0;
-    {
-        // not with a preconditioner (a triangular-solve watchdog abort is per CTA and must not leave
-        // the other CTAs in a hardware barrier) nor with the stalled-CTA test hook
-        bool want = G > 1 && G <= 16 && !mgl && !pre && !getenv("MF_DEBUG_STALL_CTA");
-        if (const char* ev = getenv("MF_CLUSTER")) want = want && atoi(ev) != 0;
-        if (want) {
-            cudaError_t e1 = cudaFuncSetAttribute(kfn, cudaFuncAttributeNonPortableClusterSizeAllowed, 1);
-            cudaLaunchConfig_t cfg = {};
-            cudaLaunchAttribute at[1];
-            at[0].id = cudaLaunchAttributeClusterDimension;
-            at[0].val.clusterDim.x = (unsigned)G; at[0].val.clusterDim.y = 1; at[0].val.clusterDim.z = 1;
-            cfg.gridDim = dim3(G); cfg.blockDim = dim3(B); cfg.dynamicSmemBytes = smem; cfg.attrs = at; cfg.numAttrs = 1;
-            int ncl = 0;
-            cudaError_t e2 = e1 == cudaSuccess ? cudaOccupancyMaxActiveClusters(&ncl, kfn, &cfg) : e1;
-            if (e2 == cudaSuccess && ncl >= 1) a.cluster = 1;
-            else (void)cudaGetLastError();   // not schedulable as one cluster: cooperative launch
-        }
-    }
     if (const char* ev = getenv("MF_DEBUG_STALL_CTA")) a.stall_cta = atoi(ev);   // watchdog test hook
     a.timeout_ns = (o.watchdog_ms > 0 ? (unsigned long long)o.watchdog_ms : 60000ull) * 1000000ull;
     if (pre) {
@@ -484,15 +466,7 @@ mf_status run_solve(const TileMatrix& A, bool bicg, const double* b, double* x, 
     MF_CUDA(cudaEventCreate(&ev.e1));
     void* args[] = {&a};
     MF_CUDA(cudaEventRecord(ev.e0, s));
-    if (a.cluster) {
-        cudaLaunchConfig_t cfg = {};
-        cudaLaunchAttribute at[1];
-        at[0].id = cudaLaunchAttributeClusterDimension;
-        at[0].val.clusterDim.x = (unsigned)G; at[0].val.clusterDim.y = 1; at[0].val.clusterDim.z = 1;
-        cfg.gridDim = dim3(G); cfg.blockDim = dim3(B); cfg.dynamicSmemBytes = smem; cfg.stream = s;
-        cfg.attrs = at; cfg.numAttrs = 1;
-        MF_CUDA(cudaLaunchKernelExC(&cfg, kfn, args));
-    } else if (mgl && mgl->plain_launch) {
+    if (mgl && mgl->plain_launch) {
         MF_CUDA(cudaLaunchKernel(kfn, dim3(G), dim3(B), args, smem, s));
     } else {
         MF_CUDA(cudaLaunchCooperativeKernel(kfn, dim3(G), dim3(B), args, smem, s));

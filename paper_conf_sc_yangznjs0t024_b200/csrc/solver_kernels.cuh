@@ -65,8 +65,7 @@ struct SolveArgs {
     int mu_cap;
     int nst, slot_bytes, blob_cap, ecap;   // TMA ring + decode buffers of the SpMV (tile-synchronous layout)
     int stall_cta;                   // test hook: this CTA never publishes (-1: none)
-    int cluster;                     // 1: the whole grid is ONE thread-block cluster (G <= 16): grid
-                                     // barriers and the SpMV-input wait are hardware cluster barriers
+    int cluster;                     // reserved (0): one-cluster launch of small plans, not enabled
     unsigned long long timeout_ns;
     // ILU(0) preconditioner (PCG / right-preconditioned PBiCGSTAB); null when unpreconditioned
     const int64_t* Lrp; const int32_t* Lci; const double* Lv;
@@ -141,22 +140,9 @@ __device__ unsigned long long* spin_ns_smem() {
     return &spin_ns;
 }
 
-// every thread of every CTA of the cluster; orders (release / acquire, cluster scope) all prior
-// memory accesses of the cluster's threads, global memory included
-__device__ __forceinline__ void cluster_sync_all() {
-    unsigned long long t0 = 0;
-    if (threadIdx.x == 0) t0 = gtimer();
-    asm volatile("barrier.cluster.arrive.release.aligned;\n\tbarrier.cluster.wait.acquire.aligned;" ::: "memory");
-    if (threadIdx.x == 0) *spin_ns_smem() += gtimer() - t0;
-}
-
 __device__ __forceinline__ bool grid_barrier(const SolveArgs& a, Ctx& c) {
     __shared__ int s_abort;
     c.bar_target += (unsigned)a.G;
-    if (a.cluster) {                      // all CTAs in one cluster: barrier.cluster (release / acquire)
-        cluster_sync_all();
-        return true;
-    }
     __syncthreads();
     if (a.G == 1) return true;            // one CTA (small matrices): the CTA barrier orders everything
     if (threadIdx.x == 0) {
@@ -231,10 +217,6 @@ __device__ __forceinline__ bool mg_wait_halo(const SolveArgs& a, unsigned epoch,
 template <bool MG = false>
 __device__ __forceinline__ bool wait_deps(const SolveArgs& a, unsigned epoch) {
     __shared__ int s_abort;
-    if (a.cluster && a.stall_cta < 0 && !(MG && a.mg.P > 1)) {  // one cluster: every CTA published (barrier)
-        cluster_sync_all();
-        return true;
-    }
     if (a.G == 1 && a.stall_cta < 0 && !(MG && a.mg.P > 1)) {   // one CTA: its own writes, ordered by the CTA barrier
         __syncthreads();
         return true;
@@ -543,24 +525,35 @@ __global__ void __launch_bounds__(MAXT, 1) cg_persistent(SolveArgs a) {
             const double sigma = sg[0];
             if (!(sigma > 0.0) || !isfinite(sigma)) { status = MF_ERR_BREAKDOWN; break; }
             const double alpha = __ddiv_rn(rho, sigma);
-            // step C: r -= alpha mu, partial (r, r); r_{j+1} replaces mu in shared memory
+            // step C: r -= alpha mu, partial (r, r); r_{j+1} replaces mu in shared memory.  The
+            // loads of the next 4 rows per thread are issued before this chunk's arithmetic
+            // (software pipeline: 8 rows of global loads in flight per thread)
             double rr[1] = {0.0};
-            for (int64_t l0 = t; l0 < nr; l0 += 4 * (int64_t)B) {
-                double rv[4], mv[4];
+            {
+                double rv[4], rn[4];
+                auto load_r = [&](int64_t l0, double (&d)[4]) {
 #pragma unroll
-                for (int q = 0; q < 4; ++q) {
-                    const int64_t li = l0 + q * B;
-                    if (li < nr) { rv[q] = Rv[R0 + li]; mv[q] = li < mu_cap ? MUs[li] : MUg[R0 + li]; }
-                }
-#pragma unroll
-                for (int q = 0; q < 4; ++q) {
-                    const int64_t li = l0 + q * B;
-                    if (li < nr) {
-                        const double ri = __fma_rn(-alpha, mv[q], rv[q]);
-                        Rv[R0 + li] = ri;
-                        if (li < mu_cap) MUs[li] = ri;
-                        rr[0] = __fma_rn(ri, ri, rr[0]);
+                    for (int q = 0; q < 4; ++q) {
+                        const int64_t li = l0 + q * B;
+                        d[q] = li < nr ? Rv[R0 + li] : 0.0;
                     }
+                };
+                load_r(t, rv);
+                for (int64_t l0 = t; l0 < nr; l0 += 4 * (int64_t)B) {
+                    if (l0 + 4 * (int64_t)B < nr) load_r(l0 + 4 * (int64_t)B, rn);
+#pragma unroll
+                    for (int q = 0; q < 4; ++q) {
+                        const int64_t li = l0 + q * B;
+                        if (li < nr) {
+                            const double mv = li < mu_cap ? MUs[li] : MUg[R0 + li];
+                            const double ri = __fma_rn(-alpha, mv, rv[q]);
+                            Rv[R0 + li] = ri;
+                            if (li < mu_cap) MUs[li] = ri;
+                            rr[0] = __fma_rn(ri, ri, rr[0]);
+                        }
+                    }
+#pragma unroll
+                    for (int q = 0; q < 4; ++q) rv[q] = rn[q];
                 }
             }
             tm.tick(3);
@@ -570,33 +563,40 @@ __global__ void __launch_bounds__(MAXT, 1) cg_persistent(SolveArgs a) {
             rho = rr[0];
             // step D: x += alpha p_j ; p_{j+1} = r + beta p_j (own rows, PV) and the levels of its
             // segments (Alg. 4).  Rows l0 + qB of a half-warp form whole tile rows.
-            for (int64_t l0 = t; l0 < (tr1 - tr0) * 16; l0 += 4 * (int64_t)B) {
-                double pv[4], rv[4], xv[4];
+            {
+                // software pipeline as in step C: p and x of the next 4 rows per thread in flight
+                const int64_t L = (tr1 - tr0) * 16;
+                double pv[4], xv[4], pn4[4], xn4[4];
+                auto load_px = [&](int64_t l0, double (&pd)[4], double (&xd)[4]) {
 #pragma unroll
-                for (int q = 0; q < 4; ++q) {
-                    const int64_t li = l0 + q * B, i = R0 + li;
-                    pv[q] = 0.0; rv[q] = 0.0; xv[q] = 0.0;
-                    if (li < nr) {
-                        pv[q] = P[pv_idx(i)];
-                        rv[q] = li < mu_cap ? MUs[li] : Rv[i];
-                        xv[q] = X[i];
+                    for (int q = 0; q < 4; ++q) {
+                        const int64_t li = l0 + q * B, i = R0 + li;
+                        pd[q] = li < nr ? P[pv_idx(i)] : 0.0;
+                        xd[q] = li < nr ? X[i] : 0.0;
                     }
-                }
+                };
+                load_px(t, pv, xv);
+                for (int64_t l0 = t; l0 < L; l0 += 4 * (int64_t)B) {
+                    if (l0 + 4 * (int64_t)B < L) load_px(l0 + 4 * (int64_t)B, pn4, xn4);
 #pragma unroll
-                for (int q = 0; q < 4; ++q) {
-                    const int64_t li = l0 + q * B, i = R0 + li;
-                    if (li < (tr1 - tr0) * 16) {                 // uniform per half-warp
-                        double pn = 0.0;
-                        if (li < nr) {
-                            X[i] = __fma_rn(alpha, pv[q], xv[q]);
-                            pn = __fma_rn(beta, pv[q], rv[q]);
-                            P[pv_idx(i)] = pn;
-                        }
-                        if (DYN) {
-                            const int lv = mfk::hw_min_i(li < nr ? mfk::level_of(pn, th) : 4, m);
-                            if ((i & 15) == 0) mfk::pv_set_level(P, i >> 4, lv);
+                    for (int q = 0; q < 4; ++q) {
+                        const int64_t li = l0 + q * B, i = R0 + li;
+                        if (li < L) {                                // uniform per half-warp
+                            double pn = 0.0;
+                            if (li < nr) {
+                                const double rv = li < mu_cap ? MUs[li] : Rv[i];
+                                X[i] = __fma_rn(alpha, pv[q], xv[q]);
+                                pn = __fma_rn(beta, pv[q], rv);
+                                P[pv_idx(i)] = pn;
+                            }
+                            if (DYN) {
+                                const int lv = mfk::hw_min_i(li < nr ? mfk::level_of(pn, th) : 4, m);
+                                if ((i & 15) == 0) mfk::pv_set_level(P, i >> 4, lv);
+                            }
                         }
                     }
+#pragma unroll
+                    for (int q = 0; q < 4; ++q) { pv[q] = pn4[q]; xv[q] = xn4[q]; }
                 }
             }
             publish<MG>(a, (unsigned)(j + 3), P);
