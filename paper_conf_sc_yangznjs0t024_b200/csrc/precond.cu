@@ -286,8 +286,14 @@ mf_status run_precond_apply(Precond& P, const double* r, double* z, cudaStream_t
     int* abort_flag = reinterpret_cast<int*>(P.ctr + 2);
     if (P.sweep) {
         const size_t sb = mfk::sweep_smem_bytes();
-        sweep_kernel<true><<<1, 32 * mfk::SW_WARPS, sb, s>>>(P.L, nullptr, P.n, r, P.y, abort_flag);
-        sweep_kernel<false><<<1, 32 * mfk::SW_WARPS, sb, s>>>(P.U, P.udiag, P.n, P.y, z, abort_flag);
+        int nthr = 32 * mfk::SW_WARPS;
+        if (const char* ev = getenv("MF_SWEEP_WARPS")) nthr = 32 * std::max(1, std::min(mfk::SW_WARPS, atoi(ev)));
+        if (const char* ev = getenv("MF_SWEEP_SLEEP")) {
+            const int v = atoi(ev);
+            MF_CUDA(cudaMemcpyToSymbolAsync(mfk::g_sweep_sleep_ns, &v, sizeof(int), 0, cudaMemcpyHostToDevice, s));
+        }
+        sweep_kernel<true><<<1, nthr, sb, s>>>(P.L, nullptr, P.n, r, P.y, abort_flag);
+        sweep_kernel<false><<<1, nthr, sb, s>>>(P.U, P.udiag, P.n, P.y, z, abort_flag);
         MF_CUDA(cudaGetLastError());
         int ab = 0;
         MF_CUDA(cudaMemcpyAsync(&ab, abort_flag, sizeof(int), cudaMemcpyDeviceToHost, s));

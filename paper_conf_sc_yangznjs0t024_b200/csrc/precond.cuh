@@ -199,6 +199,8 @@ constexpr int SW_RING = 2048;      // recent solution values kept in shared memo
 __host__ __device__ constexpr size_t sweep_smem_bytes() {
     return (size_t)SW_WARPS * SW_CAP * (8 + 4) + (size_t)SW_RING * 8 + 64;
 }
+// spin back-off of the waiting warps (ns, 0 = none): tuning knob of the standalone apply
+static __device__ int g_sweep_sleep_ns = 0;
 template <bool FWD, bool OUTPV>
 __device__ __noinline__ bool sweep_solve(const int64_t* __restrict__ rp, const int32_t* __restrict__ ci,
                                          const double* __restrict__ val, const double* __restrict__ diag, int64_t n,
@@ -225,13 +227,16 @@ __device__ __noinline__ bool sweep_solve(const int64_t* __restrict__ rp, const i
     auto wait_done = [&](int64_t need) {
         if (seen >= need) return;
         int d = done[0];
-        for (unsigned sp = 0; d < need; ++sp, d = done[0])
+        const int slp = g_sweep_sleep_ns;
+        for (unsigned sp = 0; d < need; ++sp, d = done[0]) {
+            if (slp) __nanosleep(slp);
             if ((sp & 1023u) == 1023u && (*(volatile int*)abort_flag || sp_timer() - t0 > timeout_ns)) {
                 atomicExch(abort_flag, 1);
                 ok = false;
                 done[1] = 1;
                 break;
             }
+        }
         seen = __shfl_sync(FULL, d, 0);
         __threadfence_block();
     };

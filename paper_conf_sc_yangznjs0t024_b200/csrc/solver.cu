@@ -332,7 +332,8 @@ mf_status run_solve(const TileMatrix& A, bool bicg, const double* b, double* x, 
     const size_t fixed = fixed_smem_bytes();
     const int64_t pre_smem = pre ? (int64_t)B * 12 + 32 + (P->sweep ? (int64_t)mfk::sweep_smem_bytes() + 32 : 0) : 0;
     const int64_t ebytes = A.ts ? (int64_t)(B / 32) * A.ecap * 128 : 0;
-    const int64_t avail = (int64_t)smem_optin - (int64_t)fixed - pre_smem - 128 - (int64_t)mfk::TS_CTRL_BYTES - ebytes;
+    // - 256: the carve's alignment padding and the +64 slack of `smem` below
+    const int64_t avail = (int64_t)smem_optin - (int64_t)fixed - pre_smem - 128 - (int64_t)mfk::TS_CTRL_BYTES - ebytes - 256;
     int64_t cap = 0;
     int nst = 1;
     bool mu_onchip = true;
