@@ -683,6 +683,9 @@ mf_status convert_csr(int64_t n_rows, int64_t n_cols, int64_t nnz, const int64_t
                       const double* vals, const mf_convert_opts& o, cudaStream_t s, TileMatrix* A) {
     int sms = 0;
     MF_TRY(check_device(&sms));
+    // launch-plan arguments are validated before any device work (nothing to release on failure)
+    if (o.block_threads != 0 && (o.block_threads % 32 || o.block_threads > 1024 || o.block_threads < 32))
+        return fail(MF_ERR_INVALID_ARG, "block_threads must be a multiple of 32 in [32, 1024]");
     A->n_rows = n_rows; A->n_cols = n_cols; A->nnz = nnz; A->owner_stream = s;
     A->ntr = (n_rows + TS - 1) / TS;
     const int64_t ntr = A->ntr;

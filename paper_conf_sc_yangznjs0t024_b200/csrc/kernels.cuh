@@ -281,14 +281,25 @@ __device__ __forceinline__ void ts_issue(const unsigned char* blob_base, uint32_
 }
 
 // exact upcast of the stored bits at precision e (0 FP64, 1 FP32, 2 FP16, 3 E4M3) to binary64
+__device__ __forceinline__ double f16b_to_f64(unsigned short b);
+__device__ __forceinline__ uint32_t e4m3x2_to_f16x2(uint32_t w);
 __device__ __forceinline__ double decode_val(int e, uint64_t raw) {
     const uint32_t lo = (uint32_t)raw;
-    const __half_raw h8 = __nv_cvt_fp8_to_halfraw((__nv_fp8_storage_t)(lo & 0xFFu), __NV_E4M3);
-    const unsigned short hb = e == 3 ? h8.x : (unsigned short)lo;
-    const float f16 = __half2float(__ushort_as_half(hb));
-    const float f = e >= 2 ? f16 : __uint_as_float(lo);
-    const double d = (double)f;
+    const unsigned short hb = e == 3 ? (unsigned short)e4m3x2_to_f16x2(lo & 0xFFu) : (unsigned short)lo;
+    const double d = e >= 2 ? f16b_to_f64(hb) : (double)__uint_as_float(lo);
     return e == 0 ? __longlong_as_double((long long)raw) : d;
+}
+// binary16 bits -> binary64 (exact; one F2F.F64.F16)
+__device__ __forceinline__ double f16b_to_f64(unsigned short b) {
+    double d;
+    asm("{\n\t.reg .f16 h;\n\tmov.b16 h, %1;\n\tcvt.f64.f16 %0, h;\n\t}" : "=d"(d) : "h"(b));
+    return d;
+}
+// two E4M3 bytes (bits 0..15 of w) -> two binary16 (exact; one F2FP.F16.E4M3.UNPACK_B), byte 0 in the low half
+__device__ __forceinline__ uint32_t e4m3x2_to_f16x2(uint32_t w) {
+    uint32_t r;
+    asm("cvt.rn.f16x2.e4m3x2 %0, %1;" : "=r"(r) : "h"((unsigned short)(w & 0xFFFFu)));
+    return r;
 }
 __device__ __forceinline__ double e4m3_lo(uint32_t w2) {   // the E4M3 byte in bits 0..7 -> binary64 (exact)
     const __half_raw h = __nv_cvt_fp8_to_halfraw((__nv_fp8_storage_t)(w2 & 0xFFu), __NV_E4M3);
@@ -342,10 +353,13 @@ __device__ __forceinline__ void ts_decode_group(const TsView& v, const unsigned 
             w[0] = (double)a.x; w[1] = (double)a.y; w[2] = (double)a.z; w[3] = (double)a.w;
         } else if (Q == 2) {
             const uint2 a = *reinterpret_cast<const uint2*>(src);
-            w[0] = h16(a.x); w[1] = h16(a.x >> 16); w[2] = h16(a.y); w[3] = h16(a.y >> 16);
+            w[0] = f16b_to_f64((unsigned short)a.x); w[1] = f16b_to_f64((unsigned short)(a.x >> 16));
+            w[2] = f16b_to_f64((unsigned short)a.y); w[3] = f16b_to_f64((unsigned short)(a.y >> 16));
         } else {
             const uint32_t a = *reinterpret_cast<const uint32_t*>(src);
-            w[0] = e4m3_lo(a); w[1] = e4m3_lo(a >> 8); w[2] = e4m3_lo(a >> 16); w[3] = e4m3_lo(a >> 24);
+            const uint32_t h01 = e4m3x2_to_f16x2(a), h23 = e4m3x2_to_f16x2(a >> 16);
+            w[0] = f16b_to_f64((unsigned short)h01); w[1] = f16b_to_f64((unsigned short)(h01 >> 16));
+            w[2] = f16b_to_f64((unsigned short)h23); w[3] = f16b_to_f64((unsigned short)(h23 >> 16));
         }
         if (DYN) {
             const uint32_t g = gd[u >> 2];

@@ -38,6 +38,7 @@ template <class T>
 mf_status alloc(T** p, size_t count, cudaStream_t s) {
     *p = nullptr;
     if (count == 0) return MF_OK;
+    if (count > SIZE_MAX / sizeof(T)) return fail(MF_ERR_OOM, "device allocation size overflows size_t");
     *p = static_cast<T*>(dev_alloc(count * sizeof(T), s));
     if (!*p) return fail(MF_ERR_OOM, "device allocation of " + std::to_string(count * sizeof(T)) + " bytes failed");
     return MF_OK;

@@ -15,6 +15,7 @@
 
 #include <algorithm>
 #include <cmath>
+#include <cstdio>
 #include <vector>
 
 #include "mf_internal.cuh"
@@ -292,8 +293,41 @@ mf_status run_precond_apply(Precond& P, const double* r, double* z, cudaStream_t
             const int v = atoi(ev);
             MF_CUDA(cudaMemcpyToSymbolAsync(mfk::g_sweep_sleep_ns, &v, sizeof(int), 0, cudaMemcpyHostToDevice, s));
         }
+        long long* dbg = nullptr;
+        const int64_t nwin = (P.n + 31) / 32;
+        const bool want_dbg = getenv("MF_SWEEP_DBG") != nullptr;
+        if (want_dbg) {
+            MF_CUDA(cudaMalloc(&dbg, (size_t)nwin * 3 * 8 * 2));
+            MF_CUDA(cudaMemcpyToSymbolAsync(mfk::g_sweep_dbg, &dbg, sizeof(dbg), 0, cudaMemcpyHostToDevice, s));
+        }
         sweep_kernel<true><<<1, nthr, sb, s>>>(P.L, nullptr, P.n, r, P.y, abort_flag);
+        if (want_dbg) {
+            long long* d2 = dbg + nwin * 3;
+            MF_CUDA(cudaMemcpyToSymbolAsync(mfk::g_sweep_dbg, &d2, sizeof(d2), 0, cudaMemcpyHostToDevice, s));
+        }
         sweep_kernel<false><<<1, nthr, sb, s>>>(P.U, P.udiag, P.n, P.y, z, abort_flag);
+        if (want_dbg) {
+            std::vector<long long> h((size_t)nwin * 6);
+            MF_CUDA(cudaMemcpyAsync(h.data(), dbg, h.size() * 8, cudaMemcpyDeviceToHost, s));
+            MF_CUDA(cudaStreamSynchronize(s));
+            for (int tri = 0; tri < 2; ++tri) {
+                const long long* d = h.data() + (size_t)tri * nwin * 3;
+                double gap = 0, sw = 0, tail = 0, step = 0;
+                int64_t cntw = 0;
+                for (int64_t w = 1; w < nwin; ++w) {
+                    gap += (double)(d[w * 3] - d[(w - 1) * 3 + 2]);
+                    sw += (double)(d[w * 3 + 1] - d[w * 3]);
+                    tail += (double)(d[w * 3 + 2] - d[w * 3 + 1]);
+                    step += (double)(d[w * 3 + 2] - d[(w - 1) * 3 + 2]);
+                    ++cntw;
+                }
+                fprintf(stderr, "sweep %s: cycles per window: signal-to-signal %.0f = gap (prev signal -> sweep start) %.0f + sweep %.0f + tail %.0f\n",
+                        tri ? "U" : "L", step / cntw, gap / cntw, sw / cntw, tail / cntw);
+            }
+            MF_CUDA(cudaFree(dbg));
+            long long* z0 = nullptr;
+            MF_CUDA(cudaMemcpyToSymbolAsync(mfk::g_sweep_dbg, &z0, sizeof(z0), 0, cudaMemcpyHostToDevice, s));
+        }
         MF_CUDA(cudaGetLastError());
         int ab = 0;
         MF_CUDA(cudaMemcpyAsync(&ab, abort_flag, sizeof(int), cudaMemcpyDeviceToHost, s));

@@ -199,8 +199,11 @@ constexpr int SW_RING = 2048;      // recent solution values kept in shared memo
 __host__ __device__ constexpr size_t sweep_smem_bytes() {
     return (size_t)SW_WARPS * SW_CAP * (8 + 4) + (size_t)SW_RING * 8 + 64;
 }
+__device__ __forceinline__ unsigned smem_u32_(const void* p) { return (unsigned)__cvta_generic_to_shared(p); }
 // spin back-off of the waiting warps (ns, 0 = none): tuning knob of the standalone apply
 static __device__ int g_sweep_sleep_ns = 0;
+// diagnostics (standalone apply, MF_SWEEP_DBG): per window clock64 at sweep start / end / signal
+static __device__ long long* g_sweep_dbg = nullptr;
 template <bool FWD, bool OUTPV>
 __device__ __noinline__ bool sweep_solve(const int64_t* __restrict__ rp, const int32_t* __restrict__ ci,
                                          const double* __restrict__ val, const double* __restrict__ diag, int64_t n,
@@ -246,31 +249,23 @@ __device__ __noinline__ bool sweep_solve(const int64_t* __restrict__ rp, const i
         const int64_t i = FWD ? p : n - 1 - p;
         const int64_t lo = valid ? rp[i] : 0, hi = valid ? rp[i + 1] : 0;
         // (1) stage the window's CSR range (rows p0 .. p0+31 in solve order are consecutive rows)
+        // with asynchronous global->shared copies (all in flight at once: one memory latency);
+        // the right-hand side and the diagonal are loaded alongside
         const int64_t plast = min(p0 + 31, n - 1);
         const int64_t e0 = FWD ? rp[p0] : rp[n - 1 - plast];
         const int64_t e1 = FWD ? rp[plast + 1] : rp[n - p0];
+        const double dg = (!FWD && valid) ? diag[i] : 1.0;
+        double acc = valid ? __ldcg(in + i) : 0.0;
         const int ne = (int)(e1 - e0);
         const bool staged = ne <= SW_CAP;
         if (staged) {
-            for (int j0 = 0; j0 < ne; j0 += 128) {          // 4 loads per lane in flight
-                int32_t cc[4];
-                double vv[4];
-#pragma unroll
-                for (int u = 0; u < 4; ++u) {
-                    const int j = j0 + u * 32 + lane;
-                    cc[u] = j < ne ? __ldg(ci + e0 + j) : 0;
-                    vv[u] = j < ne ? __ldg(val + e0 + j) : 0.0;
-                }
-#pragma unroll
-                for (int u = 0; u < 4; ++u) {
-                    const int j = j0 + u * 32 + lane;
-                    if (j < ne) { wc[j] = cc[u]; wv[j] = vv[u]; }
-                }
+            for (int j = lane; j < ne; j += 32) {
+                asm volatile("cp.async.ca.shared.global [%0], [%1], 4;" ::"r"(smem_u32_(wc + j)), "l"(ci + e0 + j) : "memory");
+                asm volatile("cp.async.ca.shared.global [%0], [%1], 8;" ::"r"(smem_u32_(wv + j)), "l"(val + e0 + j) : "memory");
             }
+            asm volatile("cp.async.wait_all;" ::: "memory");
         }
         __syncwarp();
-        const double dg = (!FWD && valid) ? diag[i] : 1.0;
-        double acc = valid ? __ldcg(in + i) : 0.0;
         const int cnt = (int)(hi - lo);
         int k = 0;
         int64_t pc = INT64_MAX;      // position (solve order) of the current entry's column
@@ -287,11 +282,28 @@ __device__ __noinline__ bool sweep_solve(const int64_t* __restrict__ rp, const i
             }
         };
         load_entry();
+        // the chain's tail (computed before any wait): entries in this window (bit s of hm =
+        // position p0 + s, from index kb) and in the previous window (bit s of pm = position
+        // p0 - 32 + s, from index kp); the older entries precede them in chain order
+        unsigned hm = 0, pm = 0;
+        int kb = cnt, kp = cnt;
+        for (int kk = cnt - 1; kk >= k; --kk) {
+            const int64_t q = FWD ? lo + kk : hi - 1 - kk;
+            const int32_t cc = staged ? wc[q - e0] : __ldg(ci + q);
+            const int64_t pcc = FWD ? (int64_t)cc : n - 1 - cc;
+            if (pcc >= p0) { hm |= 1u << (int)(pcc - p0); kb = kk; kp = kk; }
+            else if (pcc >= p0 - 32) { pm |= 1u << (int)(pcc - (p0 - 32)); kp = kk; }
+            else break;
+        }
+        const double yr = FWD ? 1.0 : __drcp_rn(dg);
+        const bool dg_ok = FWD || (fabs(dg) >= 0x1p-960 && fabs(dg) <= 0x1p960);
         // (2a) entries older than the ring: their windows completed before any window in flight
         // started (ring distance > windows in flight), values from `out`
         const int64_t ring_lo = p0 - SW_RING + (int64_t)NWS * 32;
         if (__any_sync(FULL, pc < ring_lo)) {
-            wait_done(max((int64_t)0, (ring_lo >> 5)));
+            // the writer of a column stores `out` after its signal; its next window's fence (NWS
+            // windows later) publishes it
+            wait_done(max((int64_t)0, (ring_lo >> 5) + NWS));
             while (pc < ring_lo) {
                 acc = __fma_rn(-v, __ldcg(out + oidx(col)), acc);
                 ++k;
@@ -300,9 +312,10 @@ __device__ __noinline__ bool sweep_solve(const int64_t* __restrict__ rp, const i
         }
         // (2b) entries in earlier windows inside the ring, window by window: one warp-uniform wait
         // per window, then every lane consumes its entries of that window (ring values)
-        int64_t nextw = pc < p0 ? (pc >> 5) : win;
+        const int64_t pprev = p0 - 32;            // the previous window is handled after its wait
+        int64_t nextw = pc < pprev ? (pc >> 5) : win;
         for (int o = 16; o >= 1; o >>= 1) nextw = min(nextw, (int64_t)__shfl_xor_sync(FULL, (long long)nextw, o));
-        while (nextw < win) {
+        while (nextw < win - 1) {
             wait_done(nextw + 1);
             if (!ok) break;
             const int64_t wend = (nextw + 1) << 5;
@@ -311,32 +324,95 @@ __device__ __noinline__ bool sweep_solve(const int64_t* __restrict__ rp, const i
                 ++k;
                 load_entry();
             }
-            nextw = pc < p0 ? (pc >> 5) : win;
+            nextw = pc < pprev ? (pc >> 5) : win;
             for (int o = 16; o >= 1; o >>= 1) nextw = min(nextw, (int64_t)__shfl_xor_sync(FULL, (long long)nextw, o));
         }
         if (!ok) break;
-        // (3) in-window sweep: step s finalises lane s and broadcasts it
+        // previous window: positions known in advance (pm), ring values read right after its wait
+        if (win > 0) wait_done(win);
+        if (!ok) break;
+        {
+            unsigned mm = pm;
+            int kk = kp;
+            while (mm) {
+                const int sb = __ffs(mm) - 1;
+                mm &= mm - 1u;
+                const int64_t q = FWD ? lo + kk : hi - 1 - kk;
+                const double vv = staged ? wv[q - e0] : __ldg(val + q);
+                acc = __fma_rn(-vv, ring[(pprev + sb) & (SW_RING - 1)], acc);
+                ++kk;
+            }
+            k = kb;
+        }
+        // (3) in-window sweep: the lane's remaining entries are in the window, ascending; hm has
+        // bit s for an entry at position p0 + s, its value is entry kb + popc(hm below s).  Step s
+        // broadcasts lane s's final value (all its entries precede position p0 + s); every step is
+        // branch-free: a predicated fma, then the lane's value refreshed.  !FWD: the quotient by
+        // diag_i with Markstein's correction of a*RN(1/d) (correctly rounded: RN(1/d) and a one-ulp
+        // q0 give RN(a/d) for normal operands), IEEE division for zero or extreme operands.
+        long long* dbg = g_sweep_dbg;
+        if (dbg && lane == 0) dbg[win * 3] = clock64();
+        const double acc0 = acc;
         double fin = 0.0;
+        bool slow = !staged;
+        if (staged) {
+            // fast path: every step branch-free (the value load uses a valid shared address for
+            // every lane, masked afterwards), Markstein quotient; any lane with an operand outside
+            // its validity range sends the whole window to the exact path below
+            const int vb0 = FWD ? (int)(lo - e0) + kb : (int)(hi - 1 - e0) - kb;   // staged index of entry kb
+            bool bad = false;
+            auto mark = [&](double a) -> double {
+                const double q0 = __dmul_rn(a, yr);
+                const double q1 = __fma_rn(__fma_rn(-q0, dg, a), yr, q0);
+                const double aq = fabs(q1);
+                bad |= a == 0.0 || !(aq >= 0x1p-960 && aq <= 0x1p960);
+                return q1;
+            };
+            fin = FWD ? acc : mark(acc);
 #pragma unroll 8
-        for (int sstep = 0; sstep < 32; ++sstep) {
-            if (lane == sstep) fin = FWD ? acc : __ddiv_rn(acc, dg);
-            const double ys = __shfl_sync(FULL, fin, sstep);
-            if (pc == p0 + sstep) {
-                acc = __fma_rn(-v, ys, acc);
-                ++k;
-                load_entry();
+            for (int sstep = 0; sstep < 32; ++sstep) {
+                const bool hit = (hm >> sstep) & 1u;
+                const int r = __popc(hm & ((1u << sstep) - 1u));
+                const double vraw = wv[hit ? (FWD ? vb0 + r : vb0 - r) : 0];   // a valid address for every lane
+                const double vv = hit ? vraw : 0.0;
+                const double ys = __shfl_sync(FULL, fin, sstep);
+                const double na = __fma_rn(-vv, ys, acc);
+                acc = hit ? na : acc;
+                if (FWD) fin = acc;
+                else { const double nf = mark(acc); fin = hit ? nf : fin; }
+            }
+            if (!FWD) slow = __any_sync(FULL, bad || !dg_ok);
+        }
+        if (slow) {
+            // exact path: IEEE division, values from the staged buffer or global memory
+            acc = acc0;
+            fin = FWD ? acc : __ddiv_rn(acc, dg);
+            for (int sstep = 0; sstep < 32; ++sstep) {
+                const bool hit = (hm >> sstep) & 1u;
+                double vv = 0.0;
+                if (hit) {
+                    const int idx = kb + __popc(hm & ((1u << sstep) - 1u));
+                    const int64_t q = FWD ? lo + idx : hi - 1 - idx;
+                    vv = staged ? wv[q - e0] : __ldg(val + q);
+                }
+                const double ys = __shfl_sync(FULL, fin, sstep);
+                const double na = __fma_rn(-vv, ys, acc);
+                acc = hit ? na : acc;
+                if (hit) fin = FWD ? acc : __ddiv_rn(acc, dg);
             }
         }
-        if (valid) {
-            out[oidx(i)] = fin;
-            ring[p & (SW_RING - 1)] = fin;
-        }
-        __threadfence_block();
+        if (dbg && lane == 0) dbg[win * 3 + 1] = clock64();
+        if (valid) ring[p & (SW_RING - 1)] = fin;
+        __threadfence_block();     // the ring values (shared memory) before the signal
         __syncwarp();
         wait_done(win);            // windows complete in order
         if (!ok) break;
         if (lane == 0) done[0] = (int)(win + 1);
+        if (dbg && lane == 0) dbg[win * 3 + 2] = clock64();
         seen = (int)(win + 1);
+        // the global copy after the signal: readers of `out` (columns older than the ring) start
+        // at least SW_RING / 32 - NWS windows later, after this warp's later fences
+        if (valid) out[oidx(i)] = fin;
         __syncwarp();
     }
     return ok;

@@ -179,6 +179,8 @@ struct Events {
 mf_status run_spmv(const TileMatrix& A, const double* x, double* y, const uint8_t* level, int range_guard,
                    int64_t* counts_host, cudaStream_t s) {
     if (A.ntr == 0) return MF_OK;
+    if (!A.ts && (A.n_cols + 15) / 16 > ((int64_t)1 << 28))
+        return fail(MF_ERR_UNSUPPORTED, "compact layout: more than 2^28 tile columns");
     int dev = 0, smem_optin = 0;
     MF_CUDA(cudaGetDevice(&dev));
     MF_CUDA(cudaDeviceGetAttribute(&smem_optin, cudaDevAttrMaxSharedMemoryPerBlockOptin, dev));

@@ -84,6 +84,30 @@ def main():
                    "source": f"profiles/{tag}_ncu_cg.txt"}
         json.dump(d, open(tp, "w"), indent=1)
         print("\n".join(lines))
+    # DRAM traffic of the other configs' persistent solves (tools/gpu_final_r2.sh: ncu --metrics
+    # dram__bytes_read.sum,dram__bytes_write.sum on one solve each, gpurun_out/traffic_<cfg>.csv)
+    tp = os.path.join(PROF, "ncu_traffic.json")
+    d = json.load(open(tp)) if os.path.exists(tp) else {}
+    for f in sorted(os.listdir(OUT)):
+        if not (f.startswith("traffic_") and f.endswith(".csv")):
+            continue
+        cfg = f[len("traffic_"):-4]
+        lines = open(os.path.join(OUT, f)).read().splitlines()
+        hdr = [k for k, l in enumerate(lines) if l.startswith('"ID"')]
+        if not hdr:
+            continue
+        tot, kern = 0.0, None
+        for r in csv.DictReader(lines[hdr[0]:]):
+            if "_persistent" not in r["Kernel Name"]:
+                continue
+            kern = r["Kernel Name"].split("(")[0]
+            tot += to_bytes(r["Metric Unit"], r["Metric Value"])
+        if kern:
+            d[cfg] = {"dram_bytes_per_launch": tot, "kernel": kern + " (one launch = one whole solve)",
+                      "source": f"profiles/{tag}_traffic_{cfg}.csv"}
+            open(os.path.join(PROF, f"{tag}_traffic_{cfg}.csv"), "w").write("\n".join(lines[hdr[0]:]) + "\n")
+            print(cfg, kern, f"{tot/1e9:.3f} GB per launch")
+    json.dump(d, open(tp, "w"), indent=1)
 
 
 if __name__ == "__main__":
