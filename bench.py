@@ -244,6 +244,15 @@ def gpu_arm(args, rank, world):
             if T is not None:
                 close(T)
         modes["dynamic_vs_fp64_time_to_solution"] = round(modes["fp64"]["solve_ms"] / modes["dynamic"]["solve_ms"], 3)
+        if not pre:
+            # the paper-literal sticky downgrade (reading R9): iteration inflation against the
+            # per-iteration switch (cf. Table II)
+            T, r = step(mode=mf.MODE_DYNAMIC, sticky=1, raise_on_breakdown=False)
+            modes["sticky"] = {"iterations": r.iterations, "converged": r.converged, "status": r.status,
+                               "solve_ms": round(r.kernel_ms, 3),
+                               "us_per_iter": round(r.kernel_ms / max(r.iterations, 1) * 1e3, 2),
+                               "iterations_vs_dynamic": round(r.iterations / max(stats.iterations, 1), 4)}
+            close(T)
 
     peaks = _peaks()
     kms = statistics.mean(kern_ms)
@@ -285,7 +294,8 @@ def gpu_arm(args, rank, world):
         "effective_gbs": round(achieved, 1),
         "barrier_share": round(statistics.mean(bar_ms) / kms, 4),
         "phase_us_per_iter": phase_us,
-        "precision": {"tile_prec_mix": tp_mix, "dynamic_level_mix": mix},
+        "precision": {"tile_prec_mix": tp_mix, "dynamic_level_mix": mix,
+                      "nnz_prec_mix": [round(v / max(sum(info0["nval"]), 1), 4) for v in info0["nval"]]},
         "modes": modes,
         "memory": {"csr_bytes": info0["csr_bytes"], "canonical_bytes": info0["canonical_bytes"],
                    "kernel_bytes": info0["kernel_bytes"],
