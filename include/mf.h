@@ -177,7 +177,7 @@ mf_status mf_tile_matrix_export(const mf_tile_matrix* A, mf_tile_export* host, m
 mf_status mf_spmv(const mf_tile_matrix* A, const double* x, double* y, const uint8_t* level,
                   int32_t range_guard, int64_t* counts, mf_stream stream);
 /* Convergent-element retrieval (Alg. 4): level[J] of each 16-element segment of v
- * from thresholds th (host, 4 ascending doubles). */
+ * from thresholds th (host, 4 non-decreasing doubles; otherwise MF_ERR_INVALID_ARG). */
 mf_status mf_levels(const double* v, int64_t n, const double* th, uint8_t* level, mf_stream stream);
 /* (u, v) with the matrix's launch-plan reduction tree; host result. */
 mf_status mf_dot(const mf_tile_matrix* A, const double* u, const double* v, double* out, mf_stream stream);

@@ -850,13 +850,12 @@ __device__ __forceinline__ void spmv_cta(const Mat& A, int64_t tr0, int64_t tr1,
 struct Thresh {
     double t0, t1, t2, t3;
 };
+// Branch-free: the number of thresholds above |v|.  Equal to the interval test (a < t0 -> 4, else
+// a < t1 -> 3, ...) because the thresholds are tau * {1e-3, 1e-2, 1e-1, 1} rounded: non-decreasing
+// for tau >= 0, all negative (every comparison false, level 0) for tau < 0; NaN -> 0 (FP64).
 __device__ __forceinline__ int level_of(double v, const Thresh& th) {
     const double a = fabs(v);
-    if (a < th.t0) return 4;
-    if (a < th.t1) return 3;
-    if (a < th.t2) return 2;
-    if (a < th.t3) return 1;
-    return 0;   // includes NaN
+    return (int)(a < th.t0) + (int)(a < th.t1) + (int)(a < th.t2) + (int)(a < th.t3);
 }
 
 // ---- reductions

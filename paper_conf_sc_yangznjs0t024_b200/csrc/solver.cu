@@ -244,6 +244,8 @@ mf_status run_spmv(const TileMatrix& A, const double* x, double* y, const uint8_
 }
 
 mf_status run_levels(const double* v, int64_t n, const double* th, uint8_t* level, cudaStream_t s) {
+    if (!(th[0] <= th[1] && th[1] <= th[2] && th[2] <= th[3]))
+        return fail(MF_ERR_INVALID_ARG, "mf_levels: thresholds must be non-decreasing");
     if (n == 0) return MF_OK;
     Thresh t{th[0], th[1], th[2], th[3]};
     int64_t nseg = (n + 15) / 16;

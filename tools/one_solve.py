@@ -18,6 +18,6 @@ spec = W.CONFIGS[name]
 fn = mf.cg_solve if spec["solver"] == "cg" else mf.bicgstab_solve
 for _ in range(reps):
     T = mf.TileMatrix(A.n_rows, A.n_cols, rp, ci, va)
-    r = fn(T, b, max_iter=spec["max_iter"], mode=mode, history=False)
+    r = fn(T, b, max_iter=spec["max_iter"], mode=mode, history=False, switch_eps=spec.get("switch_eps"))
     print(name, r.iterations, r.converged, f"{r.kernel_ms:.3f} ms", T.info()["convert_ms"], flush=True)
     T.close()
