@@ -297,32 +297,38 @@ mf_status run_precond_apply(Precond& P, const double* r, double* z, cudaStream_t
         const int64_t nwin = (P.n + 31) / 32;
         const bool want_dbg = getenv("MF_SWEEP_DBG") != nullptr;
         if (want_dbg) {
-            MF_CUDA(cudaMalloc(&dbg, (size_t)nwin * 3 * 8 * 2));
+            MF_CUDA(cudaMalloc(&dbg, (size_t)nwin * 5 * 8 * 2));
             MF_CUDA(cudaMemcpyToSymbolAsync(mfk::g_sweep_dbg, &dbg, sizeof(dbg), 0, cudaMemcpyHostToDevice, s));
         }
         sweep_kernel<true><<<1, nthr, sb, s>>>(P.L, nullptr, P.n, r, P.y, abort_flag);
         if (want_dbg) {
-            long long* d2 = dbg + nwin * 3;
+            long long* d2 = dbg + nwin * 5;
             MF_CUDA(cudaMemcpyToSymbolAsync(mfk::g_sweep_dbg, &d2, sizeof(d2), 0, cudaMemcpyHostToDevice, s));
         }
         sweep_kernel<false><<<1, nthr, sb, s>>>(P.U, P.udiag, P.n, P.y, z, abort_flag);
         if (want_dbg) {
-            std::vector<long long> h((size_t)nwin * 6);
+            std::vector<long long> h((size_t)nwin * 10);
             MF_CUDA(cudaMemcpyAsync(h.data(), dbg, h.size() * 8, cudaMemcpyDeviceToHost, s));
             MF_CUDA(cudaStreamSynchronize(s));
             for (int tri = 0; tri < 2; ++tri) {
-                const long long* d = h.data() + (size_t)tri * nwin * 3;
-                double gap = 0, sw = 0, tail = 0, step = 0;
+                const long long* d = h.data() + (size_t)tri * nwin * 5;
+                // per window: [0] before the previous-window wait, [1] wait returned, [2] sweep start,
+                // [3] sweep end, [4] signal
+                double pre = 0, hand = 0, prev = 0, sw = 0, tail = 0, step = 0;
                 int64_t cntw = 0;
                 for (int64_t w = 1; w < nwin; ++w) {
-                    gap += (double)(d[w * 3] - d[(w - 1) * 3 + 2]);
-                    sw += (double)(d[w * 3 + 1] - d[w * 3]);
-                    tail += (double)(d[w * 3 + 2] - d[w * 3 + 1]);
-                    step += (double)(d[w * 3 + 2] - d[(w - 1) * 3 + 2]);
+                    const long long sig_prev = d[(w - 1) * 5 + 4];
+                    hand += (double)(d[w * 5 + 1] - sig_prev);        // previous signal -> wait returns
+                    pre += (double)(d[w * 5] > sig_prev ? d[w * 5] - sig_prev : 0);   // arrived late at the wait
+                    prev += (double)(d[w * 5 + 2] - d[w * 5 + 1]);
+                    sw += (double)(d[w * 5 + 3] - d[w * 5 + 2]);
+                    tail += (double)(d[w * 5 + 4] - d[w * 5 + 3]);
+                    step += (double)(d[w * 5 + 4] - sig_prev);
                     ++cntw;
                 }
-                fprintf(stderr, "sweep %s: cycles per window: signal-to-signal %.0f = gap (prev signal -> sweep start) %.0f + sweep %.0f + tail %.0f\n",
-                        tri ? "U" : "L", step / cntw, gap / cntw, sw / cntw, tail / cntw);
+                fprintf(stderr, "sweep %s: cycles per window: signal-to-signal %.0f = signal->wait-return %.0f (of which the warp "
+                        "arrived late %.0f) + previous-window entries %.0f + sweep %.0f + signalling %.0f\n",
+                        tri ? "U" : "L", step / cntw, hand / cntw, pre / cntw, prev / cntw, sw / cntw, tail / cntw);
             }
             MF_CUDA(cudaFree(dbg));
             long long* z0 = nullptr;

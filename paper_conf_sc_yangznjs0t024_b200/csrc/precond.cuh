@@ -328,13 +328,41 @@ __device__ __noinline__ bool sweep_solve(const int64_t* __restrict__ rp, const i
             for (int o = 16; o >= 1; o >>= 1) nextw = min(nextw, (int64_t)__shfl_xor_sync(FULL, (long long)nextw, o));
         }
         if (!ok) break;
-        // previous window: positions known in advance (pm), ring values read right after its wait
+        // previous window: positions known in advance (pm).  The first SW_PK entries' values and
+        // ring slots are gathered into registers BEFORE the wait; after it, their ring values are
+        // read together and the fma chain runs without per-entry address work; more entries (rare)
+        // continue in a loop.
+        constexpr int SW_PK = 8;
+        double pvv[SW_PK];
+        int pslot[SW_PK];
+        unsigned mm = pm;
+        const int npk = min(__popc(pm), SW_PK);
+        const int wpk = __reduce_max_sync(FULL, (unsigned)npk);     // the warp's longest preloaded chain
+#pragma unroll
+        for (int u = 0; u < SW_PK; ++u) {
+            const int sb = mm ? __ffs(mm) - 1 : 0;
+            if (mm) mm &= mm - 1u;
+            const int64_t q = FWD ? lo + kp + u : hi - 1 - (kp + u);
+            pvv[u] = u < npk ? (staged ? wv[q - e0] : __ldg(val + q)) : 0.0;
+            pslot[u] = (int)((pprev + sb) & (SW_RING - 1));
+        }
+        long long* dbg = g_sweep_dbg;
+        if (dbg && lane == 0) dbg[win * 5] = clock64();
         if (win > 0) wait_done(win);
         if (!ok) break;
+        if (dbg && lane == 0) dbg[win * 5 + 1] = clock64();
         {
-            unsigned mm = pm;
-            int kk = kp;
-            while (mm) {
+            double ry[SW_PK];
+#pragma unroll
+            for (int u = 0; u < SW_PK; ++u) ry[u] = ring[pslot[u]];     // valid slots for every lane
+#pragma unroll
+            for (int u = 0; u < SW_PK; ++u) {
+                if (u >= wpk) break;                                  // warp-uniform
+                const double na = __fma_rn(-pvv[u], ry[u], acc);
+                acc = u < npk ? na : acc;
+            }
+            int kk = kp + npk;
+            while (mm) {                                              // entries beyond SW_PK
                 const int sb = __ffs(mm) - 1;
                 mm &= mm - 1u;
                 const int64_t q = FWD ? lo + kk : hi - 1 - kk;
@@ -350,8 +378,7 @@ __device__ __noinline__ bool sweep_solve(const int64_t* __restrict__ rp, const i
         // branch-free: a predicated fma, then the lane's value refreshed.  !FWD: the quotient by
         // diag_i with Markstein's correction of a*RN(1/d) (correctly rounded: RN(1/d) and a one-ulp
         // q0 give RN(a/d) for normal operands), IEEE division for zero or extreme operands.
-        long long* dbg = g_sweep_dbg;
-        if (dbg && lane == 0) dbg[win * 3] = clock64();
+        if (dbg && lane == 0) dbg[win * 5 + 2] = clock64();
         const double acc0 = acc;
         double fin = 0.0;
         bool slow = !staged;
@@ -401,14 +428,14 @@ __device__ __noinline__ bool sweep_solve(const int64_t* __restrict__ rp, const i
                 if (hit) fin = FWD ? acc : __ddiv_rn(acc, dg);
             }
         }
-        if (dbg && lane == 0) dbg[win * 3 + 1] = clock64();
+        if (dbg && lane == 0) dbg[win * 5 + 3] = clock64();
         if (valid) ring[p & (SW_RING - 1)] = fin;
         __threadfence_block();     // the ring values (shared memory) before the signal
         __syncwarp();
         wait_done(win);            // windows complete in order
         if (!ok) break;
         if (lane == 0) done[0] = (int)(win + 1);
-        if (dbg && lane == 0) dbg[win * 3 + 2] = clock64();
+        if (dbg && lane == 0) dbg[win * 5 + 4] = clock64();
         seen = (int)(win + 1);
         // the global copy after the signal: readers of `out` (columns older than the ring) start
         // at least SW_RING / 32 - NWS windows later, after this warp's later fences
