@@ -310,9 +310,41 @@ __device__ __noinline__ bool sweep_solve(const int64_t* __restrict__ rp, const i
                 load_entry();
             }
         }
-        // (2b) entries in earlier windows inside the ring, window by window: one warp-uniform wait
-        // per window, then every lane consumes its entries of that window (ring values)
+        // (2b) entries in earlier windows inside the ring.  First every entry of a window already
+        // complete (one read of the counter), in batches of 4 whose loads are all in flight
+        // together (the fma chain is the only serial part); then the windows still in flight one
+        // by one (a warp-uniform wait each); the previous window last, after its own wait.
         const int64_t pprev = p0 - 32;            // the previous window is handled after its wait
+        if (staged) {
+            const int dn = done[0];
+            __threadfence_block();
+            const int64_t lim = min((int64_t)dn, win - 1) << 5;
+            while (__any_sync(FULL, pc < lim)) {
+                double yv[4], vv[4];
+                bool use[4];
+#pragma unroll
+                for (int u = 0; u < 4; ++u) {
+                    const int idx = k + u;
+                    const int64_t q = FWD ? lo + idx : hi - 1 - idx;
+                    const int qi = idx < cnt ? (int)(q - e0) : 0;
+                    const int32_t cc = wc[qi];
+                    const int64_t pcu = FWD ? (int64_t)cc : n - 1 - cc;
+                    use[u] = idx < cnt && pcu < lim;
+                    yv[u] = ring[use[u] ? (int)(pcu & (SW_RING - 1)) : 0];
+                    vv[u] = wv[qi];
+                }
+                int used = 0;
+#pragma unroll
+                for (int u = 0; u < 4; ++u) {
+                    const bool go = use[u] && used == u;        // positions ascend: a prefix is used
+                    const double na = __fma_rn(-vv[u], yv[u], acc);
+                    acc = go ? na : acc;
+                    used += go ? 1 : 0;
+                }
+                k += used;
+                load_entry();
+            }
+        }
         int64_t nextw = pc < pprev ? (pc >> 5) : win;
         for (int o = 16; o >= 1; o >>= 1) nextw = min(nextw, (int64_t)__shfl_xor_sync(FULL, (long long)nextw, o));
         while (nextw < win - 1) {

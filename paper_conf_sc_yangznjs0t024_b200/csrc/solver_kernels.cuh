@@ -151,7 +151,11 @@ __device__ __forceinline__ bool grid_barrier(const SolveArgs& a, Ctx& c) {
         int ab = 0;
         while (ld_acquire(a.bar) < c.bar_target) {
             if (*(volatile int*)a.abort_flag) { ab = 1; break; }
-            if (gtimer() - t0 > a.timeout_ns) { atomicExch(a.abort_flag, 1); ab = 1; break; }
+            const unsigned long long dt = gtimer() - t0;
+            if (dt > a.timeout_ns) { atomicExch(a.abort_flag, 1); ab = 1; break; }
+            // long waits (one CTA at work, e.g. the triangular-solve sweep): back off, so that
+            // 147 pollers do not keep the L2 line and the memory system busy
+            if (dt > 20000ull) __nanosleep(1000);
         }
         __threadfence();
         *spin_ns_smem() += gtimer() - t0;

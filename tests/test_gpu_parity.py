@@ -599,3 +599,24 @@ def test_single_reduction_cg_parity(mf, orc, name, make, G, B, mode):
     assert np.array_equal(rg.x.cpu().numpy(), ro["x"])
     if mode == 2:
         assert np.array_equal(rg.level_counts, ro["level_counts"])
+
+
+ABS_CASES = [("C2-32-cg", lambda: W.make("C2", 32), "cg", 1e-7, 8, 512),
+             ("C3-64-bicg", lambda: W.make("C3", 64), "bicgstab", 1e-9, 8, 256),
+             ("C4spd-12-cg", lambda: W.make("C4spd", 1 << 12), "cg", 1e-8, 6, 256)]
+
+
+@pytest.mark.parametrize("name,make,solver,eps,G,B", ABS_CASES, ids=[c[0] for c in ABS_CASES])
+def test_literal_absolute_tau_parity(mf, orc, name, make, solver, eps, G, B):
+    """switch_absolute=1 (the literal tau = eps of Alg. 1 l.3): histories, x and the per-SpMV
+    level counts bit-identical to the oracle, with the switch actually firing."""
+    A = make()
+    ro, rg, _ = run_pair(mf, orc, A, solver, 2, G=G, B=B, max_iter=2000, switch_eps=eps, switch_absolute=True)
+    assert rg.status == ro["status"] and rg.iterations == ro["iterations"]
+    assert np.array_equal(rg.history, ro["history"])
+    assert np.array_equal(rg.x.cpu().numpy(), ro["x"])
+    assert np.array_equal(rg.level_counts, ro["level_counts"])
+    lc = np.asarray(ro["level_counts"])
+    tp = np.asarray(oracle_tiles(orc, A).arrays()["TilePrec"])
+    base = np.bincount(tp, minlength=4)[:4]
+    assert any(not np.array_equal(row[:4], base) for row in lc[: ro["n_spmv"]])   # some SpMV changed tiles
