@@ -61,6 +61,14 @@ __device__ __forceinline__ unsigned hw_mask() { return (threadIdx.x & 16) ? 0xFF
 
 // min over the half-warp (mask m): one redux.sync
 __device__ __forceinline__ int hw_min_i(int v, unsigned m) { return (int)__reduce_min_sync(m, (unsigned)v); }
+// the same for a level (0..4) when all 32 lanes are present: two full-warp reductions, each half
+// feeding the neutral 4 into the other's (no per-half masks, no divergence checks)
+__device__ __forceinline__ int hw_min_level_full(int v) {
+    const bool upper = (threadIdx.x & 16) != 0;
+    const unsigned lo = __reduce_min_sync(0xffffffffu, upper ? 4u : (unsigned)v);
+    const unsigned hi = __reduce_min_sync(0xffffffffu, upper ? (unsigned)v : 4u);
+    return (int)(upper ? hi : lo);
+}
 
 // (tile column << 3) | e_t.   e_t = bypass | max_prec(floor, min_prec(TilePrec, level))
 template <bool DYN>

@@ -580,23 +580,24 @@ __global__ void __launch_bounds__(MAXT, 1) cg_persistent(SolveArgs a) {
                     }
                 };
                 load_px(t, pv, xv);
-                for (int64_t l0 = t; l0 < L; l0 += 4 * (int64_t)B) {
+                // warp-uniform trip count (the warp's first row decides), so that the levels are two
+                // full-warp reductions; rows past the CTA's range are masked per lane
+                const int64_t lane32 = t & 31;
+                for (int64_t l0 = t; l0 - lane32 < L; l0 += 4 * (int64_t)B) {
                     if (l0 + 4 * (int64_t)B < L) load_px(l0 + 4 * (int64_t)B, pn4, xn4);
 #pragma unroll
                     for (int q = 0; q < 4; ++q) {
                         const int64_t li = l0 + q * B, i = R0 + li;
-                        if (li < L) {                                // uniform per half-warp
-                            double pn = 0.0;
-                            if (li < nr) {
-                                const double rv = li < mu_cap ? MUs[li] : Rv[i];
-                                X[i] = __fma_rn(alpha, pv[q], xv[q]);
-                                pn = __fma_rn(beta, pv[q], rv);
-                                P[pv_idx(i)] = pn;
-                            }
-                            if (DYN) {
-                                const int lv = mfk::hw_min_i(li < nr ? mfk::level_of(pn, th) : 4, m);
-                                if ((i & 15) == 0) mfk::pv_set_level(P, i >> 4, lv);
-                            }
+                        double pn = 0.0;
+                        if (li < nr) {
+                            const double rv = li < mu_cap ? MUs[li] : Rv[i];
+                            X[i] = __fma_rn(alpha, pv[q], xv[q]);
+                            pn = __fma_rn(beta, pv[q], rv);
+                            P[pv_idx(i)] = pn;
+                        }
+                        if (DYN) {
+                            const int lv = mfk::hw_min_level_full(li < nr ? mfk::level_of(pn, th) : 4);
+                            if (li < L && (i & 15) == 0) mfk::pv_set_level(P, i >> 4, lv);
                         }
                     }
 #pragma unroll
