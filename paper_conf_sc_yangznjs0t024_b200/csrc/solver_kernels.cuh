@@ -848,14 +848,25 @@ __global__ void __launch_bounds__(MAXT, 1) bicgstab_persistent(SolveArgs a) {
             tm.tick(2);
             if (eta[0] == 0.0 || !isfinite(eta[0])) { status = MF_ERR_BREAKDOWN; break; }
             const double alpha = __ddiv_rn(rho, eta[0]);
-            // s = r - alpha mu (own rows, PV) + levels of s
-            for (int64_t li = t; li < nrp; li += B) {
-                const int64_t i = R0 + li;
-                double si = 0.0;
-                if (li < nr) { si = __fma_rn(-alpha, mu_at(li), Rv[i]); S[pv_idx(i)] = si; }
-                int lv = 0;
-                if (DYN) lv = mfk::hw_min_i(li < nr ? mfk::level_of(si, th) : 4, m);
-                if ((i & 15) == 0) mfk::pv_set_level(S, i >> 4, lv);
+            // s = r - alpha mu (own rows, PV) + levels of s: 4 rows per thread with their loads
+            // issued first, a warp-uniform trip count and full-warp level reductions
+            for (int64_t l0 = t; l0 - (t & 31) < nrp; l0 += 4 * (int64_t)B) {
+                double rv4[4], mv4[4];
+#pragma unroll
+                for (int q = 0; q < 4; ++q) {
+                    const int64_t li = l0 + q * B;
+                    rv4[q] = li < nr ? Rv[R0 + li] : 0.0;
+                    mv4[q] = li < nr ? mu_at(li) : 0.0;
+                }
+#pragma unroll
+                for (int q = 0; q < 4; ++q) {
+                    const int64_t li = l0 + q * B, i = R0 + li;
+                    double si = 0.0;
+                    if (li < nr) { si = __fma_rn(-alpha, mv4[q], rv4[q]); S[pv_idx(i)] = si; }
+                    int lv = 0;
+                    if (DYN) lv = mfk::hw_min_level_full(li < nr ? mfk::level_of(si, th) : 4);
+                    if (li < nrp && (i & 15) == 0) mfk::pv_set_level(S, i >> 4, lv);
+                }
             }
             publish(a, ++epoch);
             tm.tick(3);
@@ -934,14 +945,25 @@ __global__ void __launch_bounds__(MAXT, 1) bicgstab_persistent(SolveArgs a) {
             }
             const double beta = __dmul_rn(__ddiv_rn(rv[0], rho), __ddiv_rn(alpha, omega));
             rho = rv[0];
-            // p = r + beta (p - omega mu) (own rows, PV) + levels of p
-            for (int64_t li = t; li < nrp; li += B) {
-                const int64_t i = R0 + li;
-                double pn = 0.0;
-                if (li < nr) { pn = __fma_rn(beta, __fma_rn(-omega, mu_at(li), P[pv_idx(i)]), Rv[i]); P[pv_idx(i)] = pn; }
-                int lv = 0;
-                if (DYN) lv = mfk::hw_min_i(li < nr ? mfk::level_of(pn, th) : 4, m);
-                if ((i & 15) == 0) mfk::pv_set_level(P, i >> 4, lv);
+            // p = r + beta (p - omega mu) (own rows, PV) + levels of p (as the s update)
+            for (int64_t l0 = t; l0 - (t & 31) < nrp; l0 += 4 * (int64_t)B) {
+                double pv4[4], mv4[4], rv4[4];
+#pragma unroll
+                for (int q = 0; q < 4; ++q) {
+                    const int64_t li = l0 + q * B, i = R0 + li;
+                    pv4[q] = li < nr ? P[pv_idx(i)] : 0.0;
+                    mv4[q] = li < nr ? mu_at(li) : 0.0;
+                    rv4[q] = li < nr ? Rv[i] : 0.0;
+                }
+#pragma unroll
+                for (int q = 0; q < 4; ++q) {
+                    const int64_t li = l0 + q * B, i = R0 + li;
+                    double pn = 0.0;
+                    if (li < nr) { pn = __fma_rn(beta, __fma_rn(-omega, mv4[q], pv4[q]), rv4[q]); P[pv_idx(i)] = pn; }
+                    int lv = 0;
+                    if (DYN) lv = mfk::hw_min_level_full(li < nr ? mfk::level_of(pn, th) : 4);
+                    if (li < nrp && (i & 15) == 0) mfk::pv_set_level(P, i >> 4, lv);
+                }
             }
             publish(a, ++epoch);
             tm.tick(9);
