@@ -908,10 +908,10 @@ __global__ void __launch_bounds__(MAXT, 1) bicgstab_persistent(SolveArgs a) {
             if (omega == 0.0 || !isfinite(omega)) { status = MF_ERR_BREAKDOWN; break; }
             // x += alpha p + omega s ; r = s - omega theta ; partial (r, r0*), (r, r)
             double rv[2] = {0.0, 0.0};
-            for (int64_t l0 = t; l0 < nr; l0 += 2 * (int64_t)B) {
-                double sv[2], pv[2], xv[2], tv[2], hv[2];
+            for (int64_t l0 = t; l0 < nr; l0 += 4 * (int64_t)B) {
+                double sv[4], pv[4], xv[4], tv[4], hv[4];
 #pragma unroll
-                for (int q = 0; q < 2; ++q) {
+                for (int q = 0; q < 4; ++q) {
                     const int64_t li = l0 + q * B;
                     if (li < nr) {
                         const int64_t i = R0 + li;
@@ -920,7 +920,7 @@ __global__ void __launch_bounds__(MAXT, 1) bicgstab_persistent(SolveArgs a) {
                     }
                 }
 #pragma unroll
-                for (int q = 0; q < 2; ++q) {
+                for (int q = 0; q < 4; ++q) {
                     const int64_t li = l0 + q * B;
                     if (li < nr) {
                         const int64_t i = R0 + li;
