@@ -361,10 +361,26 @@ def dist_arm(args, rank, world):
     fn = dist.cg_solve if spec["solver"] == "cg" else dist.bicgstab_solve
     eps = spec.get("switch_eps")
 
+    # execution: auto (the device-initiated single kernel per rank when every rank is in one NVLink
+    # domain, else host-orchestrated).  If the first solve fails on any rank (watchdog, setup), all
+    # ranks switch to the host-orchestrated path (dist_mode 1) and the line says so.
+    sel = {"dist_mode": 0, "fallback": None}
+
     def step():
         D = dist.DistTileMatrix(comm, n, rb, re, rp, ci, va)
-        return D, fn(D, b, max_iter=spec["max_iter"], mode=mf.MODE_DYNAMIC, switch_eps=eps, history=False)
+        return D, fn(D, b, max_iter=spec["max_iter"], mode=mf.MODE_DYNAMIC, switch_eps=eps, history=False,
+                     dist_mode=sel["dist_mode"], watchdog_ms=30000)
 
+    try:
+        D, r = step()
+        ok, why = int(bool(r.converged)), "not converged"
+        D.close()
+    except mf.MFError as e:
+        ok, why = 0, str(e)[:200]
+    flag = torch.tensor([ok], dtype=torch.int32, device=dev)
+    td.all_reduce(flag, op=td.ReduceOp.MIN)
+    if int(flag.item()) == 0:
+        sel["dist_mode"], sel["fallback"] = 1, f"device-initiated kernel failed ({why}); host-orchestrated path"
     for _ in range(args.warmup):
         D, r = step()
         conv_launches = D.info()["convert_launches"]
@@ -401,7 +417,8 @@ def dist_arm(args, rank, world):
     for _ in range(args.steps):
         rpd, cid, vad, bd = (t.to(dev, non_blocking=True) for t in hp)
         D = dist.DistTileMatrix(comm, n, rb, re, rpd, cid, vad)
-        r = fn(D, bd, max_iter=spec["max_iter"], mode=mf.MODE_DYNAMIC, switch_eps=eps, history=False)
+        r = fn(D, bd, max_iter=spec["max_iter"], mode=mf.MODE_DYNAMIC, switch_eps=eps, history=False,
+               dist_mode=sel["dist_mode"], watchdog_ms=30000)
         xh.copy_(r.x, non_blocking=True)
         e2e_it += r.iterations
         D.close()
@@ -418,7 +435,8 @@ def dist_arm(args, rank, world):
                    "mode": "dynamic mixed (FP64/FP32/FP16/E4M3 tiles + bypass)",
                    "step": "per-rank conversion of its rows + one distributed solve",
                    "parallelism": f"row blocks over {world} GPUs (libmf: NCCL halo of the SpMV input + rank-ordered all-gathered partials)",
-                   "partition_rows": bnd, "l2": "inputs larger than L2 per step (whole solve)"},
+                   "partition_rows": bnd, "l2": "inputs larger than L2 per step (whole solve)",
+                   "dist_mode": "auto (device-initiated when available)" if sel["fallback"] is None else sel["fallback"]},
         "iterations": r.iterations,
         "solve_kernel_ms_rank0": round(statistics.mean(kms), 3),
         "halo_segments_rank0": halo["halo_segments"], "halo_bytes_per_exchange_rank0": halo["halo_segments"] * 144,
