@@ -341,6 +341,18 @@ __device__ __forceinline__ TsView ts_view(const unsigned char* slot, int blob_ca
     return v;
 }
 
+// the dynamic switch for 4 decoded values whose segment level lv exceeds their TilePrec q:
+// bypass -> 0; else RNE at e_t = min(lv, floor) when that is below q (range guard R19)
+struct D4 {
+    double a, b, c, d;
+};
+static __device__ __noinline__ D4 ts_lower4(D4 w, int lv, int floor_, int q) {
+    if (lv == BYP) return D4{0.0, 0.0, 0.0, 0.0};
+    const int e = min(lv, floor_);
+    if (e == q) return w;
+    return D4{round_to(w.a, e), round_to(w.b, e), round_to(w.c, e), round_to(w.d, e)};
+}
+
 // Decode of one warp's group of n columns at TilePrec Q (warp-uniform) into its buffer E: values
 // vb[0 .. 16n) -> E[slot0*16 ..), 4 values per lane per step, exact upcast.  Dynamic switch (Alg. 5
 // l.2-4, range guard R19): bypass -> 0, e_t below TilePrec -> RNE_{e_t}(stored).  Sticky variant
@@ -392,15 +404,9 @@ __device__ __forceinline__ void ts_decode_group(const TsView& v, const unsigned 
                         }
                 }
             } else if (lv > Q) {
-                if (lv == BYP) { w[0] = w[1] = w[2] = w[3] = 0.0; }
-                else {
-                    int e = lv;
-                    if (range_guard) e = min(e, (int)((g >> 16) & 3u));
-                    if (e != Q) {
-#pragma unroll
-                        for (int k = 0; k < 4; ++k) w[k] = round_to(w[k], e);
-                    }
-                }
+                // rare path out of line: keeps the hot decode loop small (instruction cache)
+                const D4 r = ts_lower4(D4{w[0], w[1], w[2], w[3]}, lv, range_guard ? (int)((g >> 16) & 3u) : 3, Q);
+                w[0] = r.a; w[1] = r.b; w[2] = r.c; w[3] = r.d;
             }
         }
         // the two 16-byte halves in a lane-rotated order: conflict-free shared stores
